@@ -1,0 +1,130 @@
+/*
+ * mcl.h -- C ABI of the B200-native MultiCL device-mapper search (libmcl.so).
+ *
+ * The operation (Aji, Pena, Balaji, Feng, IEEE CLUSTER 2015, SS V.A
+ * "Device Mapper": "apply a simple dynamic programming approach to determine the ideal
+ * queue-device mapping that minimizes the concurrent execution time"; PAPER.md
+ * L2106-2118, SS VI.B.1: the scheduler "computes the aggregate cost metric from the data
+ * transfer and kernel execution costs"), per scheduling epoch e:
+ *
+ *   C[q][d]   = cost_kernel[e][q][d] + cost_xfer[e][q][d]        (integer ns)
+ *   m         = sum_q d_q * D^(Q-1-q)     mapping index, queue 0 most significant digit
+ *   L_d(m)    = sum over queues q placed on device d of C[q][d]   (queues on one device
+ *               serialise; an idle device has load 0)
+ *   ms(m)     = max_d L_d(m)              (distinct devices run concurrently)
+ *   result    = the LOWEST index m* among the mappings with minimal ms, its digits and ms.
+ *
+ * All D^Q mappings are scored exhaustively on the GPU (hand-written sm_100a kernels).
+ * Costs are exact unsigned integers, so results are bit-exact (no tolerance).
+ *
+ * Threading: a handle is used by one host thread at a time. Different handles are
+ * independent. All calls are synchronous: they return after every output is written.
+ */
+#ifndef MCL_H_
+#define MCL_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct mcl_mapper mcl_mapper_t; /* opaque; owned by the library */
+
+typedef enum {
+  MCL_OK = 0,
+  MCL_E_INVAL = -1,  /* NULL required pointer, Q == 0, D == 0, D > 16, Q > 32, bad config */
+  MCL_E_RANGE = -2,  /* D^Q > 2^48, or some cost entry >= 2^48 */
+  MCL_E_CUDA = -3,   /* a CUDA runtime call failed (see mcl_last_error_string) */
+  MCL_E_NCCL = -4,   /* an NCCL call failed, or NCCL could not be loaded */
+  MCL_E_NOMEM = -5   /* device / pinned-host allocation failed */
+} mcl_status_t;
+
+#define MCL_MAX_QUEUES 32
+#define MCL_MAX_DEVICES 16
+#define MCL_MAX_ENTRY_BITS 48 /* every cost entry must be < 2^48 */
+#define MCL_MAX_INDEX_BITS 48 /* D^Q must be <= 2^48 */
+
+typedef struct {
+  int device;      /* CUDA device ordinal this handle runs on                            */
+  void* stream;    /* cudaStream_t to run on; NULL = a non-blocking stream owned by the handle */
+  void* nccl_comm; /* ncclComm_t (e.g. torch ProcessGroupNCCL._comm_ptr()) or NULL        */
+  int rank;        /* this process's shard, 0 <= rank < world                             */
+  int world;       /* number of shards; 0 or 1 = the whole index space                    */
+} mcl_config_t;
+
+/*
+ * Create a mapper handle on cfg->device.
+ *   cfg  : required. With nccl_comm == NULL and world > 1 the handle searches only shard
+ *          `rank` of every epoch's index space and returns that shard's local argmin (a
+ *          sub-range search; used to test sharding on one GPU). With nccl_comm != NULL,
+ *          rank/world must equal the communicator's and every mcl_map_queues call is
+ *          COLLECTIVE (see below).
+ *   out  : receives the handle. The handle owns its scratch (per-CTA partial results,
+ *          staging buffers, a mapped host status word), allocated here and grown on demand.
+ * Errors: MCL_E_INVAL (NULL pointers, bad rank/world, bad device), MCL_E_CUDA, MCL_E_NOMEM,
+ *         MCL_E_NCCL (nccl_comm given but libnccl could not be resolved).
+ */
+mcl_status_t mcl_mapper_create(const mcl_config_t* cfg, mcl_mapper_t** out);
+
+/*
+ * Find the minimum-makespan queue->device mapping of every epoch.
+ *   Q, D          : queues and devices; 1 <= Q <= 32, 1 <= D <= 16, D^Q <= 2^48.
+ *   epochs        : number of independent epochs E (0 = no-op, returns MCL_OK).
+ *   cost_kernel   : [E][Q][D] uint64, C order: per-queue aggregate kernel time on each
+ *                   device (the kernel profiler's output).
+ *   cost_xfer     : [E][Q][D] uint64, C order: cost of moving the queue's buffers to each
+ *                   device (derived from the device profiles).
+ *   mapping_index : [E] uint64 out: lowest index of an optimal mapping.
+ *   mapping       : [E][Q] uint8 out: its device per queue (digit q of the index), or NULL.
+ *   makespan      : [E] uint64 out: its makespan, in the same unit as the costs.
+ * Every pointer may be device memory (the fast path: no copies) or host memory (pageable
+ * or pinned; detected with cudaPointerGetAttributes and staged through handle-owned device
+ * buffers inside the call). The caller owns all buffers; the library never frees them.
+ * Inputs are only read; outputs are fully written on MCL_OK and unspecified on error.
+ *
+ * Sharding: the index space [0, D^Q) of each epoch is cut into `world` contiguous ranges
+ * [floor(r*N/G), floor((r+1)*N/G)) (in whole blocks of the innermost digits). With a
+ * communicator, each rank searches its range and one ncclAllReduce(MIN, uint64) over the
+ * packed key (makespan << index_bits | index) combines them, so every rank receives the
+ * identical global result (bit-identical for every world size). When the makespan does not
+ * fit beside the index in 64 bits, a two-step reduction (min makespan, then min index
+ * among the ranks holding it) is used instead. All ranks must pass identical inputs.
+ *
+ * Errors: MCL_E_INVAL (NULL required pointer, Q/D out of bounds), MCL_E_RANGE (D^Q > 2^48
+ *         or an entry >= 2^48, detected on the device), MCL_E_CUDA, MCL_E_NCCL.
+ */
+mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                            const uint64_t* cost_kernel, const uint64_t* cost_xfer,
+                            uint64_t* mapping_index, uint8_t* mapping, uint64_t* makespan);
+
+/* Destroy a handle (NULL-safe). Frees the handle's scratch; never the caller's buffers and
+   never the NCCL communicator (its owner, e.g. the torch process group, keeps it). */
+void mcl_mapper_destroy(mcl_mapper_t* h);
+
+/* Static text for a status code. */
+const char* mcl_status_string(mcl_status_t s);
+
+/* Text of the last CUDA/NCCL error seen on this handle ("" if none). Valid until the next
+   call on the handle. NULL handle: the last creation error of this thread. */
+const char* mcl_last_error_string(const mcl_mapper_t* h);
+
+/*
+ * Introspection for tests and benchmarks (not needed to use the mapper).
+ * mcl_last_launch_info fills, for the most recent successful mcl_map_queues call on h:
+ *   info[0] = kernel path id (1 = register-blocked u32 search, 2 = register-blocked u64
+ *             search, 3 = generic search, 4 = small batched (thread per epoch))
+ *   info[1] = number of kernels launched by the call, info[2] = CTAs of the main kernel,
+ *   info[3] = threads per CTA, info[4] = 1 if an NCCL all-reduce ran,
+ *   info[5] = index bits of the packed key, info[6] = 1 if the two-step reduce ran.
+ */
+mcl_status_t mcl_last_launch_info(const mcl_mapper_t* h, int64_t info[8]);
+
+/* Library version string "mcl <major>.<minor> sm_100a". */
+const char* mcl_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* MCL_H_ */

@@ -1,0 +1,58 @@
+/*
+ * mcl_ext.h -- measurement and communicator helpers of libmcl.so (C ABI).
+ *
+ * Not needed to use the mapper (that is include/mcl.h); used by bench.py and the tests to
+ * time the search kernel on its own stream, to measure the integer-pipe peak that bounds it
+ * (SURVEY.md SS8(d) roofline, component N7), and to build an NCCL communicator without a
+ * torch process group.
+ */
+#ifndef MCL_EXT_H_
+#define MCL_EXT_H_
+
+#include <stdint.h>
+
+#include "mcl.h"
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* Enable (1) / disable (0) CUDA-event timing of the main search kernel of every
+   mcl_map_queues call on h. Events are recorded on the stream the kernel is launched on. */
+mcl_status_t mcl_set_timing(mcl_mapper_t* h, int enable);
+
+/* Device time in milliseconds of the main search kernel of the last call (timing enabled),
+   and of the whole device-side sequence of that call (search + reduce + decode). */
+mcl_status_t mcl_last_kernel_time(const mcl_mapper_t* h, float* kernel_ms, float* call_ms);
+
+/*
+ * Integer-pipe throughput probe on `device` (op: 0 = 2-input min/max VIMNMX, 1 = 3-input
+ * VIMNMX3, 2 = IADD3, 3 = IMAD, 4 = VIMNMX3 and IMAD interleaved). Runs for ~1 ms at full
+ * occupancy and reports lane-operations per second, lane-operations per SM clock, and the
+ * effective SM clock in MHz over the run. Synchronous. Any output pointer may be NULL.
+ */
+mcl_status_t mcl_probe_int_rate(int device, int op, double* lane_ops_per_s,
+                                double* lane_ops_per_clk_sm, double* eff_mhz);
+
+/* Testing aid: force the kernel of later mcl_map_queues calls on h. path: 0 = automatic
+   (default), 1 = register-blocked (u32 loads, falls back to 64-bit when a bound needs it),
+   2 = register-blocked with 64-bit loads, 3 = generic, 4 = small batched. A path that does
+   not support (Q, D) or the handle's sharding makes the call fail with MCL_E_INVAL. */
+mcl_status_t mcl_force_path(mcl_mapper_t* h, int path);
+
+/* Number of SMs of `device` (for roofline bookkeeping). */
+mcl_status_t mcl_device_sms(int device, int* sms);
+
+/* NCCL communicator helpers (libnccl.so.2 is resolved at run time, reusing the copy
+   torch already loaded when there is one). The unique id is 128 opaque bytes that rank 0
+   creates and every rank passes to mcl_comm_init; the communicator belongs to the caller
+   and is released with mcl_comm_destroy. */
+mcl_status_t mcl_comm_unique_id(uint8_t id_out[128]);
+mcl_status_t mcl_comm_init(int device, int world, int rank, const uint8_t id[128], void** comm_out);
+mcl_status_t mcl_comm_destroy(void* comm);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* MCL_EXT_H_ */

@@ -1,0 +1,105 @@
+// kernels.h -- internal launch interface between the C-ABI host code (mcl.cpp) and the
+// sm_100a kernels. Not part of the public ABI (that is include/mcl.h).
+#pragma once
+#include <cstddef>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace mcl {
+
+// Lexicographic (makespan, mapping index) candidate; see common.cuh.
+struct Cand {
+  uint64_t ms;
+  uint64_t idx;
+};
+
+// Outputs of one launch, per epoch.
+struct EpochOut {
+  uint64_t* index;      // [E]
+  uint64_t* makespan;   // [E]
+  uint8_t* mapping;     // [E][Q] or nullptr
+  uint64_t* key;        // [E] packed key for the cross-GPU reduce, or nullptr (single GPU)
+  uint64_t* pair;       // [E][2] (ms, idx) for the two-step cross-GPU reduce, or nullptr
+};
+
+constexpr int kBlockedMaxD = 8;  // register-blocked kernel instantiated for D = 2..8
+
+// Register-blocked search (search_blocked.cu).
+struct BlockedArgs {
+  uint32_t Q, D;
+  uint64_t E;
+  const uint64_t* K;
+  const uint64_t* X;
+  uint64_t rlo, rhi;  // this rank's block range [rlo, rhi), blocks of D^3 mappings
+  Cand* scratch;      // [E][cpe]
+  uint32_t* done;     // [E], zero on entry, self-resetting
+  EpochOut out;
+  int ibits;
+  volatile uint32_t* flags;
+  uint32_t one;
+  size_t off_red, off_dig;
+};
+
+// ceil(log2(N)): bits of the packed key's index field (N >= 1).
+inline int index_bits_host(uint64_t N) {
+  int b = 0;
+  while (b < 64 && ((N - 1) >> b)) ++b;
+  return b;
+}
+
+bool blocked_supported(uint32_t Q, uint32_t D);
+int blocked_ctas_per_sm(uint32_t D, bool wide, int threads, size_t smem);
+size_t blocked_smem_bytes(uint32_t Q, uint32_t D, bool wide, int threads, size_t* off_red,
+                          size_t* off_dig);
+cudaError_t launch_blocked(const BlockedArgs& a, bool wide, dim3 grid, int threads, size_t smem,
+                           cudaStream_t st);
+
+// Generic search (search_generic.cu): any Q <= 32, D <= 16, 64-bit loads.
+struct GenericArgs {
+  uint32_t Q, D;
+  uint64_t E;
+  const uint64_t* K;
+  const uint64_t* X;
+  uint64_t rlo, rhi;  // this rank's range in ROWS of D mappings (last digit varies in a row)
+  Cand* scratch;
+  uint32_t* done;
+  EpochOut out;
+  int ibits;
+  volatile uint32_t* flags;
+};
+size_t generic_smem_bytes(uint32_t Q, uint32_t D, int threads);
+cudaError_t launch_generic(const GenericArgs& a, dim3 grid, int threads, size_t smem,
+                           cudaStream_t st);
+
+// Small batched search (search_small.cu): one thread per epoch, tiles staged in shared
+// memory by cp.async.bulk (TMA bulk copy). Instantiated for a few (Q, D) shapes.
+struct SmallArgs {
+  uint32_t Q, D;
+  uint64_t E;
+  const uint64_t* K;
+  const uint64_t* X;
+  uint64_t* index;
+  uint64_t* makespan;
+  uint8_t* mapping;
+  volatile uint32_t* flags;
+};
+bool small_supported(uint32_t Q, uint32_t D);
+cudaError_t launch_small(const SmallArgs& a, int num_sms, cudaStream_t st, int* grid_out,
+                         int* threads_out);
+
+// Multi-GPU epilogues (reduce.cu).
+cudaError_t launch_decode_key(const uint64_t* key, uint64_t E, uint32_t Q, uint32_t D, int ibits,
+                              uint64_t* index, uint64_t* makespan, uint8_t* mapping,
+                              cudaStream_t st);
+cudaError_t launch_pair_candidates(const uint64_t* pair, const uint64_t* gms, uint64_t E,
+                                   uint64_t* cand, cudaStream_t st);
+cudaError_t launch_decode_pair(const uint64_t* gms, const uint64_t* gidx, uint64_t E, uint32_t Q,
+                               uint32_t D, uint64_t* index, uint64_t* makespan, uint8_t* mapping,
+                               cudaStream_t st);
+cudaError_t launch_extract_ms(const uint64_t* pair, uint64_t E, uint64_t* ms, cudaStream_t st);
+
+// ALU throughput probe (probe.cu), SURVEY N7.
+cudaError_t probe_alu(int op, int sms, cudaStream_t st, double* lane_ops_per_s,
+                      double* lane_ops_per_clk_sm, double* eff_mhz);
+
+}  // namespace mcl

@@ -1,0 +1,622 @@
+// mcl.cpp -- host side of libmcl.so: the C ABI of include/mcl.h and include/mcl_ext.h.
+//
+// Validation, pointer classification (device buffers are used in place, host buffers are
+// staged through handle-owned device memory), kernel selection, the shard range of this
+// rank, the cross-GPU all-reduce (NCCL resolved at run time with dlopen, so the library
+// has no link-time NCCL dependency and reuses the copy torch already loaded), and the
+// status word the kernels raise (host-mapped pinned memory, read after the stream sync).
+//
+// There is no CPU fallback: every mapping is scored by the CUDA kernels in this library;
+// without a usable CUDA device mcl_mapper_create fails with MCL_E_CUDA.
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <string>
+
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include "../../include/mcl.h"
+#include "../../include/mcl_ext.h"
+#include "kernels.h"
+
+namespace {
+
+using mcl::Cand;
+
+// ---------------------------------------------------------------- NCCL (dlopen) -------
+struct NcclApi {
+  bool ok = false;
+  std::string err;
+  ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                            cudaStream_t) = nullptr;
+  const char* (*GetErrorString)(ncclResult_t) = nullptr;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  ncclResult_t (*CommCount)(const ncclComm_t, int*) = nullptr;
+  ncclResult_t (*CommUserRank)(const ncclComm_t, int*) = nullptr;
+};
+
+NcclApi load_nccl() {
+  NcclApi api;
+  void* lib = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);  // torch's copy, if loaded
+  if (!lib) lib = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+  if (!lib) lib = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+  if (!lib) {
+    const char* e = dlerror();
+    api.err = std::string("cannot load libnccl.so.2: ") + (e ? e : "?");
+    return api;
+  }
+#define MCL_SYM(field, name)                                                   \
+  api.field = reinterpret_cast<decltype(api.field)>(dlsym(lib, name));         \
+  if (!api.field) {                                                            \
+    api.err = std::string("libnccl is missing ") + name;                       \
+    return api;                                                                \
+  }
+  MCL_SYM(AllReduce, "ncclAllReduce")
+  MCL_SYM(GetErrorString, "ncclGetErrorString")
+  MCL_SYM(GetUniqueId, "ncclGetUniqueId")
+  MCL_SYM(CommInitRank, "ncclCommInitRank")
+  MCL_SYM(CommDestroy, "ncclCommDestroy")
+  MCL_SYM(CommCount, "ncclCommCount")
+  MCL_SYM(CommUserRank, "ncclCommUserRank")
+#undef MCL_SYM
+  api.ok = true;
+  return api;
+}
+
+NcclApi& nccl() {
+  static NcclApi api = load_nccl();
+  return api;
+}
+
+thread_local std::string g_create_err;
+
+// ---------------------------------------------------------------- device buffers ------
+struct DevBuf {
+  void* p = nullptr;
+  size_t cap = 0;
+  cudaError_t ensure(size_t bytes, bool zero = false) {
+    if (bytes <= cap) return cudaSuccess;
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+    size_t want = std::max<size_t>(bytes, 256);
+    cudaError_t e = cudaMalloc(&p, want);
+    if (e != cudaSuccess) return e;
+    cap = want;
+    if (zero) return cudaMemset(p, 0, want);
+    return cudaSuccess;
+  }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+  }
+};
+
+bool mul_overflow_pow(uint32_t D, uint32_t Q, uint64_t limit, uint64_t* out) {
+  uint64_t n = 1;
+  for (uint32_t q = 0; q < Q; ++q) {
+    if (n > limit / D) return true;
+    n *= D;
+  }
+  *out = n;
+  return false;
+}
+
+}  // namespace
+
+struct mcl_mapper {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  ncclComm_t comm = nullptr;
+  int rank = 0, world = 1;
+  int num_sms = 148;
+  DevBuf scratch;          // Cand per (epoch, CTA) when an epoch spans several CTAs
+  DevBuf done;             // uint32 per epoch, zero between calls
+  DevBuf key, pair, gms, cand;
+  DevBuf in_k, in_x, out_idx, out_ms, out_map;  // staging for host pointers
+  uint32_t* flags_host = nullptr;               // host-mapped status word
+  uint32_t* flags_dev = nullptr;
+  bool timing = false;
+  int force_path = 0;
+  cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+  float kernel_ms = 0.f, call_ms = 0.f;
+  int64_t info[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  std::string last_err;
+};
+
+namespace {
+
+mcl_status_t cuda_fail(mcl_mapper* h, cudaError_t e, const char* what) {
+  std::string msg = std::string(what) + ": " + cudaGetErrorString(e);
+  if (h) h->last_err = msg; else g_create_err = msg;
+  return (e == cudaErrorMemoryAllocation) ? MCL_E_NOMEM : MCL_E_CUDA;
+}
+
+mcl_status_t nccl_fail(mcl_mapper* h, ncclResult_t r, const char* what) {
+  h->last_err = std::string(what) + ": " + (nccl().GetErrorString ? nccl().GetErrorString(r) : "?");
+  return MCL_E_NCCL;
+}
+
+#define MCL_CUDA(h, expr, what)                      \
+  do {                                               \
+    cudaError_t _e = (expr);                         \
+    if (_e != cudaSuccess) return cuda_fail(h, _e, what); \
+  } while (0)
+
+// Is `p` usable in place by kernels on h->device?
+mcl_status_t classify(mcl_mapper* h, const void* p, bool* on_device) {
+  cudaPointerAttributes at;
+  cudaError_t e = cudaPointerGetAttributes(&at, p);
+  if (e != cudaSuccess) {  // unregistered host memory on older runtimes
+    cudaGetLastError();
+    *on_device = false;
+    return MCL_OK;
+  }
+  if (at.type == cudaMemoryTypeDevice) {
+    if (at.device != h->device) {
+      h->last_err = "device pointer belongs to another CUDA device";
+      return MCL_E_INVAL;
+    }
+    *on_device = true;
+  } else if (at.type == cudaMemoryTypeManaged) {
+    *on_device = true;
+  } else {
+    *on_device = false;  // pageable or pinned host memory: staged
+  }
+  return MCL_OK;
+}
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+// Shard [0, units) of every epoch into `world` contiguous ranges; this rank's range.
+void shard(uint64_t units, int rank, int world, uint64_t* lo, uint64_t* hi) {
+  if (world <= 1) {
+    *lo = 0;
+    *hi = units;
+    return;
+  }
+  // exact floor(r * units / world) without overflow (units <= 2^48, world <= 2^15)
+  *lo = (uint64_t)(((__uint128_t)units * rank) / world);
+  *hi = (uint64_t)(((__uint128_t)units * (rank + 1)) / world);
+}
+
+// CTAs per epoch and threads per CTA for `units` work units per epoch in this rank.
+void size_grid(mcl_mapper* h, uint64_t E, uint64_t units, int ctas_per_sm, int threads,
+               dim3* grid) {
+  const uint64_t slots = (uint64_t)h->num_sms * std::max(1, ctas_per_sm);
+  uint64_t cpe = 1;
+  if (E < slots) {
+    cpe = (slots + E - 1) / E;
+    const uint64_t useful = std::max<uint64_t>(1, (units + threads - 1) / threads);
+    cpe = std::min(cpe, useful);
+    if (cpe > 65535) cpe = 65535;
+  }
+  grid->x = (unsigned)cpe;
+  grid->y = (unsigned)std::min<uint64_t>(E, 65535);
+  grid->z = 1;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* mcl_version(void) { return "mcl 0.1 sm_100a"; }
+
+const char* mcl_status_string(mcl_status_t s) {
+  switch (s) {
+    case MCL_OK: return "MCL_OK: success";
+    case MCL_E_INVAL: return "MCL_E_INVAL: invalid argument";
+    case MCL_E_RANGE: return "MCL_E_RANGE: D^Q > 2^48 or a cost entry >= 2^48";
+    case MCL_E_CUDA: return "MCL_E_CUDA: CUDA runtime error";
+    case MCL_E_NCCL: return "MCL_E_NCCL: NCCL error";
+    case MCL_E_NOMEM: return "MCL_E_NOMEM: out of memory";
+  }
+  return "unknown mcl status";
+}
+
+const char* mcl_last_error_string(const mcl_mapper_t* h) {
+  return h ? h->last_err.c_str() : g_create_err.c_str();
+}
+
+mcl_status_t mcl_mapper_create(const mcl_config_t* cfg, mcl_mapper_t** out) {
+  g_create_err.clear();
+  if (!cfg || !out) return MCL_E_INVAL;
+  *out = nullptr;
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess) return cuda_fail(nullptr, e, "cudaGetDeviceCount");
+  if (cfg->device < 0 || cfg->device >= ndev) {
+    g_create_err = "device ordinal out of range";
+    return MCL_E_INVAL;
+  }
+  const int world = cfg->world <= 0 ? 1 : cfg->world;
+  if (cfg->rank < 0 || cfg->rank >= world || world > 32768) {
+    g_create_err = "rank/world out of range";
+    return MCL_E_INVAL;
+  }
+  if (cfg->nccl_comm) {
+    if (!nccl().ok) {
+      g_create_err = nccl().err;
+      return MCL_E_NCCL;
+    }
+    int n = 0, r = 0;
+    if (nccl().CommCount((ncclComm_t)cfg->nccl_comm, &n) != ncclSuccess ||
+        nccl().CommUserRank((ncclComm_t)cfg->nccl_comm, &r) != ncclSuccess) {
+      g_create_err = "invalid NCCL communicator";
+      return MCL_E_NCCL;
+    }
+    if (n != world || r != cfg->rank) {
+      g_create_err = "rank/world do not match the NCCL communicator";
+      return MCL_E_INVAL;
+    }
+  }
+  DeviceGuard g(cfg->device);
+  mcl_mapper* h = new mcl_mapper();
+  h->device = cfg->device;
+  h->comm = (ncclComm_t)cfg->nccl_comm;
+  h->rank = cfg->rank;
+  h->world = world;
+  auto fail = [&](cudaError_t err, const char* what) {
+    mcl_status_t s = cuda_fail(nullptr, err, what);
+    mcl_mapper_destroy(h);
+    return s;
+  };
+  e = cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, h->device);
+  if (e != cudaSuccess) return fail(e, "cudaDeviceGetAttribute");
+  if (cfg->stream) {
+    h->stream = (cudaStream_t)cfg->stream;
+  } else {
+    e = cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking);
+    if (e != cudaSuccess) return fail(e, "cudaStreamCreate");
+    h->own_stream = true;
+  }
+  e = cudaHostAlloc((void**)&h->flags_host, 64, cudaHostAllocMapped);
+  if (e != cudaSuccess) return fail(e, "cudaHostAlloc(flags)");
+  std::memset(h->flags_host, 0, 64);
+  e = cudaHostGetDevicePointer((void**)&h->flags_dev, h->flags_host, 0);
+  if (e != cudaSuccess) return fail(e, "cudaHostGetDevicePointer");
+  for (auto& ev : h->ev) {
+    e = cudaEventCreate(&ev);
+    if (e != cudaSuccess) return fail(e, "cudaEventCreate");
+  }
+  e = h->done.ensure(4096 * sizeof(uint32_t), true);
+  if (e != cudaSuccess) return fail(e, "cudaMalloc(done)");
+  *out = h;
+  return MCL_OK;
+}
+
+void mcl_mapper_destroy(mcl_mapper_t* h) {
+  if (!h) return;
+  {
+    DeviceGuard g(h->device);
+    if (h->stream) cudaStreamSynchronize(h->stream);
+    for (DevBuf* b : {&h->scratch, &h->done, &h->key, &h->pair, &h->gms, &h->cand, &h->in_k,
+                      &h->in_x, &h->out_idx, &h->out_ms, &h->out_map})
+      b->release();
+    if (h->flags_host) cudaFreeHost(h->flags_host);
+    for (auto& ev : h->ev)
+      if (ev) cudaEventDestroy(ev);
+    if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
+  }
+  delete h;
+}
+
+mcl_status_t mcl_last_launch_info(const mcl_mapper_t* h, int64_t info[8]) {
+  if (!h || !info) return MCL_E_INVAL;
+  for (int i = 0; i < 8; ++i) info[i] = h->info[i];
+  return MCL_OK;
+}
+
+mcl_status_t mcl_set_timing(mcl_mapper_t* h, int enable) {
+  if (!h) return MCL_E_INVAL;
+  h->timing = enable != 0;
+  return MCL_OK;
+}
+
+mcl_status_t mcl_force_path(mcl_mapper_t* h, int path) {
+  if (!h || path < 0 || path > 4) return MCL_E_INVAL;
+  h->force_path = path;
+  return MCL_OK;
+}
+
+mcl_status_t mcl_last_kernel_time(const mcl_mapper_t* h, float* kernel_ms, float* call_ms) {
+  if (!h) return MCL_E_INVAL;
+  if (kernel_ms) *kernel_ms = h->kernel_ms;
+  if (call_ms) *call_ms = h->call_ms;
+  return MCL_OK;
+}
+
+mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                            const uint64_t* cost_kernel, const uint64_t* cost_xfer,
+                            uint64_t* mapping_index, uint8_t* mapping, uint64_t* makespan) {
+  if (!h) return MCL_E_INVAL;
+  h->last_err.clear();
+  if (Q == 0 || D == 0 || Q > MCL_MAX_QUEUES || D > MCL_MAX_DEVICES) {
+    h->last_err = "Q must be in [1, 32] and D in [1, 16]";
+    return MCL_E_INVAL;
+  }
+  uint64_t N = 0;
+  if (mul_overflow_pow(D, Q, 1ull << MCL_MAX_INDEX_BITS, &N)) {
+    h->last_err = "D^Q exceeds 2^48";
+    return MCL_E_RANGE;
+  }
+  if (epochs == 0) return MCL_OK;
+  if (!cost_kernel || !cost_xfer || !mapping_index || !makespan) {
+    h->last_err = "NULL required pointer";
+    return MCL_E_INVAL;
+  }
+  if (epochs > (1ull << 40) / ((uint64_t)Q * D)) {
+    h->last_err = "epochs too large";
+    return MCL_E_INVAL;
+  }
+  DeviceGuard g(h->device);
+  // With a communicator the call is collective (a 1-rank communicator exercises the same
+  // packed-key all-reduce path on a single GPU).
+  const bool multi = h->comm != nullptr;
+
+  // ---- where do the buffers live? host buffers are staged through device memory ----
+  bool dk, dx, di, dm, dmap = true;
+  mcl_status_t st;
+  if ((st = classify(h, cost_kernel, &dk)) != MCL_OK) return st;
+  if ((st = classify(h, cost_xfer, &dx)) != MCL_OK) return st;
+  if ((st = classify(h, mapping_index, &di)) != MCL_OK) return st;
+  if ((st = classify(h, makespan, &dm)) != MCL_OK) return st;
+  if (mapping && (st = classify(h, mapping, &dmap)) != MCL_OK) return st;
+  const size_t in_bytes = (size_t)epochs * Q * D * sizeof(uint64_t);
+  const uint64_t* K = cost_kernel;
+  const uint64_t* X = cost_xfer;
+  uint64_t* o_idx = mapping_index;
+  uint64_t* o_ms = makespan;
+  uint8_t* o_map = mapping;
+  cudaStream_t s = h->stream;
+  if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[2], s), "cudaEventRecord");
+  if (!dk) {
+    MCL_CUDA(h, h->in_k.ensure(in_bytes), "cudaMalloc(staging)");
+    MCL_CUDA(h, cudaMemcpyAsync(h->in_k.p, cost_kernel, in_bytes, cudaMemcpyHostToDevice, s), "H2D");
+    K = (const uint64_t*)h->in_k.p;
+  }
+  if (!dx) {
+    MCL_CUDA(h, h->in_x.ensure(in_bytes), "cudaMalloc(staging)");
+    MCL_CUDA(h, cudaMemcpyAsync(h->in_x.p, cost_xfer, in_bytes, cudaMemcpyHostToDevice, s), "H2D");
+    X = (const uint64_t*)h->in_x.p;
+  }
+  if (!di) {
+    MCL_CUDA(h, h->out_idx.ensure(epochs * 8), "cudaMalloc(staging)");
+    o_idx = (uint64_t*)h->out_idx.p;
+  }
+  if (!dm) {
+    MCL_CUDA(h, h->out_ms.ensure(epochs * 8), "cudaMalloc(staging)");
+    o_ms = (uint64_t*)h->out_ms.p;
+  }
+  if (mapping && !dmap) {
+    MCL_CUDA(h, h->out_map.ensure(epochs * Q), "cudaMalloc(staging)");
+    o_map = (uint8_t*)h->out_map.p;
+  }
+
+  const int ibits = mcl::index_bits_host(N);
+  mcl::EpochOut out{o_idx, o_ms, o_map, nullptr, nullptr};
+  if (multi) {
+    MCL_CUDA(h, h->key.ensure(epochs * 8), "cudaMalloc(key)");
+    MCL_CUDA(h, h->pair.ensure(epochs * 16), "cudaMalloc(pair)");
+    out.key = (uint64_t*)h->key.p;
+    out.pair = (uint64_t*)h->pair.p;
+  }
+  MCL_CUDA(h, h->done.ensure(epochs * sizeof(uint32_t), true), "cudaMalloc(done)");
+
+  // ---- choose the kernel ----
+  const bool shard_mode = h->world > 1;  // NCCL collective or single-GPU shard test
+  int path;
+  if (!shard_mode && !multi && mcl::small_supported(Q, D)) path = 4;
+  else if (mcl::blocked_supported(Q, D)) path = 1;
+  else path = 3;
+  if (h->force_path) {
+    const int f = h->force_path;
+    const bool ok = (f == 3) || ((f == 1 || f == 2) && mcl::blocked_supported(Q, D)) ||
+                    (f == 4 && !shard_mode && !multi && mcl::small_supported(Q, D));
+    if (!ok) {
+      h->last_err = "forced kernel path does not support this shape / sharding";
+      return MCL_E_INVAL;
+    }
+    path = f;
+  }
+
+  int nlaunch = 0;
+  for (int attempt = 0; attempt < 2; ++attempt) {
+    *(volatile uint32_t*)h->flags_host = 0;
+    nlaunch = 0;
+    dim3 grid(1, 1, 1);
+    int threads = 0;
+    if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[0], s), "cudaEventRecord");
+    if (path == 4) {
+      mcl::SmallArgs a{Q, D, epochs, K, X, o_idx, o_ms, o_map, h->flags_dev};
+      int gx = 0;
+      MCL_CUDA(h, mcl::launch_small(a, h->num_sms, s, &gx, &threads), "search_small launch");
+      grid.x = gx;
+    } else if (path == 1 || path == 2) {
+      const bool wide = (path == 2);
+      const uint64_t nb = N / ((uint64_t)D * D * D);
+      uint64_t lo, hi;
+      shard(nb, h->rank, h->world, &lo, &hi);
+      // batched epochs: smaller CTAs so every thread still walks >= 16 blocks
+      threads = 256;
+      if (epochs > 1) {
+        const uint64_t per_epoch = hi - lo;
+        while (threads > 32 && per_epoch / threads < 16) threads >>= 1;
+      }
+      mcl::BlockedArgs a{};
+      a.Q = Q; a.D = D; a.E = epochs; a.K = K; a.X = X; a.rlo = lo; a.rhi = hi;
+      a.out = out; a.ibits = ibits; a.flags = h->flags_dev; a.one = 1;
+      const size_t smem = mcl::blocked_smem_bytes(Q, D, wide, threads, &a.off_red, &a.off_dig);
+      int occ = mcl::blocked_ctas_per_sm(D, wide, threads, smem);
+      size_grid(h, epochs, hi - lo, occ, threads, &grid);
+      if (grid.x > 1) {
+        MCL_CUDA(h, h->scratch.ensure((size_t)epochs * grid.x * sizeof(Cand)), "cudaMalloc(scratch)");
+        a.scratch = (Cand*)h->scratch.p;
+      }
+      a.done = (uint32_t*)h->done.p;
+      MCL_CUDA(h, mcl::launch_blocked(a, wide, grid, threads, smem, s), "search_blocked launch");
+    } else {
+      const uint64_t rows = N / D;
+      uint64_t lo, hi;
+      shard(rows, h->rank, h->world, &lo, &hi);
+      threads = 128;
+      if (epochs > 1) {
+        while (threads > 32 && (hi - lo) / threads < 16) threads >>= 1;
+      }
+      mcl::GenericArgs a{};
+      a.Q = Q; a.D = D; a.E = epochs; a.K = K; a.X = X; a.rlo = lo; a.rhi = hi;
+      a.out = out; a.ibits = ibits; a.flags = h->flags_dev;
+      const size_t smem = mcl::generic_smem_bytes(Q, D, threads);
+      size_grid(h, epochs, hi - lo, 8, threads, &grid);
+      if (grid.x > 1) {
+        MCL_CUDA(h, h->scratch.ensure((size_t)epochs * grid.x * sizeof(Cand)), "cudaMalloc(scratch)");
+        a.scratch = (Cand*)h->scratch.p;
+      }
+      a.done = (uint32_t*)h->done.p;
+      MCL_CUDA(h, mcl::launch_generic(a, grid, threads, smem, s), "search_generic launch");
+    }
+    ++nlaunch;
+    if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[1], s), "cudaEventRecord");
+    h->info[0] = path;
+    h->info[2] = (int64_t)grid.x * grid.y;
+    h->info[3] = threads;
+    h->info[4] = 0;
+    h->info[5] = ibits;
+    h->info[6] = 0;
+
+    if (multi) {
+      ncclResult_t r = nccl().AllReduce(out.key, out.key, epochs, ncclUint64, ncclMin, h->comm, s);
+      if (r != ncclSuccess) return nccl_fail(h, r, "ncclAllReduce(key)");
+      MCL_CUDA(h, mcl::launch_decode_key(out.key, epochs, Q, D, ibits, o_idx, o_ms, o_map, s), "decode launch");
+      nlaunch += 1;
+      h->info[4] = 1;
+    }
+    MCL_CUDA(h, cudaStreamSynchronize(s), "search kernel");
+    const uint32_t flags = *(volatile uint32_t*)h->flags_host;
+    if (flags & 1u) {
+      h->last_err = "a cost entry is >= 2^48";
+      return MCL_E_RANGE;
+    }
+    if (flags & 2u) {  // some epoch's bound needs 64-bit loads: rerun the wide kernel
+      if (path != 1) {
+        h->last_err = "internal: 64-bit request from a 64-bit kernel";
+        return MCL_E_CUDA;
+      }
+      path = 2;
+      continue;
+    }
+    if (multi && (flags & 4u)) {  // key does not pack: two-step lexicographic all-reduce
+      uint64_t* gms;
+      uint64_t* cand;
+      MCL_CUDA(h, h->gms.ensure(epochs * 8), "cudaMalloc(gms)");
+      MCL_CUDA(h, h->cand.ensure(epochs * 8), "cudaMalloc(cand)");
+      gms = (uint64_t*)h->gms.p;
+      cand = (uint64_t*)h->cand.p;
+      MCL_CUDA(h, mcl::launch_extract_ms(out.pair, epochs, gms, s), "extract launch");
+      ncclResult_t r = nccl().AllReduce(gms, gms, epochs, ncclUint64, ncclMin, h->comm, s);
+      if (r != ncclSuccess) return nccl_fail(h, r, "ncclAllReduce(ms)");
+      MCL_CUDA(h, mcl::launch_pair_candidates(out.pair, gms, epochs, cand, s), "cand launch");
+      r = nccl().AllReduce(cand, cand, epochs, ncclUint64, ncclMin, h->comm, s);
+      if (r != ncclSuccess) return nccl_fail(h, r, "ncclAllReduce(idx)");
+      MCL_CUDA(h, mcl::launch_decode_pair(gms, cand, epochs, Q, D, o_idx, o_ms, o_map, s), "decode launch");
+      nlaunch += 3;
+      h->info[6] = 1;
+      MCL_CUDA(h, cudaStreamSynchronize(s), "two-step reduce");
+    }
+    break;
+  }
+  h->info[1] = nlaunch;
+
+  // ---- results back to host buffers ----
+  if (!di) MCL_CUDA(h, cudaMemcpyAsync(mapping_index, o_idx, epochs * 8, cudaMemcpyDeviceToHost, s), "D2H");
+  if (!dm) MCL_CUDA(h, cudaMemcpyAsync(makespan, o_ms, epochs * 8, cudaMemcpyDeviceToHost, s), "D2H");
+  if (mapping && !dmap)
+    MCL_CUDA(h, cudaMemcpyAsync(mapping, o_map, epochs * Q, cudaMemcpyDeviceToHost, s), "D2H");
+  if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[3], s), "cudaEventRecord");
+  MCL_CUDA(h, cudaStreamSynchronize(s), "D2H");
+  if (h->timing) {
+    cudaEventElapsedTime(&h->kernel_ms, h->ev[0], h->ev[1]);
+    cudaEventElapsedTime(&h->call_ms, h->ev[2], h->ev[3]);
+  }
+  return MCL_OK;
+}
+
+mcl_status_t mcl_probe_int_rate(int device, int op, double* lane_ops_per_s,
+                                double* lane_ops_per_clk_sm, double* eff_mhz) {
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) return MCL_E_INVAL;
+  DeviceGuard g(device);
+  int sms = 0;
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess)
+    return MCL_E_CUDA;
+  double r = 0, c = 0, m = 0;
+  cudaError_t e = mcl::probe_alu(op, sms, nullptr, &r, &c, &m);
+  if (e == cudaErrorInvalidValue) return MCL_E_INVAL;
+  if (e != cudaSuccess) return cuda_fail(nullptr, e, "probe");
+  if (lane_ops_per_s) *lane_ops_per_s = r;
+  if (lane_ops_per_clk_sm) *lane_ops_per_clk_sm = c;
+  if (eff_mhz) *eff_mhz = m;
+  return MCL_OK;
+}
+
+mcl_status_t mcl_device_sms(int device, int* sms) {
+  if (!sms) return MCL_E_INVAL;
+  cudaError_t e = cudaDeviceGetAttribute(sms, cudaDevAttrMultiProcessorCount, device);
+  return e == cudaSuccess ? MCL_OK : cuda_fail(nullptr, e, "cudaDeviceGetAttribute");
+}
+
+mcl_status_t mcl_comm_unique_id(uint8_t id_out[128]) {
+  if (!id_out) return MCL_E_INVAL;
+  if (!nccl().ok) {
+    g_create_err = nccl().err;
+    return MCL_E_NCCL;
+  }
+  ncclUniqueId id;
+  if (nccl().GetUniqueId(&id) != ncclSuccess) return MCL_E_NCCL;
+  std::memcpy(id_out, &id, sizeof(id));
+  return MCL_OK;
+}
+
+mcl_status_t mcl_comm_init(int device, int world, int rank, const uint8_t id[128], void** comm_out) {
+  if (!id || !comm_out || world < 1 || rank < 0 || rank >= world) return MCL_E_INVAL;
+  if (!nccl().ok) {
+    g_create_err = nccl().err;
+    return MCL_E_NCCL;
+  }
+  DeviceGuard g(device);
+  ncclUniqueId uid;
+  std::memcpy(&uid, id, sizeof(uid));
+  ncclComm_t c = nullptr;
+  ncclResult_t r = nccl().CommInitRank(&c, world, uid, rank);
+  if (r != ncclSuccess) {
+    g_create_err = std::string("ncclCommInitRank: ") + nccl().GetErrorString(r);
+    return MCL_E_NCCL;
+  }
+  *comm_out = c;
+  return MCL_OK;
+}
+
+mcl_status_t mcl_comm_destroy(void* comm) {
+  if (!comm) return MCL_OK;
+  if (!nccl().ok) return MCL_E_NCCL;
+  return nccl().CommDestroy((ncclComm_t)comm) == ncclSuccess ? MCL_OK : MCL_E_NCCL;
+}
+
+}  // extern "C"

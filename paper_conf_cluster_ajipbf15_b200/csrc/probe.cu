@@ -1,0 +1,97 @@
+// probe.cu -- integer-pipe throughput probe: the denominator of the
+// mapper's roofline, measured on the same GPU and at the same clocks as the search.
+//
+// Each op kind runs 16 independent cyclic chains per thread at full occupancy (8 CTAs x
+// 256 threads per SM); lane-ops per SM clock come from clock64() deltas, the wall rate
+// from CUDA events on the launching stream. Op kinds:
+//   0 VIMNMX (2-input min/max)   1 VIMNMX3 (3-input)   2 IADD3   3 IMAD
+//   4 VIMNMX3 + IMAD interleaved (are the ALU and FMA pipes issued concurrently?)
+#include "kernels.h"
+
+namespace mcl {
+
+namespace {
+constexpr int kRegs = 16;
+constexpr int kIters = 4096;
+
+template <int OP>
+__global__ void __launch_bounds__(256) probe_kernel(uint32_t* out, uint32_t seed,
+                                                    unsigned long long* cyc) {
+  uint32_t r[kRegs], s[kRegs];
+#pragma unroll
+  for (int i = 0; i < kRegs; ++i) {
+    r[i] = seed * (threadIdx.x + 1) * (i + 7) + blockIdx.x;
+    s[i] = r[i] ^ 0x9e3779b9u;
+  }
+  const long long t0 = clock64();
+  for (int it = 0; it < kIters; ++it) {
+#pragma unroll
+    for (int i = 0; i < kRegs; ++i) {
+      const uint32_t a = r[i], b = r[(i + 1) % kRegs], c = r[(i + 5) % kRegs];
+      if (OP == 0) r[i] = max(a, b);
+      if (OP == 1) r[i] = __vimin3_u32(a, b, c);
+      if (OP == 2) r[i] = a + b + c;
+      if (OP == 3) r[i] = a * b + c;
+      if (OP == 4) {
+        r[i] = __vimin3_u32(a, b, c);
+        s[i] = s[i] * s[(i + 1) % kRegs] + s[(i + 3) % kRegs];
+      }
+    }
+  }
+  const long long t1 = clock64();
+  uint32_t acc = 0;
+#pragma unroll
+  for (int i = 0; i < kRegs; ++i) acc ^= r[i] ^ (OP == 4 ? s[i] : 0u);
+  if (acc == 0x12345678u) out[0] = acc;
+  if (threadIdx.x == 0) atomicMax(cyc, (unsigned long long)(t1 - t0));
+}
+
+template <int OP>
+cudaError_t run(int sms, cudaStream_t st, double* rate, double* per_clk, double* mhz) {
+  uint32_t* out = nullptr;
+  unsigned long long* cyc = nullptr;
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  cudaError_t err = cudaMalloc(&out, 4);
+  if (err == cudaSuccess) err = cudaMalloc(&cyc, 8);
+  if (err == cudaSuccess) err = cudaEventCreate(&e0);
+  if (err == cudaSuccess) err = cudaEventCreate(&e1);
+  const int ctas_per_sm = 8, threads = 256, blocks = sms * ctas_per_sm;
+  if (err == cudaSuccess) {
+    for (int w = 0; w < 3; ++w) probe_kernel<OP><<<blocks, threads, 0, st>>>(out, 3, cyc);
+    cudaMemsetAsync(cyc, 0, 8, st);
+    cudaEventRecord(e0, st);
+    probe_kernel<OP><<<blocks, threads, 0, st>>>(out, 3, cyc);
+    cudaEventRecord(e1, st);
+    err = cudaEventSynchronize(e1);
+  }
+  if (err == cudaSuccess) {
+    float ms = 0;
+    unsigned long long c = 0;
+    cudaEventElapsedTime(&ms, e0, e1);
+    err = cudaMemcpy(&c, cyc, 8, cudaMemcpyDeviceToHost);
+    const double ops_per_thread = (double)kIters * kRegs * (OP == 4 ? 2 : 1);
+    *rate = (double)blocks * threads * ops_per_thread / (ms * 1e-3);
+    *per_clk = (double)ctas_per_sm * threads * ops_per_thread / (double)c;
+    *mhz = (double)c / (ms * 1e3);
+  }
+  if (e0) cudaEventDestroy(e0);
+  if (e1) cudaEventDestroy(e1);
+  if (out) cudaFree(out);
+  if (cyc) cudaFree(cyc);
+  return err;
+}
+}  // namespace
+
+cudaError_t probe_alu(int op, int sms, cudaStream_t st, double* rate, double* per_clk,
+                      double* mhz) {
+  switch (op) {
+    case 0: return run<0>(sms, st, rate, per_clk, mhz);
+    case 1: return run<1>(sms, st, rate, per_clk, mhz);
+    case 2: return run<2>(sms, st, rate, per_clk, mhz);
+    case 3: return run<3>(sms, st, rate, per_clk, mhz);
+    case 4: return run<4>(sms, st, rate, per_clk, mhz);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+}  // namespace mcl

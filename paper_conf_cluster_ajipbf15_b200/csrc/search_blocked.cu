@@ -1,0 +1,393 @@
+// search_blocked.cu -- the register-blocked exhaustive mapper search.
+//
+// One thread scores whole BLOCKS of D^3 mappings: the three innermost queues
+// a = Q-3, b = Q-2, c = Q-1 (digits i, j, k) vary inside a block, the outer Q-3 digits are
+// fixed and give the prefix load vector P[d] (queues on one device
+// serialise, devices run concurrently). With M = max_d P[d] and every cost >= 0, the
+// makespan of leaf (i, j, k) is max(M, load of each device the inner queues touch), which
+// the compiler-unrolled leaf table below forms with ONE integer max per mapping:
+//
+//   i, j, k distinct : max3(P_i+A_i, P_j+B_j, max(M, P_k+C_k))
+//   i == j != k      : max (P_i+A_i+B_i, max(M, P_k+C_k))
+//   i == k != j      : max3(P_i+A_i+C_i, P_j+B_j, M)
+//   j == k != i      : max3(P_i+A_i, P_j+B_j+C_j, M)
+//   i == j == k      : max (M, P_i+A_i+B_i+C_i)
+//
+// (A, B, C = the composed cost rows C[q][.] = K + X of queues a, b, c.)
+// Every leaf's makespan is formed explicitly in a register; the argmin is folded with the
+// sm_100a three-input minimum (VIMNMX3: two mappings per ALU instruction), so the floor is
+// 1.5 ALU instructions per mapping. The block minimum is compared
+// with the thread's running best (strict <, blocks visited in increasing index order);
+// only the single best block is re-scanned at the end to recover the lowest leaf index.
+//
+// The outer digits walk an odometer: digit x (queue Q-4) is the block loop, the digits of
+// queues 0..Q-5 live in shared memory and update the base load vector by one-hot vectors
+// V[q][x] (V[q][x][d] = C[q][x] if d == x else 0) so every register index stays static.
+#include "common.cuh"
+#include "kernels.h"
+
+namespace mcl {
+
+namespace {
+
+// Adds routed to the FMA pipe (IMAD) so the ALU pipe is left for min/max: `one` is a
+// runtime 1 the compiler cannot fold.
+__device__ __forceinline__ uint32_t add_f(uint32_t a, uint32_t b, uint32_t one) {
+  uint32_t r;
+  asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(one), "r"(b));
+  return r;
+}
+__device__ __forceinline__ uint64_t add_f(uint64_t a, uint64_t b, uint32_t) { return a + b; }
+
+// Integer min/max: VIMNMX (two inputs) and VIMNMX3 (three inputs) for 32-bit lanes.
+__device__ __forceinline__ uint32_t max2(uint32_t a, uint32_t b) { return max(a, b); }
+__device__ __forceinline__ uint32_t max3(uint32_t a, uint32_t b, uint32_t c) { return __vimax3_u32(a, b, c); }
+__device__ __forceinline__ uint32_t min2(uint32_t a, uint32_t b) { return min(a, b); }
+__device__ __forceinline__ uint32_t min3(uint32_t a, uint32_t b, uint32_t c) { return __vimin3_u32(a, b, c); }
+__device__ __forceinline__ uint64_t max2(uint64_t a, uint64_t b) { return a > b ? a : b; }
+__device__ __forceinline__ uint64_t max3(uint64_t a, uint64_t b, uint64_t c) { return max2(a, max2(b, c)); }
+__device__ __forceinline__ uint64_t min2(uint64_t a, uint64_t b) { return a < b ? a : b; }
+__device__ __forceinline__ uint64_t min3(uint64_t a, uint64_t b, uint64_t c) { return min2(a, min2(b, c)); }
+
+// Shared-memory layout of the per-epoch tables (T = uint32_t or uint64_t).
+//   in[7][D]      : A, B, C, A+B, A+C, B+C, A+B+C of the three inner queues
+//   V[O][D][D]    : one-hot outer vectors, O = Q - 3
+// Enumerate the D^3 leaves of one block in increasing index order, calling f(leaf, ms).
+template <typename T, int D, typename F>
+__device__ __forceinline__ void for_each_leaf(const T (&P)[D], const T* __restrict__ in,
+                                              uint32_t one, F&& f) {
+  T M = P[0];
+#pragma unroll
+  for (int d = 1; d < D; ++d) M = max2(M, P[d]);
+  T PA[D], PB[D], PCM[D], PAB[D], PAC[D], PBC[D], PABC[D];
+#pragma unroll
+  for (int d = 0; d < D; ++d) {
+    PA[d] = add_f(P[d], in[0 * D + d], one);
+    PB[d] = add_f(P[d], in[1 * D + d], one);
+    PCM[d] = max2(M, add_f(P[d], in[2 * D + d], one));
+    PAB[d] = add_f(P[d], in[3 * D + d], one);
+    PAC[d] = add_f(P[d], in[4 * D + d], one);
+    PBC[d] = add_f(P[d], in[5 * D + d], one);
+    PABC[d] = add_f(P[d], in[6 * D + d], one);
+  }
+#pragma unroll
+  for (int i = 0; i < D; ++i)
+#pragma unroll
+    for (int j = 0; j < D; ++j)
+#pragma unroll
+      for (int k = 0; k < D; ++k) {
+        T v;
+        if (i != j && i != k && j != k) v = max3(PA[i], PB[j], PCM[k]);
+        else if (i == j && j != k) v = max2(PAB[i], PCM[k]);
+        else if (i == k && i != j) v = max3(PAC[i], PB[j], M);
+        else if (j == k && i != j) v = max3(PA[i], PBC[j], M);
+        else v = max2(M, PABC[i]);
+        f((i * D + j) * D + k, v);
+      }
+}
+
+// Minimum makespan over one block, folded two leaves per three-input min.
+template <typename T, int D>
+__device__ __forceinline__ T block_eval(const T (&P)[D], const T* __restrict__ in, uint32_t one) {
+  constexpr T kMax = ~T(0);
+  T acc[4] = {kMax, kMax, kMax, kMax};
+  T pend = kMax;
+  for_each_leaf<T, D>(P, in, one, [&](int leaf, T v) {
+    if (leaf & 1) {
+      acc[(leaf >> 1) & 3] = min3(acc[(leaf >> 1) & 3], pend, v);
+    } else {
+      pend = v;
+    }
+  });
+  constexpr int kLeaves = D * D * D;
+  T g = min3(acc[0], acc[1], min2(acc[2], acc[3]));
+  if (kLeaves & 1) g = min2(g, pend);
+  return g;
+}
+
+// Lowest leaf of the block whose makespan equals `target` (the block is known to hold one).
+template <typename T, int D>
+__device__ __forceinline__ uint32_t block_first(const T (&P)[D], const T* __restrict__ in,
+                                                uint32_t one, T target) {
+  uint32_t first = 0xffffffffu;
+  for_each_leaf<T, D>(P, in, one, [&](int leaf, T v) {
+    first = (v == target && first == 0xffffffffu) ? (uint32_t)leaf : first;
+  });
+  return first;
+}
+
+template <typename T, int D>
+__device__ __forceinline__ void load_vec(T (&v)[D], const T* __restrict__ src) {
+#pragma unroll
+  for (int d = 0; d < D; ++d) v[d] = src[d];
+}
+
+// Prefix loads P of block `blk` (outer digits of queues 0..O-1), decoded from scratch.
+template <typename T, int D>
+__device__ __forceinline__ void prefix_of(T (&P)[D], uint64_t blk, int O, const T* __restrict__ V,
+                                          uint32_t one) {
+#pragma unroll
+  for (int d = 0; d < D; ++d) P[d] = 0;
+  for (int q = O - 1; q >= 0; --q) {
+    const uint32_t dq = (uint32_t)(blk % D);
+    blk /= D;
+    const T* v = V + ((size_t)q * D + dq) * D;
+#pragma unroll
+    for (int d = 0; d < D; ++d) P[d] = add_f(P[d], v[d], one);
+  }
+}
+
+}  // namespace
+
+// Kernel: gridDim.x = CTAs per epoch (cpe), gridDim.y = epochs handled concurrently.
+template <typename T, int D>
+__global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
+    search_blocked_kernel(BlockedArgs a) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const uint32_t Q = a.Q;
+  const int O = (int)Q - 3;  // outer queues (>= 0)
+  const int nthr = blockDim.x, tid = threadIdx.x;
+  // layout: C64[Q*D] u64 | in[7*D] T | V[O*D*D] T | red[32] Cand | dig[(O-1)*nthr] u8
+  uint64_t* C64 = reinterpret_cast<uint64_t*>(smem_raw);
+  T* in = reinterpret_cast<T*>(C64 + Q * D);
+  T* V = in + 7 * D;
+  Cand* red = reinterpret_cast<Cand*>(
+      reinterpret_cast<unsigned char*>(smem_raw) + a.off_red);
+  uint8_t* dig = reinterpret_cast<uint8_t*>(smem_raw) + a.off_dig;
+  __shared__ __align__(16) T zero[D];
+  if (threadIdx.x < D) zero[threadIdx.x] = 0;
+  __shared__ int s_bad;
+  __shared__ uint64_t s_ub;
+
+  for (uint64_t e = blockIdx.y; e < a.E; e += gridDim.y) {
+    // ---- a1: cost composition C = K + X, range check, bound UB = sum_q max_d C ----
+    __syncthreads();  // the previous epoch's tables are no longer read
+    if (tid == 0) { s_bad = 0; s_ub = 0; }
+    __syncthreads();
+    const uint64_t* Ke = a.K + e * Q * D;
+    const uint64_t* Xe = a.X + e * Q * D;
+    for (uint32_t t = tid; t < Q * D; t += nthr) {
+      const uint64_t k = Ke[t], x = Xe[t];
+      if (k >= kEntryLimit || x >= kEntryLimit) s_bad = 1;
+      C64[t] = k + x;
+    }
+    __syncthreads();
+    if (s_bad) {
+      if (tid == 0 && blockIdx.x == 0) raise_flag(a.flags, kFlagRange);
+      continue;
+    }
+    if (tid < 32) {  // one warp: per-queue row max, then the sum over queues
+      uint64_t part = 0;
+      for (uint32_t q = tid; q < Q; q += 32) {
+        uint64_t m = 0;
+        for (int d = 0; d < D; ++d) m = max2(m, C64[q * D + d]);
+        part += m;
+      }
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) part += __shfl_xor_sync(0xffffffffu, part, off);
+      if (tid == 0) s_ub = part;
+    }
+    __syncthreads();
+    if (sizeof(T) == 4 && s_ub >= (1ull << 32)) {
+      if (tid == 0 && blockIdx.x == 0) raise_flag(a.flags, kFlagNeedU64);
+      continue;
+    }
+    // ---- tables: inner sums and one-hot outer vectors ----
+    for (int t = tid; t < D; t += nthr) {
+      const uint64_t A = C64[(Q - 3) * D + t], B = C64[(Q - 2) * D + t], Cc = C64[(Q - 1) * D + t];
+      in[0 * D + t] = (T)A;
+      in[1 * D + t] = (T)B;
+      in[2 * D + t] = (T)Cc;
+      in[3 * D + t] = (T)(A + B);
+      in[4 * D + t] = (T)(A + Cc);
+      in[5 * D + t] = (T)(B + Cc);
+      in[6 * D + t] = (T)(A + B + Cc);
+    }
+    for (int t = tid; t < O * D * D; t += nthr) {
+      const int q = t / (D * D), x = (t / D) % D, d = t % D;
+      V[t] = (d == x) ? (T)C64[q * D + x] : (T)0;
+    }
+    __syncthreads();
+
+    // ---- a2-a5: this thread's contiguous block range inside the rank's range ----
+    const uint64_t nb_rank = a.rhi - a.rlo;
+    const uint64_t T_all = (uint64_t)gridDim.x * nthr;
+    const uint64_t gt = (uint64_t)blockIdx.x * nthr + tid;
+    const uint64_t per = nb_rank / T_all, rem = nb_rank % T_all;
+    const uint64_t b0 = a.rlo + gt * per + (gt < rem ? gt : rem);
+    uint64_t nleft = per + (gt < rem ? 1 : 0);
+
+    T best = ~T(0);
+    uint64_t best_blk = kNone;
+    const uint32_t one = a.one;
+    if (nleft) {
+      {
+        // digit x = queue O-1 runs fastest; queues 0..O-2 are the odometer in smem.
+        // Q == 3 (O == 0): a single block whose prefix is the zero vector.
+        const T* Vx = (O >= 1) ? V + (size_t)(O - 1) * D * D : zero;
+        uint32_t x = (uint32_t)(b0 % D);
+        uint64_t hi = b0 / D;
+        T base[D];
+#pragma unroll
+        for (int d = 0; d < D; ++d) base[d] = 0;
+        for (int q = O - 2; q >= 0; --q) {
+          const uint32_t dq = (uint32_t)(hi % D);
+          hi /= D;
+          dig[q * nthr + tid] = (uint8_t)dq;
+          const T* v = V + ((size_t)q * D + dq) * D;
+#pragma unroll
+          for (int d = 0; d < D; ++d) base[d] = add_f(base[d], v[d], one);
+        }
+        uint64_t blk = b0;
+        while (true) {
+          for (; x < (uint32_t)D && nleft; ++x, --nleft, ++blk) {
+            T P[D], vx[D];
+            load_vec<T, D>(vx, Vx + x * D);
+#pragma unroll
+            for (int d = 0; d < D; ++d) P[d] = add_f(base[d], vx[d], one);
+            const T g = block_eval<T, D>(P, in, one);
+            if (g < best) {
+              best = g;
+              best_blk = blk;
+            }
+          }
+          if (!nleft) break;
+          x = 0;
+          // odometer increment of the outer digits, updating base by one-hot deltas
+          for (int q = O - 2; q >= 0; --q) {
+            const uint32_t old = dig[q * nthr + tid];
+            const uint32_t nw = (old + 1 == (uint32_t)D) ? 0u : old + 1;
+            dig[q * nthr + tid] = (uint8_t)nw;
+            const T* vo = V + ((size_t)q * D + old) * D;
+            const T* vn = V + ((size_t)q * D + nw) * D;
+#pragma unroll
+            for (int d = 0; d < D; ++d) base[d] = base[d] - vo[d] + vn[d];
+            if (nw != 0) break;
+          }
+        }
+      }
+    }
+    // ---- a5: lowest index inside the best block, then warp / CTA / epoch argmin ----
+    Cand c{kNone, kNone};
+    if (best_blk != kNone) {
+      T P[D];
+      prefix_of<T, D>(P, best_blk, O, V, one);
+      const uint32_t leaf = block_first<T, D>(P, in, one, best);
+      c.ms = (uint64_t)best;
+      c.idx = best_blk * (uint64_t)(D * D * D) + leaf;
+    }
+    c = block_min(c, red);
+    if (gridDim.x == 1) {
+      if (tid == 0) write_epoch(a.out, e, Q, D, a.ibits, c, a.flags);
+      continue;
+    }
+    __shared__ bool s_last;
+    if (tid == 0) {
+      a.scratch[e * gridDim.x + blockIdx.x] = c;
+      __threadfence();
+      const uint32_t prev = atomicAdd(&a.done[e], 1u);
+      s_last = (prev == gridDim.x - 1);
+    }
+    __syncthreads();
+    if (s_last) {
+      __threadfence();
+      Cand r{kNone, kNone};
+      for (uint32_t t = tid; t < gridDim.x; t += nthr) {
+        const volatile uint64_t* o =
+            reinterpret_cast<const volatile uint64_t*>(&a.scratch[e * gridDim.x + t]);
+        r = cand_min(r, Cand{o[0], o[1]});
+      }
+      r = block_min(r, red);
+      if (tid == 0) {
+        write_epoch(a.out, e, Q, D, a.ibits, r, a.flags);
+        a.done[e] = 0;  // self-reset for the next call
+      }
+    }
+  }
+}
+
+template <typename T, int D>
+static cudaError_t launch_blocked_t(const BlockedArgs& a, dim3 grid, int threads, size_t smem,
+                                   cudaStream_t st) {
+  auto k = search_blocked_kernel<T, D>;
+  {  // always: the default 48 KB cap also counts the kernel's static shared memory
+    cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (err != cudaSuccess) return err;
+  }
+  k<<<grid, threads, smem, st>>>(a);
+  return cudaGetLastError();
+}
+
+size_t blocked_smem_bytes(uint32_t Q, uint32_t D, bool wide, int threads, size_t* off_red,
+                          size_t* off_dig) {
+  const size_t tsz = wide ? 8 : 4;
+  const int O = (int)Q - 3;
+  size_t off = (size_t)Q * D * 8 + 7 * D * tsz + (size_t)(O > 0 ? O : 0) * D * D * tsz;
+  off = (off + 15) & ~size_t(15);
+  *off_red = off;
+  off += 32 * sizeof(Cand);
+  *off_dig = off;
+  off += (size_t)(O > 1 ? O - 1 : 0) * threads;
+  return (off + 15) & ~size_t(15);
+}
+
+namespace {
+template <typename T, int D>
+int occ_t(int threads, size_t smem) {
+  int n = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, search_blocked_kernel<T, D>, threads, smem) !=
+      cudaSuccess)
+    return 1;
+  return n < 1 ? 1 : n;
+}
+}  // namespace
+
+int blocked_ctas_per_sm(uint32_t D, bool wide, int threads, size_t smem) {
+#ifdef MCL_ONLY_D
+  if (D != MCL_ONLY_D) return 1;
+  return wide ? occ_t<uint64_t, MCL_ONLY_D>(threads, smem) : occ_t<uint32_t, MCL_ONLY_D>(threads, smem);
+#else
+  switch (D) {
+    case 2: return wide ? occ_t<uint64_t, 2>(threads, smem) : occ_t<uint32_t, 2>(threads, smem);
+    case 3: return wide ? occ_t<uint64_t, 3>(threads, smem) : occ_t<uint32_t, 3>(threads, smem);
+    case 4: return wide ? occ_t<uint64_t, 4>(threads, smem) : occ_t<uint32_t, 4>(threads, smem);
+    case 5: return wide ? occ_t<uint64_t, 5>(threads, smem) : occ_t<uint32_t, 5>(threads, smem);
+    case 6: return wide ? occ_t<uint64_t, 6>(threads, smem) : occ_t<uint32_t, 6>(threads, smem);
+    case 7: return wide ? occ_t<uint64_t, 7>(threads, smem) : occ_t<uint32_t, 7>(threads, smem);
+    case 8: return wide ? occ_t<uint64_t, 8>(threads, smem) : occ_t<uint32_t, 8>(threads, smem);
+    default: return 1;
+  }
+#endif
+}
+
+bool blocked_supported(uint32_t Q, uint32_t D) { return Q >= 3 && D >= 2 && D <= kBlockedMaxD; }
+
+cudaError_t launch_blocked(const BlockedArgs& a, bool wide, dim3 grid, int threads, size_t smem,
+                           cudaStream_t st) {
+#ifdef MCL_ONLY_D
+#define MCL_CASE(DD)                                                                  \
+  case DD:                                                                            \
+    if (DD != MCL_ONLY_D) return cudaErrorInvalidValue;                               \
+    return wide ? launch_blocked_t<uint64_t, DD % MCL_ONLY_D == 0 ? DD : MCL_ONLY_D>(a, grid, threads, smem, st) \
+                : launch_blocked_t<uint32_t, DD % MCL_ONLY_D == 0 ? DD : MCL_ONLY_D>(a, grid, threads, smem, st);
+#else
+#define MCL_CASE(DD)                                                                  \
+  case DD:                                                                            \
+    return wide ? launch_blocked_t<uint64_t, DD>(a, grid, threads, smem, st)          \
+                : launch_blocked_t<uint32_t, DD>(a, grid, threads, smem, st);
+#endif
+  switch (a.D) {
+    MCL_CASE(2)
+    MCL_CASE(3)
+    MCL_CASE(4)
+    MCL_CASE(5)
+    MCL_CASE(6)
+    MCL_CASE(7)
+    MCL_CASE(8)
+    default:
+      return cudaErrorInvalidValue;
+  }
+#undef MCL_CASE
+}
+
+}  // namespace mcl

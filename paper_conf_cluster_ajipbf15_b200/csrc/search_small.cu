@@ -1,0 +1,217 @@
+// search_small.cu -- batched search for tiny index spaces (D^Q <= 81), one thread per epoch
+// (FDM-Seismology 2 queues x 3 devices x 10^6 epochs, and cfg1).
+//
+// The work per epoch is a handful of integer ops; the kernel is bound by HBM (96 B of
+// costs in, 18 B of results out per epoch at Q=2, D=3). A persistent grid streams tiles of
+// blockDim.x epochs: one elected thread moves a tile's K and X slabs global -> shared with
+// cp.async.bulk (the TMA bulk-copy engine, SASS UBLKCP) completing on an mbarrier, double
+// buffered so the next tile is in flight while the current one is scored. Each thread then
+// scores its epoch's D^Q mappings from shared memory with compile-time digits (so every
+// load index is static), in increasing index order with a strict '<' (lowest index wins
+// ties, BASELINE.json north_star), and writes its outputs coalesced.
+#include "common.cuh"
+#include "kernels.h"
+
+namespace mcl {
+
+namespace {
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra WAIT_%=;\n"
+      "}\n" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+template <int Q, int D>
+struct Pow {
+  static constexpr int N = D * Pow<Q - 1, D>::N;
+};
+template <int D>
+struct Pow<0, D> {
+  static constexpr int N = 1;
+};
+
+}  // namespace
+
+template <int Q, int D>
+__global__ void __launch_bounds__(256) search_small_kernel(SmallArgs a, int use_tma) {
+  constexpr int QD = Q * D;
+  constexpr int N = Pow<Q, D>::N;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  __shared__ __align__(8) uint64_t bar[2];
+  const int TE = blockDim.x, tid = threadIdx.x;
+  uint64_t* sK[2];
+  uint64_t* sX[2];
+  sK[0] = reinterpret_cast<uint64_t*>(smem_raw);
+  sX[0] = sK[0] + (size_t)TE * QD;
+  sK[1] = sX[0] + (size_t)TE * QD;
+  sX[1] = sK[1] + (size_t)TE * QD;
+
+  const uint64_t E = a.E;
+  const uint64_t ntiles = (E + TE - 1) / TE;
+  // a tile goes through TMA iff it is full (the ragged last tile uses plain loads) and the
+  // caller's pointers are 16-byte aligned (use_tma)
+  auto tile_tma = [&](uint64_t t) { return use_tma && (t + 1) * TE <= E; };
+  auto issue = [&](uint64_t t, int s) {
+    const uint32_t bytes = (uint32_t)((size_t)TE * QD * 8);
+    fence_proxy_async();
+    mbar_expect_tx(&bar[s], 2 * bytes);
+    bulk_g2s(sK[s], a.K + t * TE * QD, bytes, &bar[s]);
+    bulk_g2s(sX[s], a.X + t * TE * QD, bytes, &bar[s]);
+  };
+  if (tid == 0) {
+    mbar_init(&bar[0], 1);
+    mbar_init(&bar[1], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  uint32_t phase[2] = {0, 0};
+  uint64_t t = blockIdx.x;
+  if (tid == 0 && t < ntiles && tile_tma(t)) issue(t, 0);
+  bool bad = false;
+  for (int it = 0; t < ntiles; t += gridDim.x, ++it) {
+    const int s = it & 1;
+    const uint64_t tn = t + gridDim.x;
+    if (tid == 0 && tn < ntiles && tile_tma(tn)) issue(tn, s ^ 1);
+    if (tile_tma(t)) {
+      mbar_wait(&bar[s], phase[s]);
+      phase[s] ^= 1u;
+    } else {
+      const uint64_t n = (E - t * TE < (uint64_t)TE) ? E - t * TE : (uint64_t)TE;
+      for (uint64_t j = tid; j < n * QD; j += TE) {
+        sK[s][j] = a.K[t * TE * QD + j];
+        sX[s][j] = a.X[t * TE * QD + j];
+      }
+      __syncthreads();
+    }
+    const uint64_t e = t * TE + tid;
+    if (e < E) {
+      uint64_t C[Q][D];
+      const uint64_t* k = sK[s] + (size_t)tid * QD;
+      const uint64_t* x = sX[s] + (size_t)tid * QD;
+#pragma unroll
+      for (int q = 0; q < Q; ++q)
+#pragma unroll
+        for (int d = 0; d < D; ++d) {
+          const uint64_t kv = k[q * D + d], xv = x[q * D + d];
+          bad |= (kv >= kEntryLimit) | (xv >= kEntryLimit);
+          C[q][d] = kv + xv;  // a1: aggregate cost
+        }
+      uint64_t best = kNone;
+      uint32_t bi = 0;
+#pragma unroll
+      for (int m = 0; m < N; ++m) {
+        uint64_t L[D];
+#pragma unroll
+        for (int d = 0; d < D; ++d) L[d] = 0;
+        int rest = m;
+#pragma unroll
+        for (int q = Q - 1; q >= 0; --q) {
+          const int dq = rest % D;
+          rest /= D;
+          L[dq] += C[q][dq];
+        }
+        uint64_t ms = L[0];
+#pragma unroll
+        for (int d = 1; d < D; ++d) ms = max(ms, L[d]);
+        if (ms < best) {
+          best = ms;
+          bi = (uint32_t)m;
+        }
+      }
+      a.index[e] = bi;
+      a.makespan[e] = best;
+      if (a.mapping) {
+        uint32_t rest = bi;
+#pragma unroll
+        for (int q = Q - 1; q >= 0; --q) {
+          a.mapping[e * Q + q] = (uint8_t)(rest % D);
+          rest /= D;
+        }
+      }
+    }
+    __syncthreads();  // stage s is free for the prefetch issued next iteration
+  }
+  if (__any_sync(0xffffffffu, bad) && (tid & 31) == 0) raise_flag(a.flags, kFlagRange);
+}
+
+namespace {
+template <int Q, int D>
+cudaError_t launch_small_t(const SmallArgs& a, int num_sms, cudaStream_t st, int* grid_out,
+                           int* threads_out) {
+  const int threads = 256;
+  const size_t smem = (size_t)4 * threads * Q * D * 8;  // 2 stages x (K, X)
+  auto k = search_small_kernel<Q, D>;
+  {  // always: the default 48 KB cap also counts the kernel's static shared memory
+    cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (err != cudaSuccess) return err;
+  }
+  int per_sm = 0;
+  cudaError_t err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, threads, smem);
+  if (err != cudaSuccess) return err;
+  if (per_sm < 1) per_sm = 1;
+  const uint64_t ntiles = (a.E + threads - 1) / threads;
+  uint64_t grid = (uint64_t)num_sms * per_sm;
+  if (grid > ntiles) grid = ntiles;
+  const int use_tma = ((reinterpret_cast<uintptr_t>(a.K) | reinterpret_cast<uintptr_t>(a.X)) & 15) == 0;
+  k<<<(unsigned)grid, threads, smem, st>>>(a, use_tma);
+  *grid_out = (int)grid;
+  *threads_out = threads;
+  return cudaGetLastError();
+}
+}  // namespace
+
+bool small_supported(uint32_t Q, uint32_t D) {
+  return (Q == 2 && (D >= 2 && D <= 4)) || (Q == 3 && (D >= 2 && D <= 4)) ||
+         (Q == 4 && (D == 2 || D == 3));
+}
+
+cudaError_t launch_small(const SmallArgs& a, int num_sms, cudaStream_t st, int* grid_out,
+                         int* threads_out) {
+  const uint32_t key = a.Q * 100 + a.D;
+  switch (key) {
+    case 202: return launch_small_t<2, 2>(a, num_sms, st, grid_out, threads_out);
+    case 203: return launch_small_t<2, 3>(a, num_sms, st, grid_out, threads_out);
+    case 204: return launch_small_t<2, 4>(a, num_sms, st, grid_out, threads_out);
+    case 302: return launch_small_t<3, 2>(a, num_sms, st, grid_out, threads_out);
+    case 303: return launch_small_t<3, 3>(a, num_sms, st, grid_out, threads_out);
+    case 304: return launch_small_t<3, 4>(a, num_sms, st, grid_out, threads_out);
+    case 402: return launch_small_t<4, 2>(a, num_sms, st, grid_out, threads_out);
+    case 403: return launch_small_t<4, 3>(a, num_sms, st, grid_out, threads_out);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+}  // namespace mcl

@@ -1,0 +1,266 @@
+"""Thin Python binding of libmcl.so (include/mcl.h, include/mcl_ext.h) -- argument
+marshalling only. Every mapping is scored by the library's CUDA kernels; there is no
+Python or CPU fallback: if libmcl.so is missing or no CUDA device is usable, calls raise.
+
+Names mirror the C ABI: ``mcl_mapper_create``, ``mcl_map_queues``, ``mcl_mapper_destroy``,
+``mcl_status_string`` ... plus a small ``Mapper`` convenience class that accepts torch
+tensors (CUDA or CPU) or numpy arrays.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libmcl.so")
+
+MCL_OK, MCL_E_INVAL, MCL_E_RANGE, MCL_E_CUDA, MCL_E_NCCL, MCL_E_NOMEM = 0, -1, -2, -3, -4, -5
+PATH_NAMES = {1: "blocked_u32", 2: "blocked_u64", 3: "generic", 4: "small_batched"}
+
+# Every symbol the headers declare (tests check the library exports all of them).
+EXPORTED = [
+    "mcl_mapper_create", "mcl_map_queues", "mcl_mapper_destroy", "mcl_status_string",
+    "mcl_last_error_string", "mcl_last_launch_info", "mcl_version",
+    "mcl_set_timing", "mcl_last_kernel_time", "mcl_force_path", "mcl_probe_int_rate",
+    "mcl_device_sms",
+    "mcl_comm_unique_id", "mcl_comm_init", "mcl_comm_destroy",
+]
+
+
+class mcl_config_t(ctypes.Structure):
+    _fields_ = [
+        ("device", ctypes.c_int),
+        ("stream", ctypes.c_void_p),
+        ("nccl_comm", ctypes.c_void_p),
+        ("rank", ctypes.c_int),
+        ("world", ctypes.c_int),
+    ]
+
+
+class MclError(RuntimeError):
+    def __init__(self, status: int, where: str, detail: str = ""):
+        msg = f"{where}: {mcl_status_string(status)}"
+        if detail:
+            msg += f" ({detail})"
+        super().__init__(msg)
+        self.status = status
+
+
+_lib = None
+
+
+def load_library(path: str | None = None) -> ctypes.CDLL:
+    """Load libmcl.so (fails loudly if it has not been built)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    p = path or LIB_PATH
+    if not os.path.exists(p):
+        raise RuntimeError(
+            f"{p} not found: build it with `python -m paper_conf_cluster_ajipbf15_b200.build` "
+            "(there is no CPU fallback)"
+        )
+    lib = ctypes.CDLL(p)
+    vp, u32, u64, i32 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int
+    sig = {
+        "mcl_mapper_create": (i32, [ctypes.POINTER(mcl_config_t), ctypes.POINTER(vp)]),
+        "mcl_map_queues": (i32, [vp, u32, u32, u64, vp, vp, vp, vp, vp]),
+        "mcl_mapper_destroy": (None, [vp]),
+        "mcl_status_string": (ctypes.c_char_p, [i32]),
+        "mcl_last_error_string": (ctypes.c_char_p, [vp]),
+        "mcl_last_launch_info": (i32, [vp, ctypes.POINTER(ctypes.c_int64)]),
+        "mcl_version": (ctypes.c_char_p, []),
+        "mcl_set_timing": (i32, [vp, i32]),
+        "mcl_force_path": (i32, [vp, i32]),
+        "mcl_last_kernel_time": (i32, [vp, ctypes.POINTER(ctypes.c_float), ctypes.POINTER(ctypes.c_float)]),
+        "mcl_probe_int_rate": (i32, [i32, i32, ctypes.POINTER(ctypes.c_double),
+                                     ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]),
+        "mcl_device_sms": (i32, [i32, ctypes.POINTER(i32)]),
+        "mcl_comm_unique_id": (i32, [ctypes.c_char_p]),
+        "mcl_comm_init": (i32, [i32, i32, i32, ctypes.c_char_p, ctypes.POINTER(vp)]),
+        "mcl_comm_destroy": (i32, [vp]),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(lib, name)
+        f.restype = res
+        f.argtypes = args
+    _lib = lib
+    return lib
+
+
+def mcl_status_string(status: int) -> str:
+    return load_library().mcl_status_string(status).decode()
+
+
+def mcl_version() -> str:
+    return load_library().mcl_version().decode()
+
+
+def mcl_mapper_create(device: int = 0, stream: int | None = None, nccl_comm: int | None = None,
+                      rank: int = 0, world: int = 1) -> int:
+    lib = load_library()
+    cfg = mcl_config_t(device, stream or None, nccl_comm or None, rank, world)
+    h = ctypes.c_void_p()
+    st = lib.mcl_mapper_create(ctypes.byref(cfg), ctypes.byref(h))
+    if st != MCL_OK:
+        raise MclError(st, "mcl_mapper_create", lib.mcl_last_error_string(None).decode())
+    return h.value
+
+
+def mcl_mapper_destroy(handle: int | None) -> None:
+    load_library().mcl_mapper_destroy(handle)
+
+
+def mcl_map_queues(handle: int, Q: int, D: int, epochs: int, cost_kernel_ptr: int,
+                   cost_xfer_ptr: int, mapping_index_ptr: int, mapping_ptr: int | None,
+                   makespan_ptr: int) -> int:
+    """Raw call with integer pointers (device or host). Returns the status code."""
+    return load_library().mcl_map_queues(handle, Q, D, epochs, cost_kernel_ptr, cost_xfer_ptr,
+                                         mapping_index_ptr, mapping_ptr or None, makespan_ptr)
+
+
+def mcl_last_error_string(handle: int | None) -> str:
+    return load_library().mcl_last_error_string(handle).decode()
+
+
+def mcl_last_launch_info(handle: int) -> list[int]:
+    arr = (ctypes.c_int64 * 8)()
+    load_library().mcl_last_launch_info(handle, arr)
+    return list(arr)
+
+
+def mcl_probe_int_rate(device: int, op: int) -> tuple[float, float, float]:
+    r, c, m = ctypes.c_double(), ctypes.c_double(), ctypes.c_double()
+    st = load_library().mcl_probe_int_rate(device, op, ctypes.byref(r), ctypes.byref(c), ctypes.byref(m))
+    if st != MCL_OK:
+        raise MclError(st, "mcl_probe_int_rate", mcl_last_error_string(None))
+    return r.value, c.value, m.value
+
+
+def mcl_device_sms(device: int = 0) -> int:
+    n = ctypes.c_int()
+    st = load_library().mcl_device_sms(device, ctypes.byref(n))
+    if st != MCL_OK:
+        raise MclError(st, "mcl_device_sms")
+    return n.value
+
+
+def mcl_comm_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    st = load_library().mcl_comm_unique_id(buf)
+    if st != MCL_OK:
+        raise MclError(st, "mcl_comm_unique_id", mcl_last_error_string(None))
+    return buf.raw
+
+
+def mcl_comm_init(device: int, world: int, rank: int, uid: bytes) -> int:
+    comm = ctypes.c_void_p()
+    st = load_library().mcl_comm_init(device, world, rank, uid, ctypes.byref(comm))
+    if st != MCL_OK:
+        raise MclError(st, "mcl_comm_init", mcl_last_error_string(None))
+    return comm.value
+
+
+def mcl_comm_destroy(comm: int | None) -> None:
+    load_library().mcl_comm_destroy(comm)
+
+
+def _ptr_and_keepalive(x, dtype):
+    """(pointer, owner) for a torch tensor or numpy array of the given numpy dtype."""
+    try:
+        import torch
+    except ImportError:  # pragma: no cover
+        torch = None
+    if torch is not None and isinstance(x, torch.Tensor):
+        want = {np.uint64: torch.uint64, np.uint8: torch.uint8}[dtype]
+        if x.dtype != want or not x.is_contiguous():
+            raise TypeError(f"expected a contiguous {want} tensor")
+        return x.data_ptr(), x
+    a = np.asarray(x)
+    if a.dtype != dtype or not a.flags.c_contiguous:
+        raise TypeError(f"expected a C-contiguous {np.dtype(dtype)} array")
+    return a.ctypes.data, a
+
+
+class Mapper:
+    """One mapper handle (see include/mcl.h). Use as a context manager or call close()."""
+
+    def __init__(self, device: int = 0, stream: int | None = None, nccl_comm: int | None = None,
+                 rank: int = 0, world: int = 1):
+        self.device = device
+        self.handle = mcl_mapper_create(device, stream, nccl_comm, rank, world)
+
+    def close(self):
+        if self.handle:
+            mcl_mapper_destroy(self.handle)
+            self.handle = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    def __del__(self):  # pragma: no cover
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def map_queues_into(self, K, X, index, mapping, makespan) -> None:
+        """Run the search writing into caller-owned outputs. K, X: [E, Q, D] uint64;
+        index, makespan: [E] uint64; mapping: [E, Q] uint8 or None. Tensors may live on the
+        handle's CUDA device or on the host."""
+        E, Q, D = (int(s) for s in K.shape)
+        pk, _k = _ptr_and_keepalive(K, np.uint64)
+        px, _x = _ptr_and_keepalive(X, np.uint64)
+        pi, _i = _ptr_and_keepalive(index, np.uint64)
+        pm, _m = _ptr_and_keepalive(makespan, np.uint64)
+        pmap = None
+        if mapping is not None:
+            pmap, _mp = _ptr_and_keepalive(mapping, np.uint8)
+        st = mcl_map_queues(self.handle, Q, D, E, pk, px, pi, pmap, pm)
+        if st != MCL_OK:
+            raise MclError(st, "mcl_map_queues", mcl_last_error_string(self.handle))
+
+    def map_queues(self, K, X, with_mapping: bool = True):
+        """Convenience: allocate outputs like K (same device / numpy) and return
+        (index[E], mapping[E, Q] or None, makespan[E])."""
+        if K.ndim == 2:
+            K, X = K[None], X[None]
+        E, Q, D = (int(s) for s in K.shape)
+        try:
+            import torch
+        except ImportError:  # pragma: no cover
+            torch = None
+        if torch is not None and isinstance(K, torch.Tensor):
+            idx = torch.empty(E, dtype=torch.uint64, device=K.device)
+            ms = torch.empty(E, dtype=torch.uint64, device=K.device)
+            mp = torch.empty((E, Q), dtype=torch.uint8, device=K.device) if with_mapping else None
+        else:
+            idx = np.empty(E, dtype=np.uint64)
+            ms = np.empty(E, dtype=np.uint64)
+            mp = np.empty((E, Q), dtype=np.uint8) if with_mapping else None
+        self.map_queues_into(K, X, idx, mp, ms)
+        return idx, mp, ms
+
+    def launch_info(self) -> dict:
+        i = mcl_last_launch_info(self.handle)
+        return {"path": PATH_NAMES.get(i[0], str(i[0])), "launches": i[1], "ctas": i[2],
+                "threads": i[3], "allreduce": bool(i[4]), "index_bits": i[5], "two_step": bool(i[6])}
+
+    def force_path(self, path: int) -> None:
+        """Testing aid: 0 auto, 1 blocked u32, 2 blocked u64, 3 generic, 4 small batched."""
+        st = load_library().mcl_force_path(self.handle, path)
+        if st != MCL_OK:
+            raise MclError(st, "mcl_force_path")
+
+    def set_timing(self, enable: bool = True) -> None:
+        load_library().mcl_set_timing(self.handle, 1 if enable else 0)
+
+    def last_kernel_time_ms(self) -> tuple[float, float]:
+        k, c = ctypes.c_float(), ctypes.c_float()
+        load_library().mcl_last_kernel_time(self.handle, ctypes.byref(k), ctypes.byref(c))
+        return k.value, c.value

@@ -1,0 +1,340 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, bit-exact.
+
+Integer costs, so (index, makespan, mapping) must be identical for every epoch. Run on a
+B200 with ``pytest -m gpu``.
+"""
+from __future__ import annotations
+
+import json
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+from conftest import cuda_available
+from paper_conf_cluster_ajipbf15_b200 import workloads
+from paper_conf_cluster_ajipbf15_b200.mcl import MCL_E_INVAL, MCL_E_RANGE, Mapper, MclError
+
+pytestmark = pytest.mark.gpu
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    if not cuda_available():
+        pytest.fail("no CUDA device: the -m gpu tests must run on a GPU box")
+    import torch
+
+    return torch
+
+
+@pytest.fixture(scope="module")
+def mapper(torch_cuda):
+    m = Mapper(0)
+    yield m
+    m.close()
+
+
+def to_dev(torch, a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def run_gpu(torch, mp, K, X, path=0):
+    mp.force_path(path)
+    try:
+        idx, mapping, ms = mp.map_queues(to_dev(torch, K), to_dev(torch, X))
+    finally:
+        mp.force_path(0)
+    return idx.cpu().numpy(), mapping.cpu().numpy(), ms.cpu().numpy()
+
+
+def assert_same(got, want, ctx=""):
+    gi, gmp, gms = got
+    wi, wms, wmp = want
+    bad = np.nonzero((gi != wi) | (gms != wms))[0]
+    assert bad.size == 0, f"{ctx}: {bad.size} epochs differ, first {bad[:5]}: gpu {gi[bad[:5]]}/{gms[bad[:5]]} oracle {wi[bad[:5]]}/{wms[bad[:5]]}"
+    assert (gmp == wmp).all(), ctx
+
+
+# ------------------------------------------------------------------ hand cases ---------
+def _hand_cases():
+    with open(os.path.join(GOLDEN, "hand_cases.json")) as f:
+        return json.load(f)["cases"]
+
+
+@pytest.mark.parametrize("case", _hand_cases(), ids=lambda c: c["name"])
+@pytest.mark.parametrize("path", [0, 1, 2, 3])
+def test_hand_cases_gpu(torch_cuda, mapper, case, path):
+    K = np.array(case["K"], dtype=np.uint64)[None]
+    X = np.array(case["X"], dtype=np.uint64)[None]
+    Q, D = K.shape[1:]
+    if path in (1, 2) and not (Q >= 3 and 2 <= D <= 8):
+        pytest.skip("blocked kernel needs Q >= 3, 2 <= D <= 8")
+    gi, gmp, gms = run_gpu(torch_cuda, mapper, K, X, path)
+    assert int(gi[0]) == case["index"] and int(gms[0]) == case["makespan"]
+    assert list(gmp[0]) == case["mapping"]
+
+
+# --------------------------------------------------- random shapes, every kernel path --
+SHAPES = [(q, d) for q in range(1, 8) for d in range(1, 9) if d**q <= 300_000]
+
+
+@pytest.mark.parametrize("Q,D", SHAPES)
+def test_random_shapes_all_paths(torch_cuda, mapper, Q, D):
+    E = 64 if D**Q <= 5000 else 8
+    for seed, maker in ((10 * Q + D, workloads.random_tables), (1000 + 10 * Q + D, workloads.small_int_tables)):
+        K, X = maker(seed, E, Q, D)
+        want = oracle.oracle_map(K, X)
+        paths = [0, 3]
+        if Q >= 3 and 2 <= D <= 8:
+            paths += [1, 2]
+        for p in paths:
+            assert_same(run_gpu(torch_cuda, mapper, K, X, p), want, f"Q={Q} D={D} path={p} {maker.__name__}")
+
+
+def test_generic_large_d(torch_cuda, mapper):
+    for Q, D in ((2, 16), (3, 16), (4, 12), (5, 9), (4, 10)):
+        K, X = workloads.random_tables(7 * Q + D, 3, Q, D)
+        assert_same(run_gpu(torch_cuda, mapper, K, X), oracle.oracle_map(K, X), f"Q={Q} D={D}")
+
+
+def test_batched_equals_single_and_permutation(torch_cuda, mapper):
+    K, X = workloads.random_tables(99, 40, 6, 4, hi=1 << 10)
+    gi, gmp, gms = run_gpu(torch_cuda, mapper, K, X)
+    for e in (0, 7, 39):
+        si, smp, sms = run_gpu(torch_cuda, mapper, K[e:e + 1], X[e:e + 1])
+        assert si[0] == gi[e] and sms[0] == gms[e] and (smp[0] == gmp[e]).all()
+    perm = np.random.default_rng(3).permutation(40)
+    pi, _, pms = run_gpu(torch_cuda, mapper, K[perm], X[perm])
+    assert (pi == gi[perm]).all() and (pms == gms[perm]).all()
+
+
+# ------------------------------------------------------------- the five configs -------
+@pytest.mark.parametrize("name", list(workloads.NPB_RATIO))
+def test_cfg1_npb(torch_cuda, mapper, name):
+    K, X = workloads.cfg1_npb(name)
+    assert_same(run_gpu(torch_cuda, mapper, K, X), oracle.oracle_map(K, X), name)
+    assert_same(run_gpu(torch_cuda, mapper, K, X, 1), oracle.oracle_map(K, X), name)
+
+
+def test_cfg1_random_seeds(torch_cuda, mapper):
+    Ks, Xs = zip(*(workloads.cfg1_random(s) for s in range(2000)))
+    K, X = np.concatenate(Ks), np.concatenate(Xs)
+    want = oracle.oracle_map(K, X)
+    for p in (0, 1, 3):
+        assert_same(run_gpu(torch_cuda, mapper, K, X, p), want, f"cfg1 x2000 path {p}")
+
+
+def test_cfg2_full(torch_cuda, mapper):
+    K, X = workloads.cfg2()
+    assert_same(run_gpu(torch_cuda, mapper, K, X), oracle.oracle_map(K, X), "cfg2")
+    assert mapper.launch_info()["path"] == "blocked_u32"
+
+
+def test_cfg3_full(torch_cuda, mapper):
+    K, X = workloads.cfg3()
+    want = oracle.oracle_map(K, X)
+    assert_same(run_gpu(torch_cuda, mapper, K, X), want, "cfg3")
+    assert mapper.launch_info()["path"] == "small_batched"
+    # the paper's two regimes (Fig. 9): column-major -> (C, C); row-major -> the two GPUs
+    _, mp, _ = run_gpu(torch_cuda, mapper, K[:1000], X[:1000])
+    assert (mp[0::2] == 0).all()
+    assert (np.sort(mp[1::2], axis=1) == [1, 2]).all()
+
+
+def test_cfg3_ragged_and_unaligned(torch_cuda, mapper):
+    """Tail tiles (E not a multiple of the tile) and a 16-byte-misaligned base pointer take
+    the plain-load path instead of cp.async.bulk."""
+    torch = torch_cuda
+    K, X = workloads.cfg3(E=4097, seed=11)
+    want = oracle.oracle_map(K, X)
+    assert_same(run_gpu(torch, mapper, K, X), want, "ragged")
+    Kd = torch.zeros(4097 * 6 + 1, dtype=torch.uint64, device="cuda")
+    Xd = torch.zeros(4097 * 6 + 1, dtype=torch.uint64, device="cuda")
+    Kd[1:] = torch.from_numpy(K.reshape(-1)).cuda()
+    Xd[1:] = torch.from_numpy(X.reshape(-1)).cuda()
+    idx = torch.empty(4097, dtype=torch.uint64, device="cuda")
+    ms = torch.empty_like(idx)
+    mp = torch.empty((4097, 2), dtype=torch.uint8, device="cuda")
+    mapper.map_queues_into(Kd[1:].view(4097, 2, 3), Xd[1:].view(4097, 2, 3), idx, mp, ms)
+    assert_same((idx.cpu().numpy(), mp.cpu().numpy(), ms.cpu().numpy()), want, "unaligned")
+
+
+def _golden_full():
+    path = os.path.join(GOLDEN, "full_configs.json")
+    return json.load(open(path))["cases"] if os.path.exists(path) else {}
+
+
+@pytest.mark.parametrize("key", sorted(_golden_full()))
+def test_full_single_epoch_configs(torch_cuda, mapper, key):
+    """cfg4 / cfg5 at full size, in the launch configuration bench.py times, against the
+    oracle's full run (tests/golden/full_configs.json, scripts/make_golden.py)."""
+    case = _golden_full()[key]
+    K, X = workloads.make(case["config"], seed=case["seed"])
+    gi, gmp, gms = run_gpu(torch_cuda, mapper, K, X)
+    assert int(gi[0]) == case["index"] and int(gms[0]) == case["makespan"]
+    assert list(gmp[0]) == case["mapping"]
+
+
+@pytest.mark.parametrize("name,G", [("cfg4", 3), ("cfg4", 8), ("cfg5", 7), ("cfg5", 4096)])
+def test_full_size_shards_sampled(torch_cuda, name, G):
+    """At full size, sampled shards: the GPU's shard-local argmin equals the oracle's on the
+    same index sub-range (the oracle computes these one by one), and (when every shard is
+    run) the min over all shards equals the unsharded result."""
+    torch = torch_cuda
+    K, X = workloads.make(name)
+    Q, D = K.shape[1:]
+    N = D**Q
+    unit = D**3  # blocked kernel shards whole blocks of the 3 innermost digits
+    nb = N // unit
+    Kd, Xd = to_dev(torch, K), to_dev(torch, X)
+    ranks = list(range(G)) if G <= 16 else sorted({0, 1, G // 2, G - 2, G - 1} |
+                                                  set(np.random.default_rng(G).integers(0, G, 20).tolist()))
+    results = []
+    for r in ranks:
+        with Mapper(0, rank=r, world=G) as m:
+            idx, mp, ms = m.map_queues(Kd, Xd)
+            assert m.launch_info()["path"] == "blocked_u32"
+        results.append((int(ms[0].item()), int(idx[0].item())))
+        lo, hi = (nb * r // G) * unit, (nb * (r + 1) // G) * unit
+        assert lo <= results[-1][1] < hi
+        if hi - lo <= 6 * 10**8 and (G > 16 or r in (0, G // 2, G - 1)):
+            oi, oms, _ = oracle.oracle_map(K, X, lo=lo, hi=hi)
+            assert (int(oms[0]), int(oi[0])) == results[-1], f"shard {r}/{G}"
+    if len(ranks) == G:
+        with Mapper(0) as m:
+            idx, mp, ms = m.map_queues(Kd, Xd)
+        assert min(results) == (int(ms[0].item()), int(idx[0].item()))
+
+
+# ------------------------------------------------------------------- edge cases -------
+def test_u64_fallback_and_max_entries(torch_cuda, mapper):
+    """Bounds >= 2^32 need 64-bit loads: the u32 kernel detects it on the device and the
+    call reruns with the 64-bit kernel. Entries up to 2^48 - 1 are accepted."""
+    rng = np.random.default_rng(5)
+    K = rng.integers((1 << 47), (1 << 48) - 1, size=(5, 6, 4), dtype=np.uint64)
+    X = np.zeros_like(K)
+    X[:, :, 1:] = rng.integers(0, 1 << 20, size=(5, 6, 3), dtype=np.uint64)
+    want = oracle.oracle_map(K, X)
+    for p in (0, 1, 3):
+        assert_same(run_gpu(torch_cuda, mapper, K, X, p), want, f"u64 path {p}")
+    run_gpu(torch_cuda, mapper, K, X, 1)
+    assert mapper.launch_info()["path"] == "blocked_u64"
+    K = np.full((2, 5, 3), (1 << 48) - 1, dtype=np.uint64)
+    assert_same(run_gpu(torch_cuda, mapper, K, np.zeros_like(K)), oracle.oracle_map(K, np.zeros_like(K)), "max")
+
+
+def test_u32_boundary(torch_cuda, mapper):
+    """Bounds just below and just above 2^32."""
+    for total in ((1 << 32) - 1, 1 << 32):
+        K = np.zeros((1, 4, 3), dtype=np.uint64)
+        K[0, :, 0] = total // 4
+        K[0, 0, 0] += total - 4 * (total // 4)
+        K[0, :, 1:] = total // 4 + 1
+        X = np.zeros_like(K)
+        assert_same(run_gpu(torch_cuda, mapper, K, X, 1), oracle.oracle_map(K, X), str(total))
+
+
+def test_degenerate_ties(torch_cuda, mapper):
+    """All-equal (maximal ties), all-zero (every mapping ties at 0) and one-hot cheap device."""
+    for Q, D in ((8, 4), (12, 3), (6, 8), (5, 5)):
+        zeros = np.zeros((1, Q, D), np.uint64)
+        eq = np.full((1, Q, D), 7, np.uint64)
+        hot = np.full((1, Q, D), 1000, np.uint64)
+        hot[0, :, D - 1] = 1
+        for K in (zeros, eq, hot):
+            assert_same(run_gpu(torch_cuda, mapper, K, zeros), oracle.oracle_map(K, zeros), f"{Q}x{D}")
+
+
+def test_range_and_argument_errors(torch_cuda, mapper):
+    torch = torch_cuda
+    K = np.zeros((1, 4, 3), np.uint64)
+    K[0, 2, 1] = 1 << 48
+    for p in (0, 1, 3):
+        with pytest.raises(MclError) as e:
+            run_gpu(torch, mapper, K, np.zeros_like(K), p)
+        assert e.value.status == MCL_E_RANGE
+    # D^Q > 2^48
+    with pytest.raises(MclError) as e:
+        mapper.map_queues(np.zeros((1, 13, 16), np.uint64), np.zeros((1, 13, 16), np.uint64))
+    assert e.value.status == MCL_E_RANGE
+    with pytest.raises(MclError) as e:
+        mapper.map_queues(np.zeros((1, 2, 17), np.uint64), np.zeros((1, 2, 17), np.uint64))
+    assert e.value.status == MCL_E_INVAL
+    with pytest.raises(MclError) as e:
+        mapper.map_queues(np.zeros((1, 33, 1), np.uint64), np.zeros((1, 33, 1), np.uint64))
+    assert e.value.status == MCL_E_INVAL
+    # epochs == 0 is a no-op
+    from paper_conf_cluster_ajipbf15_b200.mcl import mcl_map_queues
+
+    assert mcl_map_queues(mapper.handle, 3, 3, 0, 0, 0, 0, None, 0) == 0
+    # the mapper keeps working after errors
+    K, X = workloads.cfg1_npb("FT")
+    assert_same(run_gpu(torch, mapper, K, X), oracle.oracle_map(K, X), "after errors")
+    # forced path that cannot run this shape
+    with pytest.raises(MclError) as e:
+        run_gpu(torch, mapper, np.zeros((1, 2, 3), np.uint64), np.zeros((1, 2, 3), np.uint64), 1)
+    assert e.value.status == MCL_E_INVAL
+
+
+def test_host_buffers_e2e(torch_cuda, mapper):
+    """Host (numpy, pageable) and pinned torch buffers are staged inside the call."""
+    torch = torch_cuda
+    K, X = workloads.cfg2(E=300, seed=21)
+    want = oracle.oracle_map(K, X)
+    idx, mp, ms = mapper.map_queues(K, X)
+    assert_same((idx, mp, ms), want, "numpy")
+    Kp = torch.from_numpy(K).pin_memory()
+    Xp = torch.from_numpy(X).pin_memory()
+    idx, mp, ms = mapper.map_queues(Kp, Xp)
+    assert_same((idx.numpy(), mp.numpy(), ms.numpy()), want, "pinned")
+    # mixed: device inputs, host outputs
+    i2 = np.empty(300, np.uint64)
+    m2 = np.empty(300, np.uint64)
+    p2 = np.empty((300, 8), np.uint8)
+    mapper.map_queues_into(to_dev(torch, K), to_dev(torch, X), i2, p2, m2)
+    assert_same((i2, p2, m2), want, "mixed")
+    # mapping output is optional
+    idx, mp, ms = mapper.map_queues(K, X, with_mapping=False)
+    assert mp is None and (idx == want[0]).all()
+
+
+def test_external_stream(torch_cuda):
+    torch = torch_cuda
+    s = torch.cuda.Stream()
+    K, X = workloads.cfg2(E=50, seed=4)
+    with Mapper(0, stream=s.cuda_stream) as m:
+        got = m.map_queues(to_dev(torch, K), to_dev(torch, X))
+    assert_same(tuple(t.cpu().numpy() for t in got), oracle.oracle_map(K, X), "stream")
+
+
+def test_nccl_single_rank_collective_path(torch_cuda):
+    """A 1-rank NCCL communicator runs the multi-GPU sequence (packed key, all-reduce,
+    decode) on one GPU; large makespans take the two-step lexicographic reduce."""
+    torch = torch_cuda
+    from paper_conf_cluster_ajipbf15_b200 import mcl
+
+    comm = mcl.mcl_comm_init(0, 1, 0, mcl.mcl_comm_unique_id())
+    try:
+        with Mapper(0, nccl_comm=comm, rank=0, world=1) as m:
+            K, X = workloads.cfg4(seed=4, Q=12)
+            got = m.map_queues(to_dev(torch, K), to_dev(torch, X))
+            info = m.launch_info()
+            assert info["allreduce"] and not info["two_step"]
+            assert_same(tuple(t.cpu().numpy() for t in got), oracle.oracle_map(K, X), "packed")
+            K = np.random.default_rng(1).integers(1 << 46, 1 << 47, size=(3, 9, 4), dtype=np.uint64)
+            X = np.zeros_like(K)
+            got = m.map_queues(to_dev(torch, K), to_dev(torch, X))
+            assert m.launch_info()["two_step"]
+            assert_same(tuple(t.cpu().numpy() for t in got), oracle.oracle_map(K, X), "two-step")
+    finally:
+        mcl.mcl_comm_destroy(comm)
+
+
+def test_probe(torch_cuda):
+    from paper_conf_cluster_ajipbf15_b200 import mcl
+
+    for op in range(5):
+        rate, per_clk, mhz = mcl.mcl_probe_int_rate(0, op)
+        assert rate > 1e12 and 30 < per_clk < 140 and 500 < mhz < 2500
