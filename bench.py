@@ -219,7 +219,9 @@ def main():
         dist.broadcast_object_list(obj, src=0)
         comm = mcl.mcl_comm_init(local, world, rank, obj[0])
 
-    stream = torch.cuda.current_stream(dev)
+    # a dedicated stream: the mapper, the L2 flush and the timing events all run on it
+    stream = torch.cuda.Stream(dev)
+    torch.cuda.set_stream(stream)
     # batched workloads: every rank runs its own full batch (weak scaling, no collective);
     # single-epoch workloads: the index space is sharded across ranks (strong scaling)
     Kd = torch.from_numpy(K).to(dev)
@@ -298,7 +300,8 @@ def main():
         sms = mcl.mcl_device_sms(local)
         clocks = clk.summary()
         max_mhz = clocks.get("sm_max_mhz") or 1965
-        mappings_per_launch = mappings_per_step / (world if is_batched(w) else world)
+        # per GPU and launch: the full batch (batched replicas) or this rank's index shard
+        mappings_per_launch = w["E"] * w["N"] if is_batched(w) else w["N"] / world
         if info["path"] in ("blocked_u32", "blocked_u64", "generic"):
             achieved = ALU_INSTR_PER_MAPPING * mappings_per_launch / (kern_mean / 1e3) / 1e12
             peak = ALU_LANES_PER_CLK_SM * sms * max_mhz * 1e6 / 1e12

@@ -1,6 +1,7 @@
 // kernels.h -- internal launch interface between the C-ABI host code (mcl.cpp) and the
 // sm_100a kernels. Not part of the public ABI (that is include/mcl.h).
 #pragma once
+#include <atomic>
 #include <cstddef>
 #include <cstdint>
 #include <cuda_runtime.h>
@@ -23,6 +24,27 @@ struct EpochOut {
 };
 
 constexpr int kBlockedMaxD = 8;  // register-blocked kernel instantiated for D = 2..8
+
+// Per-kernel, per-device cache of the dynamic shared-memory attribute already granted, so
+// the hot launch path does not re-issue cudaFuncSetAttribute every call.
+struct SmemAttrCache {
+  std::atomic<size_t> granted[64];
+  SmemAttrCache() {
+    for (auto& g : granted) g.store(0);
+  }
+};
+
+template <typename F>
+cudaError_t ensure_smem(F* kernel, size_t smem, SmemAttrCache& cache) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::atomic<size_t>& g = cache.granted[dev & 63];
+  if (g.load(std::memory_order_relaxed) >= smem + 1) return cudaSuccess;
+  // always set it: the default 48 KB cap also counts the kernel's static shared memory
+  cudaError_t err = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (err == cudaSuccess) g.store(smem + 1, std::memory_order_relaxed);
+  return err;
+}
 
 // Register-blocked search (search_blocked.cu).
 struct BlockedArgs {

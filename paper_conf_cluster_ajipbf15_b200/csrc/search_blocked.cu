@@ -310,10 +310,9 @@ template <typename T, int D>
 static cudaError_t launch_blocked_t(const BlockedArgs& a, dim3 grid, int threads, size_t smem,
                                    cudaStream_t st) {
   auto k = search_blocked_kernel<T, D>;
-  {  // always: the default 48 KB cap also counts the kernel's static shared memory
-    cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (err != cudaSuccess) return err;
-  }
+  static SmemAttrCache cache;
+  cudaError_t err = ensure_smem(k, smem, cache);
+  if (err != cudaSuccess) return err;
   k<<<grid, threads, smem, st>>>(a);
   return cudaGetLastError();
 }
@@ -334,11 +333,18 @@ size_t blocked_smem_bytes(uint32_t Q, uint32_t D, bool wide, int threads, size_t
 namespace {
 template <typename T, int D>
 int occ_t(int threads, size_t smem) {
+  // cache the last (threads, smem) query: the launch path asks the same question every call
+  static std::atomic<uint64_t> last{0};
+  const uint64_t key = ((uint64_t)threads << 40) | ((uint64_t)smem << 8);
+  const uint64_t hit = last.load(std::memory_order_relaxed);
+  if (hit && (hit & ~0xffull) == key) return (int)(hit & 0xff);
   int n = 0;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, search_blocked_kernel<T, D>, threads, smem) !=
       cudaSuccess)
     return 1;
-  return n < 1 ? 1 : n;
+  n = n < 1 ? 1 : (n > 255 ? 255 : n);
+  last.store(key | (uint64_t)n, std::memory_order_relaxed);
+  return n;
 }
 }  // namespace
 

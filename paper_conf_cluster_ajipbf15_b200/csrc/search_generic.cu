@@ -117,11 +117,9 @@ size_t generic_smem_bytes(uint32_t Q, uint32_t D, int threads) {
 
 cudaError_t launch_generic(const GenericArgs& a, dim3 grid, int threads, size_t smem,
                            cudaStream_t st) {
-  {  // always: the default 48 KB cap also counts the kernel's static shared memory
-    cudaError_t err = cudaFuncSetAttribute(search_generic_kernel,
-                                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (err != cudaSuccess) return err;
-  }
+  static SmemAttrCache cache;
+  cudaError_t err = ensure_smem(search_generic_kernel, smem, cache);
+  if (err != cudaSuccess) return err;
   search_generic_kernel<<<grid, threads, smem, st>>>(a);
   return cudaGetLastError();
 }

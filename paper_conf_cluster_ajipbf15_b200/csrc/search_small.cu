@@ -171,17 +171,26 @@ namespace {
 template <int Q, int D>
 cudaError_t launch_small_t(const SmallArgs& a, int num_sms, cudaStream_t st, int* grid_out,
                            int* threads_out) {
-  const int threads = 256;
+  // tile = one epoch per thread; tiny batches (cfg1: one epoch) get a single warp
+  const int threads = a.E >= 256 ? 256 : (int)((a.E + 31) / 32 * 32);
   const size_t smem = (size_t)4 * threads * Q * D * 8;  // 2 stages x (K, X)
   auto k = search_small_kernel<Q, D>;
-  {  // always: the default 48 KB cap also counts the kernel's static shared memory
-    cudaError_t err = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (err != cudaSuccess) return err;
-  }
-  int per_sm = 0;
-  cudaError_t err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, threads, smem);
+  static SmemAttrCache cache;
+  cudaError_t err = ensure_smem(k, smem, cache);
   if (err != cudaSuccess) return err;
-  if (per_sm < 1) per_sm = 1;
+  static std::atomic<int> occ256[64];  // CTAs per SM at 256 threads, per device (0 = unknown)
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int per_sm = 1;
+  if (threads == 256) {
+    per_sm = occ256[dev & 63].load(std::memory_order_relaxed);
+    if (per_sm == 0) {
+      err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, threads, smem);
+      if (err != cudaSuccess) return err;
+      if (per_sm < 1) per_sm = 1;
+      occ256[dev & 63].store(per_sm, std::memory_order_relaxed);
+    }
+  }
   const uint64_t ntiles = (a.E + threads - 1) / threads;
   uint64_t grid = (uint64_t)num_sms * per_sm;
   if (grid > ntiles) grid = ntiles;

@@ -1,0 +1,21 @@
+"""Run one workload through the mapper a few times (for ncu / compute-sanitizer runs)."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+from paper_conf_cluster_ajipbf15_b200 import Mapper, workloads  # noqa: E402
+
+name = sys.argv[1] if len(sys.argv) > 1 else "cfg5"
+reps = int(sys.argv[2]) if len(sys.argv) > 2 else 3
+kw = {}
+if len(sys.argv) > 3:  # optional epochs override for batched configs (sanitizer runs)
+    kw["E"] = int(sys.argv[3])
+K, X = workloads.make(name, **kw)
+Kd, Xd = torch.from_numpy(K).cuda(), torch.from_numpy(X).cuda()
+with Mapper(0) as m:
+    for _ in range(reps):
+        idx, mp, ms = m.map_queues(Kd, Xd)
+    torch.cuda.synchronize()
+    print(name, m.launch_info(), int(idx[0]), int(ms[0]))
