@@ -6,6 +6,9 @@
 // from CUDA events on the launching stream. Op kinds:
 //   0 VIMNMX (2-input min/max)   1 VIMNMX3 (3-input)   2 IADD3   3 IMAD
 //   4 VIMNMX3 + IMAD interleaved (are the ALU and FMA pipes issued concurrently?)
+//   5 IMAD.HI (signed, opaque multiplier): the sign-mask step of an FMA-pipe max
+//   6 max on the FMA pipe (IMAD, IMAD.HI, IMAD: 3 instructions per max) interleaved
+//     1:1 with VIMNMX on the ALU pipe
 #include "kernels.h"
 
 namespace mcl {
@@ -14,9 +17,25 @@ namespace {
 constexpr int kRegs = 16;
 constexpr int kIters = 4096;
 
+__device__ __forceinline__ int32_t mulhi_s32(int32_t a, int32_t b) {
+  int32_t r;
+  asm volatile("mul.hi.s32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+  return r;
+}
+
+// max(a, b) for a, b < 2^31 on the FMA pipe: nd = b - a, m = sign mask of nd, r = b + nd*m
+__device__ __forceinline__ uint32_t max_fma(uint32_t a, uint32_t b, int32_t one, int32_t neg1) {
+  int32_t nd, r;
+  asm("mad.lo.s32 %0, %1, %2, %3;" : "=r"(nd) : "r"((int32_t)a), "r"(neg1), "r"((int32_t)b));
+  const int32_t m = mulhi_s32(nd, one);
+  asm("mad.lo.s32 %0, %1, %2, %3;" : "=r"(r) : "r"(nd), "r"(m), "r"((int32_t)b));
+  return (uint32_t)r;
+}
+
 template <int OP>
 __global__ void __launch_bounds__(256) probe_kernel(uint32_t* out, uint32_t seed,
                                                     unsigned long long* cyc) {
+  const int32_t one = (int32_t)(seed >> 1), neg1 = -one;  // seed == 3: opaque 1 and -1
   uint32_t r[kRegs], s[kRegs];
 #pragma unroll
   for (int i = 0; i < kRegs; ++i) {
@@ -36,12 +55,17 @@ __global__ void __launch_bounds__(256) probe_kernel(uint32_t* out, uint32_t seed
         r[i] = __vimin3_u32(a, b, c);
         s[i] = s[i] * s[(i + 1) % kRegs] + s[(i + 3) % kRegs];
       }
+      if (OP == 5) r[i] = (uint32_t)mulhi_s32((int32_t)a, (int32_t)b);
+      if (OP == 6) {
+        r[i] = max(a, b);
+        s[i] = max_fma(s[i], s[(i + 1) % kRegs], one, neg1);  // throughput only
+      }
     }
   }
   const long long t1 = clock64();
   uint32_t acc = 0;
 #pragma unroll
-  for (int i = 0; i < kRegs; ++i) acc ^= r[i] ^ (OP == 4 ? s[i] : 0u);
+  for (int i = 0; i < kRegs; ++i) acc ^= r[i] ^ ((OP == 4 || OP == 6) ? s[i] : 0u);
   if (acc == 0x12345678u) out[0] = acc;
   if (threadIdx.x == 0) atomicMax(cyc, (unsigned long long)(t1 - t0));
 }
@@ -69,7 +93,8 @@ cudaError_t run(int sms, cudaStream_t st, double* rate, double* per_clk, double*
     unsigned long long c = 0;
     cudaEventElapsedTime(&ms, e0, e1);
     err = cudaMemcpy(&c, cyc, 8, cudaMemcpyDeviceToHost);
-    const double ops_per_thread = (double)kIters * kRegs * (OP == 4 ? 2 : 1);
+    // lane-ops: op 4 counts both instructions; op 6 counts 1 ALU max + 1 FMA-pipe max
+    const double ops_per_thread = (double)kIters * kRegs * ((OP == 4 || OP == 6) ? 2 : 1);
     *rate = (double)blocks * threads * ops_per_thread / (ms * 1e-3);
     *per_clk = (double)ctas_per_sm * threads * ops_per_thread / (double)c;
     *mhz = (double)c / (ms * 1e3);
@@ -90,6 +115,8 @@ cudaError_t probe_alu(int op, int sms, cudaStream_t st, double* rate, double* pe
     case 2: return run<2>(sms, st, rate, per_clk, mhz);
     case 3: return run<3>(sms, st, rate, per_clk, mhz);
     case 4: return run<4>(sms, st, rate, per_clk, mhz);
+    case 5: return run<5>(sms, st, rate, per_clk, mhz);
+    case 6: return run<6>(sms, st, rate, per_clk, mhz);
     default: return cudaErrorInvalidValue;
   }
 }

@@ -28,6 +28,11 @@
 
 namespace mcl {
 
+#ifndef MCL_SUPER_MAX_D
+#define MCL_SUPER_MAX_D 5
+#endif
+constexpr int kSuperMaxD = MCL_SUPER_MAX_D;  // super-block path for u32 and D <= this
+
 namespace {
 
 // Adds routed to the FMA pipe (IMAD) so the ALU pipe is left for min/max: `one` is a
@@ -49,27 +54,45 @@ __device__ __forceinline__ uint64_t max3(uint64_t a, uint64_t b, uint64_t c) { r
 __device__ __forceinline__ uint64_t min2(uint64_t a, uint64_t b) { return a < b ? a : b; }
 __device__ __forceinline__ uint64_t min3(uint64_t a, uint64_t b, uint64_t c) { return min2(a, min2(b, c)); }
 
-// Shared-memory layout of the per-epoch tables (T = uint32_t or uint64_t).
-//   in[7][D]      : A, B, C, A+B, A+C, B+C, A+B+C of the three inner queues
-//   V[O][D][D]    : one-hot outer vectors, O = Q - 3
-// Enumerate the D^3 leaves of one block in increasing index order, calling f(leaf, ms).
-template <typename T, int D, typename F>
-__device__ __forceinline__ void for_each_leaf(const T (&P)[D], const T* __restrict__ in,
-                                              uint32_t one, F&& f) {
+// Per-block sums of the prefix loads P with the inner queues' costs (A, B, C = rows
+// Q-3, Q-2, Q-1 of the composed cost table):
+//   a = P+A, b = P+B, c = P+C, ab = P+A+B, ac = P+A+C, bc = P+B+C, abc = P+A+B+C.
+// Shared-memory table `in[7][D]` holds A, B, C, A+B, A+C, B+C, A+B+C.
+template <typename T, int D>
+struct Sums {
+  T a[D], b[D], c[D], ab[D], ac[D], bc[D], abc[D];
+};
+
+template <typename T, int D>
+__device__ __forceinline__ void make_sums(Sums<T, D>& s, const T (&P)[D], const T* __restrict__ in,
+                                          uint32_t one) {
+#pragma unroll
+  for (int d = 0; d < D; ++d) {
+    s.a[d] = add_f(P[d], in[0 * D + d], one);
+    s.b[d] = add_f(P[d], in[1 * D + d], one);
+    s.c[d] = add_f(P[d], in[2 * D + d], one);
+    s.ab[d] = add_f(P[d], in[3 * D + d], one);
+    s.ac[d] = add_f(P[d], in[4 * D + d], one);
+    s.bc[d] = add_f(P[d], in[5 * D + d], one);
+    s.abc[d] = add_f(P[d], in[6 * D + d], one);
+  }
+}
+
+template <typename T, int D>
+__device__ __forceinline__ T max_of(const T (&P)[D]) {
   T M = P[0];
 #pragma unroll
   for (int d = 1; d < D; ++d) M = max2(M, P[d]);
-  T PA[D], PB[D], PCM[D], PAB[D], PAC[D], PBC[D], PABC[D];
+  return M;
+}
+
+// Enumerate the D^3 leaves of one block in increasing index order, calling f(leaf, ms).
+// M = max_d P[d] (prefix makespan).
+template <typename T, int D, typename F>
+__device__ __forceinline__ void for_each_leaf(const Sums<T, D>& s, T M, F&& f) {
+  T PCM[D];
 #pragma unroll
-  for (int d = 0; d < D; ++d) {
-    PA[d] = add_f(P[d], in[0 * D + d], one);
-    PB[d] = add_f(P[d], in[1 * D + d], one);
-    PCM[d] = max2(M, add_f(P[d], in[2 * D + d], one));
-    PAB[d] = add_f(P[d], in[3 * D + d], one);
-    PAC[d] = add_f(P[d], in[4 * D + d], one);
-    PBC[d] = add_f(P[d], in[5 * D + d], one);
-    PABC[d] = add_f(P[d], in[6 * D + d], one);
-  }
+  for (int d = 0; d < D; ++d) PCM[d] = max2(M, s.c[d]);
 #pragma unroll
   for (int i = 0; i < D; ++i)
 #pragma unroll
@@ -77,22 +100,22 @@ __device__ __forceinline__ void for_each_leaf(const T (&P)[D], const T* __restri
 #pragma unroll
       for (int k = 0; k < D; ++k) {
         T v;
-        if (i != j && i != k && j != k) v = max3(PA[i], PB[j], PCM[k]);
-        else if (i == j && j != k) v = max2(PAB[i], PCM[k]);
-        else if (i == k && i != j) v = max3(PAC[i], PB[j], M);
-        else if (j == k && i != j) v = max3(PA[i], PBC[j], M);
-        else v = max2(M, PABC[i]);
+        if (i != j && i != k && j != k) v = max3(s.a[i], s.b[j], PCM[k]);
+        else if (i == j && j != k) v = max2(s.ab[i], PCM[k]);
+        else if (i == k && i != j) v = max3(s.ac[i], s.b[j], M);
+        else if (j == k && i != j) v = max3(s.a[i], s.bc[j], M);
+        else v = max2(M, s.abc[i]);
         f((i * D + j) * D + k, v);
       }
 }
 
 // Minimum makespan over one block, folded two leaves per three-input min.
 template <typename T, int D>
-__device__ __forceinline__ T block_eval(const T (&P)[D], const T* __restrict__ in, uint32_t one) {
+__device__ __forceinline__ T block_eval(const Sums<T, D>& s, T M) {
   constexpr T kMax = ~T(0);
   T acc[4] = {kMax, kMax, kMax, kMax};
   T pend = kMax;
-  for_each_leaf<T, D>(P, in, one, [&](int leaf, T v) {
+  for_each_leaf<T, D>(s, M, [&](int leaf, T v) {
     if (leaf & 1) {
       acc[(leaf >> 1) & 3] = min3(acc[(leaf >> 1) & 3], pend, v);
     } else {
@@ -105,15 +128,50 @@ __device__ __forceinline__ T block_eval(const T (&P)[D], const T* __restrict__ i
   return g;
 }
 
+template <typename T, int D>
+__device__ __forceinline__ T block_eval(const T (&P)[D], const T* __restrict__ in, uint32_t one) {
+  Sums<T, D> s;
+  make_sums<T, D>(s, P, in, one);
+  return block_eval<T, D>(s, max_of<T, D>(P));
+}
+
 // Lowest leaf of the block whose makespan equals `target` (the block is known to hold one).
 template <typename T, int D>
 __device__ __forceinline__ uint32_t block_first(const T (&P)[D], const T* __restrict__ in,
                                                 uint32_t one, T target) {
+  Sums<T, D> s;
+  make_sums<T, D>(s, P, in, one);
   uint32_t first = 0xffffffffu;
-  for_each_leaf<T, D>(P, in, one, [&](int leaf, T v) {
+  for_each_leaf<T, D>(s, max_of<T, D>(P), [&](int leaf, T v) {
     first = (v == target && first == 0xffffffffu) ? (uint32_t)leaf : first;
   });
   return first;
+}
+
+// A SUPER-BLOCK: the D blocks x = 0..D-1 of the fourth-innermost digit (queue Q-4) with
+// the same outer prefix `base`. Only device x's load changes between them, so the sums of
+// the other devices are shared and the block loop is unrolled with static x (used for
+// small D, where a D^3 block alone is too short to amortise its setup).
+template <typename T, int D>
+__device__ __forceinline__ void superblock_eval(const T (&base)[D], const T* __restrict__ in,
+                                                const T* __restrict__ c4, uint32_t one, T (&g)[D]) {
+  Sums<T, D> sb;
+  make_sums<T, D>(sb, base, in, one);
+  const T Mb = max_of<T, D>(base);
+#pragma unroll
+  for (int x = 0; x < D; ++x) {
+    const T cx = c4[x];
+    Sums<T, D> s = sb;
+    s.a[x] = add_f(sb.a[x], cx, one);
+    s.b[x] = add_f(sb.b[x], cx, one);
+    s.c[x] = add_f(sb.c[x], cx, one);
+    s.ab[x] = add_f(sb.ab[x], cx, one);
+    s.ac[x] = add_f(sb.ac[x], cx, one);
+    s.bc[x] = add_f(sb.bc[x], cx, one);
+    s.abc[x] = add_f(sb.abc[x], cx, one);
+    const T M = max2(Mb, add_f(base[x], cx, one));
+    g[x] = block_eval<T, D>(s, M);
+  }
 }
 
 template <typename T, int D>
@@ -147,10 +205,11 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
   const uint32_t Q = a.Q;
   const int O = (int)Q - 3;  // outer queues (>= 0)
   const int nthr = blockDim.x, tid = threadIdx.x;
-  // layout: C64[Q*D] u64 | in[7*D] T | V[O*D*D] T | red[32] Cand | dig[(O-1)*nthr] u8
+  // layout: C64[Q*D] u64 | in[8*D] T | V[O*D*D] T | red[32] Cand | dig[(O-1)*nthr] u8
+  // (in[0..7) = inner sums, in[7] = composed costs of queue Q-4)
   uint64_t* C64 = reinterpret_cast<uint64_t*>(smem_raw);
   T* in = reinterpret_cast<T*>(C64 + Q * D);
-  T* V = in + 7 * D;
+  T* V = in + 8 * D;
   Cand* red = reinterpret_cast<Cand*>(
       reinterpret_cast<unsigned char*>(smem_raw) + a.off_red);
   uint8_t* dig = reinterpret_cast<uint8_t*>(smem_raw) + a.off_dig;
@@ -158,6 +217,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
   if (threadIdx.x < D) zero[threadIdx.x] = 0;
   __shared__ int s_bad;
   __shared__ uint64_t s_ub;
+  constexpr bool kSuper = (sizeof(T) == 4 && D <= kSuperMaxD);
 
   for (uint64_t e = blockIdx.y; e < a.E; e += gridDim.y) {
     // ---- a1: cost composition C = K + X, range check, bound UB = sum_q max_d C ----
@@ -203,6 +263,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
       in[5 * D + t] = (T)(B + Cc);
       in[6 * D + t] = (T)(A + B + Cc);
     }
+    for (int t = tid; t < D; t += nthr) in[7 * D + t] = (O >= 1) ? (T)C64[(O - 1) * D + t] : (T)0;
     for (int t = tid; t < O * D * D; t += nthr) {
       const int q = t / (D * D), x = (t / D) % D, d = t % D;
       V[t] = (d == x) ? (T)C64[q * D + x] : (T)0;
@@ -225,6 +286,8 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
         // digit x = queue O-1 runs fastest; queues 0..O-2 are the odometer in smem.
         // Q == 3 (O == 0): a single block whose prefix is the zero vector.
         const T* Vx = (O >= 1) ? V + (size_t)(O - 1) * D * D : zero;
+        // composed costs of queue O-1 (the x digit), for the super-block path
+        const T* c4 = (O >= 1) ? in + 7 * D : zero;
         uint32_t x = (uint32_t)(b0 % D);
         uint64_t hi = b0 / D;
         T base[D];
@@ -240,6 +303,22 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
         }
         uint64_t blk = b0;
         while (true) {
+          if (kSuper && x == 0 && nleft >= (uint64_t)D) {
+            T g[D];
+            superblock_eval<T, D>(base, in, c4, one, g);
+            T gs = g[0];
+#pragma unroll
+            for (int t = 1; t < D; ++t) gs = min2(gs, g[t]);
+            if (gs < best) {  // rare: locate the first block holding the new minimum
+              best = gs;
+#pragma unroll
+              for (int t = D - 1; t >= 0; --t)
+                if (g[t] == gs) best_blk = blk + t;
+            }
+            x = D;
+            nleft -= D;
+            blk += D;
+          }
           for (; x < (uint32_t)D && nleft; ++x, --nleft, ++blk) {
             T P[D], vx[D];
             load_vec<T, D>(vx, Vx + x * D);
@@ -321,7 +400,7 @@ size_t blocked_smem_bytes(uint32_t Q, uint32_t D, bool wide, int threads, size_t
                           size_t* off_dig) {
   const size_t tsz = wide ? 8 : 4;
   const int O = (int)Q - 3;
-  size_t off = (size_t)Q * D * 8 + 7 * D * tsz + (size_t)(O > 0 ? O : 0) * D * D * tsz;
+  size_t off = (size_t)Q * D * 8 + 8 * D * tsz + (size_t)(O > 0 ? O : 0) * D * D * tsz;
   off = (off + 15) & ~size_t(15);
   *off_red = off;
   off += 32 * sizeof(Cand);
