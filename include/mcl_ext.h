@@ -21,8 +21,9 @@ extern "C" {
    mcl_map_queues call on h. Events are recorded on the stream the kernel is launched on. */
 mcl_status_t mcl_set_timing(mcl_mapper_t* h, int enable);
 
-/* Device time in milliseconds of the main search kernel of the last call (timing enabled),
-   and of the whole device-side sequence of that call (search + reduce + decode). */
+/* Device time in milliseconds of the main search kernel of the last call (timing >= 1),
+   and of the whole device-side sequence of that call, staging copies included (timing 2;
+   else 0). enable: 0 = off, 1 = search kernel only (two events), 2 = kernel and call. */
 mcl_status_t mcl_last_kernel_time(const mcl_mapper_t* h, float* kernel_ms, float* call_ms);
 
 /*

@@ -12,6 +12,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -123,10 +124,10 @@ struct mcl_mapper {
   DevBuf in_k, in_x, out_idx, out_ms, out_map;  // staging for host pointers
   uint32_t* flags_host = nullptr;               // host-mapped status word
   uint32_t* flags_dev = nullptr;
-  bool timing = false;
+  int timing = 0;               // 0 off, 1 search kernel, 2 search kernel + whole call
+  bool timing_pending = false;  // events recorded, elapsed times not read yet
   int force_path = 0;
   cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
-  float kernel_ms = 0.f, call_ms = 0.f;
   int64_t info[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   std::string last_err;
 };
@@ -326,7 +327,9 @@ mcl_status_t mcl_last_launch_info(const mcl_mapper_t* h, int64_t info[8]) {
 
 mcl_status_t mcl_set_timing(mcl_mapper_t* h, int enable) {
   if (!h) return MCL_E_INVAL;
-  h->timing = enable != 0;
+  if (enable < 0 || enable > 2) return MCL_E_INVAL;
+  h->timing = enable;
+  h->timing_pending = false;
   return MCL_OK;
 }
 
@@ -338,8 +341,15 @@ mcl_status_t mcl_force_path(mcl_mapper_t* h, int path) {
 
 mcl_status_t mcl_last_kernel_time(const mcl_mapper_t* h, float* kernel_ms, float* call_ms) {
   if (!h) return MCL_E_INVAL;
-  if (kernel_ms) *kernel_ms = h->kernel_ms;
-  if (call_ms) *call_ms = h->call_ms;
+  float k = 0.f, c = 0.f;
+  if (h->timing_pending) {  // the call synchronised its stream, so the events are complete
+    DeviceGuard g(h->device);
+    if (cudaEventElapsedTime(&k, h->ev[0], h->ev[1]) != cudaSuccess) k = 0.f;
+    if (h->timing >= 2 && cudaEventElapsedTime(&c, h->ev[2], h->ev[3]) != cudaSuccess) c = 0.f;
+    cudaGetLastError();
+  }
+  if (kernel_ms) *kernel_ms = k;
+  if (call_ms) *call_ms = c;
   return MCL_OK;
 }
 
@@ -386,7 +396,7 @@ mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t ep
   uint64_t* o_ms = makespan;
   uint8_t* o_map = mapping;
   cudaStream_t s = h->stream;
-  if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[2], s), "cudaEventRecord");
+  if (h->timing >= 2) MCL_CUDA(h, cudaEventRecord(h->ev[2], s), "cudaEventRecord");
   if (!dk) {
     MCL_CUDA(h, h->in_k.ensure(in_bytes), "cudaMalloc(staging)");
     MCL_CUDA(h, cudaMemcpyAsync(h->in_k.p, cost_kernel, in_bytes, cudaMemcpyHostToDevice, s), "H2D");
@@ -457,8 +467,13 @@ mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t ep
       // batched epochs: smaller CTAs so every thread still walks >= 16 blocks
       threads = 256;
       if (epochs > 1) {
+        // batched epochs: smaller CTAs so every thread still walks >= kMinBlocks blocks
+        static const uint64_t kMinBlocks = [] {
+          const char* v = getenv("MCL_BATCH_MIN_BLOCKS");  // tuning knob (default 16)
+          return (uint64_t)((v && atoi(v) > 0) ? atoi(v) : 16);
+        }();
         const uint64_t per_epoch = hi - lo;
-        while (threads > 32 && per_epoch / threads < 16) threads >>= 1;
+        while (threads > 32 && per_epoch / threads < kMinBlocks) threads >>= 1;
       }
       mcl::BlockedArgs a{};
       a.Q = Q; a.D = D; a.E = epochs; a.K = K; a.X = X; a.rlo = lo; a.rhi = hi;
@@ -549,12 +564,9 @@ mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t ep
   if (!dm) MCL_CUDA(h, cudaMemcpyAsync(makespan, o_ms, epochs * 8, cudaMemcpyDeviceToHost, s), "D2H");
   if (mapping && !dmap)
     MCL_CUDA(h, cudaMemcpyAsync(mapping, o_map, epochs * Q, cudaMemcpyDeviceToHost, s), "D2H");
-  if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[3], s), "cudaEventRecord");
+  if (h->timing >= 2) MCL_CUDA(h, cudaEventRecord(h->ev[3], s), "cudaEventRecord");
   MCL_CUDA(h, cudaStreamSynchronize(s), "D2H");
-  if (h->timing) {
-    cudaEventElapsedTime(&h->kernel_ms, h->ev[0], h->ev[1]);
-    cudaEventElapsedTime(&h->call_ms, h->ev[2], h->ev[3]);
-  }
+  h->timing_pending = h->timing > 0;  // elapsed times are read lazily (mcl_last_kernel_time)
   return MCL_OK;
 }
 

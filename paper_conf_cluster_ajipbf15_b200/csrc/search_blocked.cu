@@ -271,17 +271,77 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
     __syncthreads();
 
     // ---- a2-a5: this thread's contiguous block range inside the rank's range ----
+    // Split points are aligned to whole CHUNKS (D^2 blocks on the super-block path) so the
+    // lanes of a warp walk chunks in lock-step; only the rank's two ends can be ragged.
     const uint64_t nb_rank = a.rhi - a.rlo;
     const uint64_t T_all = (uint64_t)gridDim.x * nthr;
     const uint64_t gt = (uint64_t)blockIdx.x * nthr + tid;
-    const uint64_t per = nb_rank / T_all, rem = nb_rank % T_all;
-    const uint64_t b0 = a.rlo + gt * per + (gt < rem ? gt : rem);
-    uint64_t nleft = per + (gt < rem ? 1 : 0);
+    const bool chunked = kSuper && O >= 2;
+    const uint64_t chunk = chunked ? (uint64_t)D * D : 1;
+    auto split = [&](uint64_t t) -> uint64_t {
+      if (t == 0) return a.rlo;
+      if (t >= T_all) return a.rhi;
+      const uint64_t per = nb_rank / T_all, rem = nb_rank % T_all;
+      uint64_t s = a.rlo + t * per + (t < rem ? t : rem);
+      s = s / chunk * chunk;
+      return s < a.rlo ? a.rlo : (s > a.rhi ? a.rhi : s);
+    };
+    const uint64_t b0 = split(gt);
+    uint64_t nleft = split(gt + 1) - b0;
 
     T best = ~T(0);
     uint64_t best_blk = kNone;
     const uint32_t one = a.one;
-    if (nleft) {
+    if (nleft && chunked) {
+      // Super-block path: queue O-1 = digit x (static, inside superblock_eval), queue
+      // O-2 = digit y (uniform loop), queues 0..O-3 = the chunk index, decoded by a loop
+      // whose trip count is the same for every lane (no divergent carries).
+      const T* c4 = in + 7 * D;
+      const T* Vy = V + (size_t)(O - 2) * D * D;
+      uint64_t blk = b0;
+      auto single = [&](uint64_t bk) {
+        T P[D];
+        prefix_of<T, D>(P, bk, O, V, one);
+        const T g = block_eval<T, D>(P, in, one);
+        if (g < best) {
+          best = g;
+          best_blk = bk;
+        }
+      };
+      for (; nleft && (blk % chunk) != 0; ++blk, --nleft) single(blk);
+      for (; nleft >= chunk; nleft -= chunk, blk += chunk) {
+        uint64_t ch = blk / chunk;
+        T base2[D];
+#pragma unroll
+        for (int d = 0; d < D; ++d) base2[d] = 0;
+        for (int q = O - 3; q >= 0; --q) {
+          const uint32_t dq = (uint32_t)(ch % D);
+          ch /= D;
+          const T* v = V + ((size_t)q * D + dq) * D;
+#pragma unroll
+          for (int d = 0; d < D; ++d) base2[d] = add_f(base2[d], v[d], one);
+        }
+        for (int y = 0; y < D; ++y) {
+          T base[D], vy[D];
+          load_vec<T, D>(vy, Vy + y * D);
+#pragma unroll
+          for (int d = 0; d < D; ++d) base[d] = add_f(base2[d], vy[d], one);
+          T g[D];
+          superblock_eval<T, D>(base, in, c4, one, g);
+          T gs = g[0];
+#pragma unroll
+          for (int t = 1; t < D; ++t) gs = min2(gs, g[t]);
+          if (gs < best) {  // rare: locate the first block holding the new minimum
+            best = gs;
+            const uint64_t bb = blk + (uint64_t)y * D;
+#pragma unroll
+            for (int t = D - 1; t >= 0; --t)
+              if (g[t] == gs) best_blk = bb + t;
+          }
+        }
+      }
+      for (; nleft; ++blk, --nleft) single(blk);
+    } else if (nleft) {
       {
         // digit x = queue O-1 runs fastest; queues 0..O-2 are the odometer in smem.
         // Q == 3 (O == 0): a single block whose prefix is the zero vector.
@@ -347,15 +407,39 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
       }
     }
     // ---- a5: lowest index inside the best block, then warp / CTA / epoch argmin ----
-    Cand c{kNone, kNone};
-    if (best_blk != kNone) {
-      T P[D];
-      prefix_of<T, D>(P, best_blk, O, V, one);
-      const uint32_t leaf = block_first<T, D>(P, in, one, best);
-      c.ms = (uint64_t)best;
-      c.idx = best_blk * (uint64_t)(D * D * D) + leaf;
+    // Thread ranges ascend with the thread id, so the CTA's lowest-index optimum belongs to
+    // the LOWEST thread whose best equals the CTA minimum; only that thread re-scans its
+    // best block (one block per CTA instead of one per thread).
+    __shared__ uint64_t s_gmin;
+    __shared__ uint32_t s_winner;
+    __shared__ Cand s_cand;
+    {
+      const uint64_t bv = (best_blk != kNone) ? (uint64_t)best : kNone;
+      uint64_t wmin = bv;
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) wmin = min(wmin, __shfl_xor_sync(0xffffffffu, wmin, off));
+      __syncthreads();  // `red` may still be read by a previous epoch's reduction
+      if ((tid & 31) == 0) red[tid >> 5].ms = wmin;
+      if (tid == 0) s_winner = 0xffffffffu;
+      __syncthreads();
+      if (tid == 0) {
+        uint64_t g = kNone;
+        for (int w = 0; w < (nthr + 31) / 32; ++w) g = min(g, red[w].ms);
+        s_gmin = g;
+        s_cand = Cand{kNone, kNone};
+      }
+      __syncthreads();
+      if (bv != kNone && bv == s_gmin) atomicMin(&s_winner, (uint32_t)tid);
+      __syncthreads();
+      if ((uint32_t)tid == s_winner) {
+        T P[D];
+        prefix_of<T, D>(P, best_blk, O, V, one);
+        const uint32_t leaf = block_first<T, D>(P, in, one, best);
+        s_cand = Cand{(uint64_t)best, best_blk * (uint64_t)(D * D * D) + leaf};
+      }
+      __syncthreads();
     }
-    c = block_min(c, red);
+    Cand c = s_cand;
     if (gridDim.x == 1) {
       if (tid == 0) write_epoch(a.out, e, Q, D, a.ibits, c, a.flags);
       continue;

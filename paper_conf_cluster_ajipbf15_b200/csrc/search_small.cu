@@ -4,8 +4,8 @@
 // The work per epoch is a handful of integer ops; the kernel is bound by HBM (96 B of
 // costs in, 18 B of results out per epoch at Q=2, D=3). A persistent grid streams tiles of
 // blockDim.x epochs: one elected thread moves a tile's K and X slabs global -> shared with
-// cp.async.bulk (the TMA bulk-copy engine, SASS UBLKCP) completing on an mbarrier, double
-// buffered so the next tile is in flight while the current one is scored. Each thread then
+// cp.async.bulk (the TMA bulk-copy engine, SASS UBLKCP) completing on an mbarrier, six
+// stages deep so several tiles are in flight while the current one is scored. Each thread then
 // scores its epoch's D^Q mappings from shared memory with compile-time digits (so every
 // load index is static), in increasing index order with a strict '<' (lowest index wins
 // ties, BASELINE.json north_star), and writes its outputs coalesced.
@@ -65,19 +65,20 @@ struct Pow<0, D> {
 
 }  // namespace
 
+constexpr int kSmallStages = 6;  // tiles in flight per CTA (TMA bulk copies)
+
 template <int Q, int D>
-__global__ void __launch_bounds__(256) search_small_kernel(SmallArgs a, int use_tma) {
+__global__ void __launch_bounds__(128) search_small_kernel(SmallArgs a, int use_tma) {
   constexpr int QD = Q * D;
   constexpr int N = Pow<Q, D>::N;
+  constexpr bool kVec = (QD % 2) == 0;  // a row of QD u64 is a whole number of 16-B vectors
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  __shared__ __align__(8) uint64_t bar[2];
+  __shared__ __align__(8) uint64_t full[kSmallStages];
   const int TE = blockDim.x, tid = threadIdx.x;
-  uint64_t* sK[2];
-  uint64_t* sX[2];
-  sK[0] = reinterpret_cast<uint64_t*>(smem_raw);
-  sX[0] = sK[0] + (size_t)TE * QD;
-  sK[1] = sX[0] + (size_t)TE * QD;
-  sX[1] = sK[1] + (size_t)TE * QD;
+  const size_t slab = (size_t)TE * QD;  // u64 per array per stage
+  uint64_t* sbase = reinterpret_cast<uint64_t*>(smem_raw);
+  auto sK = [&](int s) { return sbase + (size_t)(2 * s) * slab; };
+  auto sX = [&](int s) { return sbase + (size_t)(2 * s + 1) * slab; };
 
   const uint64_t E = a.E;
   const uint64_t ntiles = (E + TE - 1) / TE;
@@ -85,49 +86,67 @@ __global__ void __launch_bounds__(256) search_small_kernel(SmallArgs a, int use_
   // caller's pointers are 16-byte aligned (use_tma)
   auto tile_tma = [&](uint64_t t) { return use_tma && (t + 1) * TE <= E; };
   auto issue = [&](uint64_t t, int s) {
-    const uint32_t bytes = (uint32_t)((size_t)TE * QD * 8);
+    const uint32_t bytes = (uint32_t)(slab * 8);
     fence_proxy_async();
-    mbar_expect_tx(&bar[s], 2 * bytes);
-    bulk_g2s(sK[s], a.K + t * TE * QD, bytes, &bar[s]);
-    bulk_g2s(sX[s], a.X + t * TE * QD, bytes, &bar[s]);
+    mbar_expect_tx(&full[s], 2 * bytes);
+    bulk_g2s(sK(s), a.K + t * slab, bytes, &full[s]);
+    bulk_g2s(sX(s), a.X + t * slab, bytes, &full[s]);
   };
   if (tid == 0) {
-    mbar_init(&bar[0], 1);
-    mbar_init(&bar[1], 1);
+    for (int s = 0; s < kSmallStages; ++s) mbar_init(&full[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  uint32_t phase[2] = {0, 0};
-  uint64_t t = blockIdx.x;
-  if (tid == 0 && t < ntiles && tile_tma(t)) issue(t, 0);
+  // prologue: up to kSmallStages of this CTA's tiles in flight
+  if (tid == 0) {
+    uint64_t t = blockIdx.x;
+    for (int s = 0; s < kSmallStages && t < ntiles; ++s, t += gridDim.x)
+      if (tile_tma(t)) issue(t, s);
+  }
+  uint32_t phase_bits = 0;  // bit s = parity to wait for on stage s
   bool bad = false;
-  for (int it = 0; t < ntiles; t += gridDim.x, ++it) {
-    const int s = it & 1;
-    const uint64_t tn = t + gridDim.x;
-    if (tid == 0 && tn < ntiles && tile_tma(tn)) issue(tn, s ^ 1);
+  int s = 0;
+  for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
     if (tile_tma(t)) {
-      mbar_wait(&bar[s], phase[s]);
-      phase[s] ^= 1u;
+      mbar_wait(&full[s], (phase_bits >> s) & 1u);
+      phase_bits ^= 1u << s;
     } else {
       const uint64_t n = (E - t * TE < (uint64_t)TE) ? E - t * TE : (uint64_t)TE;
       for (uint64_t j = tid; j < n * QD; j += TE) {
-        sK[s][j] = a.K[t * TE * QD + j];
-        sX[s][j] = a.X[t * TE * QD + j];
+        sK(s)[j] = a.K[t * slab + j];
+        sX(s)[j] = a.X[t * slab + j];
       }
       __syncthreads();
     }
     const uint64_t e = t * TE + tid;
     if (e < E) {
+      uint64_t kv[QD], xv[QD];
+      const uint64_t* k = sK(s) + (size_t)tid * QD;
+      const uint64_t* x = sX(s) + (size_t)tid * QD;
+      if (kVec) {  // 16-byte shared loads; a 48-B row stride keeps each quarter-warp conflict-free
+#pragma unroll
+        for (int j = 0; j < QD; j += 2) {
+          const ulonglong2 k2 = *reinterpret_cast<const ulonglong2*>(k + j);
+          const ulonglong2 x2 = *reinterpret_cast<const ulonglong2*>(x + j);
+          kv[j] = k2.x;
+          kv[j + 1] = k2.y;
+          xv[j] = x2.x;
+          xv[j + 1] = x2.y;
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < QD; ++j) {
+          kv[j] = k[j];
+          xv[j] = x[j];
+        }
+      }
       uint64_t C[Q][D];
-      const uint64_t* k = sK[s] + (size_t)tid * QD;
-      const uint64_t* x = sX[s] + (size_t)tid * QD;
 #pragma unroll
       for (int q = 0; q < Q; ++q)
 #pragma unroll
         for (int d = 0; d < D; ++d) {
-          const uint64_t kv = k[q * D + d], xv = x[q * D + d];
-          bad |= (kv >= kEntryLimit) | (xv >= kEntryLimit);
-          C[q][d] = kv + xv;  // a1: aggregate cost
+          bad |= (kv[q * D + d] >= kEntryLimit) | (xv[q * D + d] >= kEntryLimit);
+          C[q][d] = kv[q * D + d] + xv[q * D + d];  // a1: aggregate cost
         }
       uint64_t best = kNone;
       uint32_t bi = 0;
@@ -162,7 +181,10 @@ __global__ void __launch_bounds__(256) search_small_kernel(SmallArgs a, int use_
         }
       }
     }
-    __syncthreads();  // stage s is free for the prefetch issued next iteration
+    __syncthreads();  // stage s is consumed: refill it with this CTA's tile kSmallStages ahead
+    const uint64_t tn = t + (uint64_t)kSmallStages * gridDim.x;
+    if (tid == 0 && tn < ntiles && tile_tma(tn)) issue(tn, s);
+    s = (s + 1 == kSmallStages) ? 0 : s + 1;
   }
   if (__any_sync(0xffffffffu, bad) && (tid & 31) == 0) raise_flag(a.flags, kFlagRange);
 }
@@ -172,23 +194,23 @@ template <int Q, int D>
 cudaError_t launch_small_t(const SmallArgs& a, int num_sms, cudaStream_t st, int* grid_out,
                            int* threads_out) {
   // tile = one epoch per thread; tiny batches (cfg1: one epoch) get a single warp
-  const int threads = a.E >= 256 ? 256 : (int)((a.E + 31) / 32 * 32);
-  const size_t smem = (size_t)4 * threads * Q * D * 8;  // 2 stages x (K, X)
+  const int threads = a.E >= 128 ? 128 : (int)((a.E + 31) / 32 * 32);
+  const size_t smem = (size_t)kSmallStages * 2 * threads * Q * D * 8;
   auto k = search_small_kernel<Q, D>;
   static SmemAttrCache cache;
   cudaError_t err = ensure_smem(k, smem, cache);
   if (err != cudaSuccess) return err;
-  static std::atomic<int> occ256[64];  // CTAs per SM at 256 threads, per device (0 = unknown)
+  static std::atomic<int> occ128[64];  // CTAs per SM at 128 threads, per device (0 = unknown)
   int dev = 0;
   cudaGetDevice(&dev);
   int per_sm = 1;
-  if (threads == 256) {
-    per_sm = occ256[dev & 63].load(std::memory_order_relaxed);
+  if (threads == 128) {
+    per_sm = occ128[dev & 63].load(std::memory_order_relaxed);
     if (per_sm == 0) {
       err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, threads, smem);
       if (err != cudaSuccess) return err;
       if (per_sm < 1) per_sm = 1;
-      occ256[dev & 63].store(per_sm, std::memory_order_relaxed);
+      occ128[dev & 63].store(per_sm, std::memory_order_relaxed);
     }
   }
   const uint64_t ntiles = (a.E + threads - 1) / threads;
