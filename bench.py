@@ -39,6 +39,9 @@ UNIT = "mappings/s"
 ALU_LANES_PER_CLK_SM = 64       # B200 ALU pipe: 16 lanes x 4 SMSPs per SM per clock (measured: probe)
 ALU_INSTR_PER_MAPPING = 1.5     # floor: 1 VIMNMX forms the makespan + 1/2 VIMNMX3 folds it
 L2_FLUSH_BYTES = 256 << 20      # > 126 MB L2
+KERNEL_NAMES = {"blocked_u32": "search_blocked_kernel<u32, D>", "blocked_u64": "search_blocked_kernel<u64, D>",
+                "generic": "search_generic_kernel", "flat_u32": "search_flat_kernel<u32, D>",
+                "small_batched": "search_small_kernel<Q, D>"}
 
 
 def parse():
@@ -302,12 +305,12 @@ def main():
         max_mhz = clocks.get("sm_max_mhz") or 1965
         # per GPU and launch: the full batch (batched replicas) or this rank's index shard
         mappings_per_launch = w["E"] * w["N"] if is_batched(w) else w["N"] / world
-        if info["path"] in ("blocked_u32", "blocked_u64", "generic"):
+        if info["path"] in ("blocked_u32", "blocked_u64", "generic", "flat_u32"):
             achieved = ALU_INSTR_PER_MAPPING * mappings_per_launch / (kern_mean / 1e3) / 1e12
             peak = ALU_LANES_PER_CLK_SM * sms * max_mhz * 1e6 / 1e12
             roof = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tops/s",
                     "frac": achieved / peak, "traffic": traffic_from_profiles(args.workload),
-                    "kernel": f"search_blocked_kernel ({info['path']})", "kernel_ms": kern_mean,
+                    "kernel": KERNEL_NAMES.get(info["path"], info["path"]), "kernel_ms": kern_mean,
                     "algorithmic": f"{ALU_INSTR_PER_MAPPING} ALU lane-instructions per mapping x "
                                    f"{mappings_per_launch:.4g} mappings per launch",
                     "peak_basis": f"derived: {ALU_LANES_PER_CLK_SM} ALU lanes/clk/SM x {sms} SMs x "

@@ -113,7 +113,8 @@ const char* mcl_last_error_string(const mcl_mapper_t* h);
  * Introspection for tests and benchmarks (not needed to use the mapper).
  * mcl_last_launch_info fills, for the most recent successful mcl_map_queues call on h:
  *   info[0] = kernel path id (1 = register-blocked u32 search, 2 = register-blocked u64
- *             search, 3 = generic search, 4 = small batched (thread per epoch))
+ *             search, 3 = generic search, 4 = small batched (thread per epoch),
+ *             5 = register-blocked u32 over a flattened (epoch, block) space)
  *   info[1] = number of kernels launched by the call, info[2] = CTAs of the main kernel,
  *   info[3] = threads per CTA, info[4] = 1 if an NCCL all-reduce ran,
  *   info[5] = index bits of the packed key, info[6] = 1 if the two-step reduce ran.

@@ -76,6 +76,25 @@ size_t blocked_smem_bytes(uint32_t Q, uint32_t D, bool wide, int threads, size_t
 cudaError_t launch_blocked(const BlockedArgs& a, bool wide, dim3 grid, int threads, size_t smem,
                            cudaStream_t st);
 
+// Batched epochs over a flattened (epoch, block) space (search_flat.cu): u32 loads, whole
+// index space per epoch (no sharding), packed keys (index bits <= 32).
+struct FlatArgs {
+  uint32_t Q, D;
+  uint64_t E;
+  const uint64_t* K;
+  const uint64_t* X;
+  uint64_t nb;            // blocks of D^3 mappings per epoch
+  int ibits;
+  uint64_t* keys;         // [E], all ones on entry, self-resetting
+  uint64_t* done_blocks;  // [E], zero on entry, self-resetting
+  EpochOut out;
+  volatile uint32_t* flags;
+  uint32_t one;
+};
+bool flat_supported(uint32_t Q, uint32_t D, int ibits);
+size_t flat_smem_bytes(uint32_t Q, uint32_t D);
+cudaError_t launch_flat(const FlatArgs& a, int num_sms, cudaStream_t st, int* grid_out);
+
 // Generic search (search_generic.cu): any Q <= 32, D <= 16, 64-bit loads.
 struct GenericArgs {
   uint32_t Q, D;

@@ -121,6 +121,7 @@ struct mcl_mapper {
   DevBuf scratch;          // Cand per (epoch, CTA) when an epoch spans several CTAs
   DevBuf done;             // uint32 per epoch, zero between calls
   DevBuf key, pair, gms, cand;
+  DevBuf flat_keys, flat_done;  // flattened batched kernel: per-epoch key / block count
   DevBuf in_k, in_x, out_idx, out_ms, out_map;  // staging for host pointers
   uint32_t* flags_host = nullptr;               // host-mapped status word
   uint32_t* flags_dev = nullptr;
@@ -308,7 +309,8 @@ void mcl_mapper_destroy(mcl_mapper_t* h) {
   {
     DeviceGuard g(h->device);
     if (h->stream) cudaStreamSynchronize(h->stream);
-    for (DevBuf* b : {&h->scratch, &h->done, &h->key, &h->pair, &h->gms, &h->cand, &h->in_k,
+    for (DevBuf* b : {&h->scratch, &h->done, &h->key, &h->pair, &h->gms, &h->cand, &h->flat_keys,
+                      &h->flat_done, &h->in_k,
                       &h->in_x, &h->out_idx, &h->out_ms, &h->out_map})
       b->release();
     if (h->flags_host) cudaFreeHost(h->flags_host);
@@ -334,7 +336,7 @@ mcl_status_t mcl_set_timing(mcl_mapper_t* h, int enable) {
 }
 
 mcl_status_t mcl_force_path(mcl_mapper_t* h, int path) {
-  if (!h || path < 0 || path > 4) return MCL_E_INVAL;
+  if (!h || path < 0 || path > 5) return MCL_E_INVAL;
   h->force_path = path;
   return MCL_OK;
 }
@@ -439,12 +441,14 @@ mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t ep
   if (h->force_path) {
     const int f = h->force_path;
     const bool ok = (f == 3) || ((f == 1 || f == 2) && mcl::blocked_supported(Q, D)) ||
+                    (f == 5 && epochs > 1 && !shard_mode && !multi &&
+                     mcl::flat_supported(Q, D, mcl::index_bits_host(N))) ||
                     (f == 4 && !shard_mode && !multi && mcl::small_supported(Q, D));
     if (!ok) {
       h->last_err = "forced kernel path does not support this shape / sharding";
       return MCL_E_INVAL;
     }
-    path = f;
+    path = (f == 5) ? 1 : f;  // 5 = the flattened form of the blocked u32 kernel
   }
 
   int nlaunch = 0;
@@ -459,18 +463,37 @@ mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t ep
       int gx = 0;
       MCL_CUDA(h, mcl::launch_small(a, h->num_sms, s, &gx, &threads), "search_small launch");
       grid.x = gx;
+    } else if (path == 1 && epochs > 1 && !shard_mode && !multi &&
+               h->force_path == 5 &&
+               mcl::flat_supported(Q, D, ibits)) {
+      // batched epochs, whole index space: flattened (epoch, block) work distribution
+      mcl::FlatArgs a{};
+      a.Q = Q; a.D = D; a.E = epochs; a.K = K; a.X = X;
+      a.nb = N / ((uint64_t)D * D * D);
+      a.ibits = ibits; a.out = out; a.flags = h->flags_dev; a.one = 1;
+      if (h->flat_keys.cap < epochs * 8) {
+        MCL_CUDA(h, h->flat_keys.ensure(epochs * 8), "cudaMalloc(keys)");
+        MCL_CUDA(h, cudaMemset(h->flat_keys.p, 0xff, h->flat_keys.cap), "cudaMemset(keys)");
+      }
+      MCL_CUDA(h, h->flat_done.ensure(epochs * 8, true), "cudaMalloc(done_blocks)");
+      a.keys = (uint64_t*)h->flat_keys.p;
+      a.done_blocks = (uint64_t*)h->flat_done.p;
+      int gx = 0;
+      MCL_CUDA(h, mcl::launch_flat(a, h->num_sms, s, &gx), "search_flat launch");
+      grid.x = gx;
+      threads = 32;
+      path = 5;
     } else if (path == 1 || path == 2) {
       const bool wide = (path == 2);
       const uint64_t nb = N / ((uint64_t)D * D * D);
       uint64_t lo, hi;
       shard(nb, h->rank, h->world, &lo, &hi);
-      // batched epochs: smaller CTAs so every thread still walks >= 16 blocks
       threads = 256;
       if (epochs > 1) {
         // batched epochs: smaller CTAs so every thread still walks >= kMinBlocks blocks
         static const uint64_t kMinBlocks = [] {
-          const char* v = getenv("MCL_BATCH_MIN_BLOCKS");  // tuning knob (default 16)
-          return (uint64_t)((v && atoi(v) > 0) ? atoi(v) : 16);
+          const char* v = getenv("MCL_BATCH_MIN_BLOCKS");  // tuning knob (default 32)
+          return (uint64_t)((v && atoi(v) > 0) ? atoi(v) : 32);
         }();
         const uint64_t per_epoch = hi - lo;
         while (threads > 32 && per_epoch / threads < kMinBlocks) threads >>= 1;
@@ -530,7 +553,7 @@ mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t ep
       return MCL_E_RANGE;
     }
     if (flags & 2u) {  // some epoch's bound needs 64-bit loads: rerun the wide kernel
-      if (path != 1) {
+      if (path != 1 && path != 5) {
         h->last_err = "internal: 64-bit request from a 64-bit kernel";
         return MCL_E_CUDA;
       }

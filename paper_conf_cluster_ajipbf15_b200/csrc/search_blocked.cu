@@ -23,179 +23,10 @@
 // The outer digits walk an odometer: digit x (queue Q-4) is the block loop, the digits of
 // queues 0..Q-5 live in shared memory and update the base load vector by one-hot vectors
 // V[q][x] (V[q][x][d] = C[q][x] if d == x else 0) so every register index stays static.
-#include "common.cuh"
-#include "kernels.h"
+#include "blocked_core.cuh"
 
 namespace mcl {
 
-#ifndef MCL_SUPER_MAX_D
-#define MCL_SUPER_MAX_D 5
-#endif
-constexpr int kSuperMaxD = MCL_SUPER_MAX_D;  // super-block path for u32 and D <= this
-
-namespace {
-
-// Adds routed to the FMA pipe (IMAD) so the ALU pipe is left for min/max: `one` is a
-// runtime 1 the compiler cannot fold.
-__device__ __forceinline__ uint32_t add_f(uint32_t a, uint32_t b, uint32_t one) {
-  uint32_t r;
-  asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(one), "r"(b));
-  return r;
-}
-__device__ __forceinline__ uint64_t add_f(uint64_t a, uint64_t b, uint32_t) { return a + b; }
-
-// Integer min/max: VIMNMX (two inputs) and VIMNMX3 (three inputs) for 32-bit lanes.
-__device__ __forceinline__ uint32_t max2(uint32_t a, uint32_t b) { return max(a, b); }
-__device__ __forceinline__ uint32_t max3(uint32_t a, uint32_t b, uint32_t c) { return __vimax3_u32(a, b, c); }
-__device__ __forceinline__ uint32_t min2(uint32_t a, uint32_t b) { return min(a, b); }
-__device__ __forceinline__ uint32_t min3(uint32_t a, uint32_t b, uint32_t c) { return __vimin3_u32(a, b, c); }
-__device__ __forceinline__ uint64_t max2(uint64_t a, uint64_t b) { return a > b ? a : b; }
-__device__ __forceinline__ uint64_t max3(uint64_t a, uint64_t b, uint64_t c) { return max2(a, max2(b, c)); }
-__device__ __forceinline__ uint64_t min2(uint64_t a, uint64_t b) { return a < b ? a : b; }
-__device__ __forceinline__ uint64_t min3(uint64_t a, uint64_t b, uint64_t c) { return min2(a, min2(b, c)); }
-
-// Per-block sums of the prefix loads P with the inner queues' costs (A, B, C = rows
-// Q-3, Q-2, Q-1 of the composed cost table):
-//   a = P+A, b = P+B, c = P+C, ab = P+A+B, ac = P+A+C, bc = P+B+C, abc = P+A+B+C.
-// Shared-memory table `in[7][D]` holds A, B, C, A+B, A+C, B+C, A+B+C.
-template <typename T, int D>
-struct Sums {
-  T a[D], b[D], c[D], ab[D], ac[D], bc[D], abc[D];
-};
-
-template <typename T, int D>
-__device__ __forceinline__ void make_sums(Sums<T, D>& s, const T (&P)[D], const T* __restrict__ in,
-                                          uint32_t one) {
-#pragma unroll
-  for (int d = 0; d < D; ++d) {
-    s.a[d] = add_f(P[d], in[0 * D + d], one);
-    s.b[d] = add_f(P[d], in[1 * D + d], one);
-    s.c[d] = add_f(P[d], in[2 * D + d], one);
-    s.ab[d] = add_f(P[d], in[3 * D + d], one);
-    s.ac[d] = add_f(P[d], in[4 * D + d], one);
-    s.bc[d] = add_f(P[d], in[5 * D + d], one);
-    s.abc[d] = add_f(P[d], in[6 * D + d], one);
-  }
-}
-
-template <typename T, int D>
-__device__ __forceinline__ T max_of(const T (&P)[D]) {
-  T M = P[0];
-#pragma unroll
-  for (int d = 1; d < D; ++d) M = max2(M, P[d]);
-  return M;
-}
-
-// Enumerate the D^3 leaves of one block in increasing index order, calling f(leaf, ms).
-// M = max_d P[d] (prefix makespan).
-template <typename T, int D, typename F>
-__device__ __forceinline__ void for_each_leaf(const Sums<T, D>& s, T M, F&& f) {
-  T PCM[D];
-#pragma unroll
-  for (int d = 0; d < D; ++d) PCM[d] = max2(M, s.c[d]);
-#pragma unroll
-  for (int i = 0; i < D; ++i)
-#pragma unroll
-    for (int j = 0; j < D; ++j)
-#pragma unroll
-      for (int k = 0; k < D; ++k) {
-        T v;
-        if (i != j && i != k && j != k) v = max3(s.a[i], s.b[j], PCM[k]);
-        else if (i == j && j != k) v = max2(s.ab[i], PCM[k]);
-        else if (i == k && i != j) v = max3(s.ac[i], s.b[j], M);
-        else if (j == k && i != j) v = max3(s.a[i], s.bc[j], M);
-        else v = max2(M, s.abc[i]);
-        f((i * D + j) * D + k, v);
-      }
-}
-
-// Minimum makespan over one block, folded two leaves per three-input min.
-template <typename T, int D>
-__device__ __forceinline__ T block_eval(const Sums<T, D>& s, T M) {
-  constexpr T kMax = ~T(0);
-  T acc[4] = {kMax, kMax, kMax, kMax};
-  T pend = kMax;
-  for_each_leaf<T, D>(s, M, [&](int leaf, T v) {
-    if (leaf & 1) {
-      acc[(leaf >> 1) & 3] = min3(acc[(leaf >> 1) & 3], pend, v);
-    } else {
-      pend = v;
-    }
-  });
-  constexpr int kLeaves = D * D * D;
-  T g = min3(acc[0], acc[1], min2(acc[2], acc[3]));
-  if (kLeaves & 1) g = min2(g, pend);
-  return g;
-}
-
-template <typename T, int D>
-__device__ __forceinline__ T block_eval(const T (&P)[D], const T* __restrict__ in, uint32_t one) {
-  Sums<T, D> s;
-  make_sums<T, D>(s, P, in, one);
-  return block_eval<T, D>(s, max_of<T, D>(P));
-}
-
-// Lowest leaf of the block whose makespan equals `target` (the block is known to hold one).
-template <typename T, int D>
-__device__ __forceinline__ uint32_t block_first(const T (&P)[D], const T* __restrict__ in,
-                                                uint32_t one, T target) {
-  Sums<T, D> s;
-  make_sums<T, D>(s, P, in, one);
-  uint32_t first = 0xffffffffu;
-  for_each_leaf<T, D>(s, max_of<T, D>(P), [&](int leaf, T v) {
-    first = (v == target && first == 0xffffffffu) ? (uint32_t)leaf : first;
-  });
-  return first;
-}
-
-// A SUPER-BLOCK: the D blocks x = 0..D-1 of the fourth-innermost digit (queue Q-4) with
-// the same outer prefix `base`. Only device x's load changes between them, so the sums of
-// the other devices are shared and the block loop is unrolled with static x (used for
-// small D, where a D^3 block alone is too short to amortise its setup).
-template <typename T, int D>
-__device__ __forceinline__ void superblock_eval(const T (&base)[D], const T* __restrict__ in,
-                                                const T* __restrict__ c4, uint32_t one, T (&g)[D]) {
-  Sums<T, D> sb;
-  make_sums<T, D>(sb, base, in, one);
-  const T Mb = max_of<T, D>(base);
-#pragma unroll
-  for (int x = 0; x < D; ++x) {
-    const T cx = c4[x];
-    Sums<T, D> s = sb;
-    s.a[x] = add_f(sb.a[x], cx, one);
-    s.b[x] = add_f(sb.b[x], cx, one);
-    s.c[x] = add_f(sb.c[x], cx, one);
-    s.ab[x] = add_f(sb.ab[x], cx, one);
-    s.ac[x] = add_f(sb.ac[x], cx, one);
-    s.bc[x] = add_f(sb.bc[x], cx, one);
-    s.abc[x] = add_f(sb.abc[x], cx, one);
-    const T M = max2(Mb, add_f(base[x], cx, one));
-    g[x] = block_eval<T, D>(s, M);
-  }
-}
-
-template <typename T, int D>
-__device__ __forceinline__ void load_vec(T (&v)[D], const T* __restrict__ src) {
-#pragma unroll
-  for (int d = 0; d < D; ++d) v[d] = src[d];
-}
-
-// Prefix loads P of block `blk` (outer digits of queues 0..O-1), decoded from scratch.
-template <typename T, int D>
-__device__ __forceinline__ void prefix_of(T (&P)[D], uint64_t blk, int O, const T* __restrict__ V,
-                                          uint32_t one) {
-#pragma unroll
-  for (int d = 0; d < D; ++d) P[d] = 0;
-  for (int q = O - 1; q >= 0; --q) {
-    const uint32_t dq = (uint32_t)(blk % D);
-    blk /= D;
-    const T* v = V + ((size_t)q * D + dq) * D;
-#pragma unroll
-    for (int d = 0; d < D; ++d) P[d] = add_f(P[d], v[d], one);
-  }
-}
-
-}  // namespace
 
 // Kernel: gridDim.x = CTAs per epoch (cpe), gridDim.y = epochs handled concurrently.
 template <typename T, int D>
@@ -292,120 +123,8 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
     T best = ~T(0);
     uint64_t best_blk = kNone;
     const uint32_t one = a.one;
-    if (nleft && chunked) {
-      // Super-block path: queue O-1 = digit x (static, inside superblock_eval), queue
-      // O-2 = digit y (uniform loop), queues 0..O-3 = the chunk index, decoded by a loop
-      // whose trip count is the same for every lane (no divergent carries).
-      const T* c4 = in + 7 * D;
-      const T* Vy = V + (size_t)(O - 2) * D * D;
-      uint64_t blk = b0;
-      auto single = [&](uint64_t bk) {
-        T P[D];
-        prefix_of<T, D>(P, bk, O, V, one);
-        const T g = block_eval<T, D>(P, in, one);
-        if (g < best) {
-          best = g;
-          best_blk = bk;
-        }
-      };
-      for (; nleft && (blk % chunk) != 0; ++blk, --nleft) single(blk);
-      for (; nleft >= chunk; nleft -= chunk, blk += chunk) {
-        uint64_t ch = blk / chunk;
-        T base2[D];
-#pragma unroll
-        for (int d = 0; d < D; ++d) base2[d] = 0;
-        for (int q = O - 3; q >= 0; --q) {
-          const uint32_t dq = (uint32_t)(ch % D);
-          ch /= D;
-          const T* v = V + ((size_t)q * D + dq) * D;
-#pragma unroll
-          for (int d = 0; d < D; ++d) base2[d] = add_f(base2[d], v[d], one);
-        }
-        for (int y = 0; y < D; ++y) {
-          T base[D], vy[D];
-          load_vec<T, D>(vy, Vy + y * D);
-#pragma unroll
-          for (int d = 0; d < D; ++d) base[d] = add_f(base2[d], vy[d], one);
-          T g[D];
-          superblock_eval<T, D>(base, in, c4, one, g);
-          T gs = g[0];
-#pragma unroll
-          for (int t = 1; t < D; ++t) gs = min2(gs, g[t]);
-          if (gs < best) {  // rare: locate the first block holding the new minimum
-            best = gs;
-            const uint64_t bb = blk + (uint64_t)y * D;
-#pragma unroll
-            for (int t = D - 1; t >= 0; --t)
-              if (g[t] == gs) best_blk = bb + t;
-          }
-        }
-      }
-      for (; nleft; ++blk, --nleft) single(blk);
-    } else if (nleft) {
-      {
-        // digit x = queue O-1 runs fastest; queues 0..O-2 are the odometer in smem.
-        // Q == 3 (O == 0): a single block whose prefix is the zero vector.
-        const T* Vx = (O >= 1) ? V + (size_t)(O - 1) * D * D : zero;
-        // composed costs of queue O-1 (the x digit), for the super-block path
-        const T* c4 = (O >= 1) ? in + 7 * D : zero;
-        uint32_t x = (uint32_t)(b0 % D);
-        uint64_t hi = b0 / D;
-        T base[D];
-#pragma unroll
-        for (int d = 0; d < D; ++d) base[d] = 0;
-        for (int q = O - 2; q >= 0; --q) {
-          const uint32_t dq = (uint32_t)(hi % D);
-          hi /= D;
-          dig[q * nthr + tid] = (uint8_t)dq;
-          const T* v = V + ((size_t)q * D + dq) * D;
-#pragma unroll
-          for (int d = 0; d < D; ++d) base[d] = add_f(base[d], v[d], one);
-        }
-        uint64_t blk = b0;
-        while (true) {
-          if (kSuper && x == 0 && nleft >= (uint64_t)D) {
-            T g[D];
-            superblock_eval<T, D>(base, in, c4, one, g);
-            T gs = g[0];
-#pragma unroll
-            for (int t = 1; t < D; ++t) gs = min2(gs, g[t]);
-            if (gs < best) {  // rare: locate the first block holding the new minimum
-              best = gs;
-#pragma unroll
-              for (int t = D - 1; t >= 0; --t)
-                if (g[t] == gs) best_blk = blk + t;
-            }
-            x = D;
-            nleft -= D;
-            blk += D;
-          }
-          for (; x < (uint32_t)D && nleft; ++x, --nleft, ++blk) {
-            T P[D], vx[D];
-            load_vec<T, D>(vx, Vx + x * D);
-#pragma unroll
-            for (int d = 0; d < D; ++d) P[d] = add_f(base[d], vx[d], one);
-            const T g = block_eval<T, D>(P, in, one);
-            if (g < best) {
-              best = g;
-              best_blk = blk;
-            }
-          }
-          if (!nleft) break;
-          x = 0;
-          // odometer increment of the outer digits, updating base by one-hot deltas
-          for (int q = O - 2; q >= 0; --q) {
-            const uint32_t old = dig[q * nthr + tid];
-            const uint32_t nw = (old + 1 == (uint32_t)D) ? 0u : old + 1;
-            dig[q * nthr + tid] = (uint8_t)nw;
-            const T* vo = V + ((size_t)q * D + old) * D;
-            const T* vn = V + ((size_t)q * D + nw) * D;
-#pragma unroll
-            for (int d = 0; d < D; ++d) base[d] = base[d] - vo[d] + vn[d];
-            if (nw != 0) break;
-          }
-        }
-      }
-    }
+    const WalkCtx<T, D> wctx{in, V, zero, dig, O, nthr, tid, one};
+    walk_blocks<T, D>(wctx, b0, nleft, best, best_blk);
     // ---- a5: lowest index inside the best block, then warp / CTA / epoch argmin ----
     // Thread ranges ascend with the thread id, so the CTA's lowest-index optimum belongs to
     // the LOWEST thread whose best equals the CTA minimum; only that thread re-scans its

@@ -17,7 +17,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libmcl.so")
 
 MCL_OK, MCL_E_INVAL, MCL_E_RANGE, MCL_E_CUDA, MCL_E_NCCL, MCL_E_NOMEM = 0, -1, -2, -3, -4, -5
-PATH_NAMES = {1: "blocked_u32", 2: "blocked_u64", 3: "generic", 4: "small_batched"}
+PATH_NAMES = {1: "blocked_u32", 2: "blocked_u64", 3: "generic", 4: "small_batched", 5: "flat_u32"}
 
 # Every symbol the headers declare (tests check the library exports all of them).
 EXPORTED = [
@@ -252,7 +252,8 @@ class Mapper:
                 "threads": i[3], "allreduce": bool(i[4]), "index_bits": i[5], "two_step": bool(i[6])}
 
     def force_path(self, path: int) -> None:
-        """Testing aid: 0 auto, 1 blocked u32, 2 blocked u64, 3 generic, 4 small batched."""
+        """Testing aid: 0 auto, 1 blocked u32 (CTA per epoch), 2 blocked u64, 3 generic,
+        4 small batched, 5 flattened batched blocked u32."""
         st = load_library().mcl_force_path(self.handle, path)
         if st != MCL_OK:
             raise MclError(st, "mcl_force_path")

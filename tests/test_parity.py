@@ -88,7 +88,7 @@ def test_random_shapes_all_paths(torch_cuda, mapper, Q, D):
         want = oracle.oracle_map(K, X)
         paths = [0, 3]
         if Q >= 3 and 2 <= D <= 8:
-            paths += [1, 2]
+            paths += [1, 2, 5]
         for p in paths:
             assert_same(run_gpu(torch_cuda, mapper, K, X, p), want, f"Q={Q} D={D} path={p} {maker.__name__}")
 
@@ -122,14 +122,20 @@ def test_cfg1_random_seeds(torch_cuda, mapper):
     Ks, Xs = zip(*(workloads.cfg1_random(s) for s in range(2000)))
     K, X = np.concatenate(Ks), np.concatenate(Xs)
     want = oracle.oracle_map(K, X)
-    for p in (0, 1, 3):
+    for p in (0, 1, 3, 5):
         assert_same(run_gpu(torch_cuda, mapper, K, X, p), want, f"cfg1 x2000 path {p}")
 
 
 def test_cfg2_full(torch_cuda, mapper):
     K, X = workloads.cfg2()
-    assert_same(run_gpu(torch_cuda, mapper, K, X), oracle.oracle_map(K, X), "cfg2")
+    want = oracle.oracle_map(K, X)
+    assert_same(run_gpu(torch_cuda, mapper, K, X), want, "cfg2")
     assert mapper.launch_info()["path"] == "blocked_u32"
+    assert_same(run_gpu(torch_cuda, mapper, K, X, 5), want, "cfg2 flattened")
+    assert_same(run_gpu(torch_cuda, mapper, K, X, 1), want, "cfg2 CTA per epoch")
+    # repeated calls reuse the self-resetting per-epoch keys; a smaller batch after a larger one
+    assert_same(run_gpu(torch_cuda, mapper, K[:37], X[:37]), tuple(w[:37] for w in want), "cfg2[:37]")
+    assert_same(run_gpu(torch_cuda, mapper, K, X), want, "cfg2 again")
 
 
 def test_cfg3_full(torch_cuda, mapper):
@@ -218,7 +224,7 @@ def test_u64_fallback_and_max_entries(torch_cuda, mapper):
     X = np.zeros_like(K)
     X[:, :, 1:] = rng.integers(0, 1 << 20, size=(5, 6, 3), dtype=np.uint64)
     want = oracle.oracle_map(K, X)
-    for p in (0, 1, 3):
+    for p in (0, 1, 3, 5):
         assert_same(run_gpu(torch_cuda, mapper, K, X, p), want, f"u64 path {p}")
     run_gpu(torch_cuda, mapper, K, X, 1)
     assert mapper.launch_info()["path"] == "blocked_u64"
