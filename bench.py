@@ -53,6 +53,8 @@ def parse():
     p.add_argument("--impl", default="mcl", choices=["mcl", "reference"])
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="CPU-oracle sample budget")
+    p.add_argument("--collective", action="store_true",
+                   help="use the NCCL all-reduce path even with one rank (exercises the N>1 code)")
     return p.parse_args()
 
 
@@ -189,7 +191,8 @@ def reference_arm(args, K, X, w, rank, world):
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+        "scaling": "weak" if is_batched(w) else "strong", "vs_baseline": None, "dtype": "u64",
+        "data": "synthetic",
         "config": {"workload": args.workload, "desc": w["desc"], "Q": w["Q"], "D": w["D"], "epochs": w["E"]},
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -214,10 +217,12 @@ def main():
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+    if world > 1 or args.collective:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29531")
+        dist.init_process_group("nccl", device_id=dev, rank=rank, world_size=world)
     comm = None
-    if world > 1 and not is_batched(w):
+    if (world > 1 or args.collective) and not is_batched(w):
         obj = [mcl.mcl_comm_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         comm = mcl.mcl_comm_init(local, world, rank, obj[0])
@@ -349,7 +354,7 @@ def main():
     mapper.close()
     if comm:
         mcl.mcl_comm_destroy(comm)
-    if world > 1:
+    if dist.is_initialized():
         dist.barrier()
         dist.destroy_process_group()
     if rank == 0:
