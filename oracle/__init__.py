@@ -49,6 +49,17 @@ def _load():
         lib.oracle_score.argtypes = [
             ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
         ]
+        lib.oracle_map_constrained.restype = ctypes.c_int
+        lib.oracle_map_constrained.argtypes = [
+            ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p,
+            ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_int,
+            ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+        ]
+        lib.oracle_score_base.restype = ctypes.c_uint64
+        lib.oracle_score_base.argtypes = [
+            ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+            ctypes.c_void_p,
+        ]
         _lib = lib
     return _lib
 
@@ -99,3 +110,42 @@ def oracle_score(K, X, mapping) -> int:
     m = np.ascontiguousarray(mapping, dtype=np.uint8)
     Q, D = K.shape
     return int(_load().oracle_score(Q, D, K.ctypes.data, X.ctypes.data, m.ctypes.data))
+
+
+def oracle_map_constrained(K, X, base=None, elig=None, lo: int = 0, hi: int = 0,
+                           threads: int | None = None):
+    """Constrained brute force (NEXT-3): ``base`` [E, D] pre-existing device loads (or None),
+    ``elig`` [E, Q] uint16 eligible-device masks (bit d = device d, 0 = any; or None).
+    Returns (index[E], makespan[E], mapping[E, Q]); raises OracleError(-1) if an epoch has
+    no feasible mapping."""
+    K = np.ascontiguousarray(K, dtype=np.uint64)
+    X = np.ascontiguousarray(X, dtype=np.uint64)
+    if K.ndim == 2:
+        K, X = K[None], X[None]
+        base = None if base is None else np.asarray(base)[None]
+        elig = None if elig is None else np.asarray(elig)[None]
+    E, Q, D = K.shape
+    b = None if base is None else np.ascontiguousarray(base, dtype=np.uint64).reshape(E, D)
+    m = None if elig is None else np.ascontiguousarray(elig, dtype=np.uint16).reshape(E, Q)
+    idx = np.zeros(E, dtype=np.uint64)
+    ms = np.zeros(E, dtype=np.uint64)
+    mp = np.zeros((E, Q), dtype=np.uint8)
+    rc = _load().oracle_map_constrained(
+        Q, D, E, K.ctypes.data, X.ctypes.data, None if b is None else b.ctypes.data,
+        None if m is None else m.ctypes.data, lo, hi, threads if threads else default_threads(),
+        idx.ctypes.data, ms.ctypes.data, mp.ctypes.data,
+    )
+    if rc != 0:
+        raise OracleError(rc)
+    return idx, ms, mp
+
+
+def oracle_score_base(K, X, base, mapping) -> int:
+    """Makespan of one mapping for one epoch's [Q, D] tables with device base loads [D]."""
+    K = np.ascontiguousarray(K, dtype=np.uint64)
+    X = np.ascontiguousarray(X, dtype=np.uint64)
+    mpg = np.ascontiguousarray(mapping, dtype=np.uint8)
+    Q, D = K.shape
+    b = None if base is None else np.ascontiguousarray(base, dtype=np.uint64)
+    return int(_load().oracle_score_base(Q, D, K.ctypes.data, X.ctypes.data,
+                                         None if b is None else b.ctypes.data, mpg.ctypes.data))

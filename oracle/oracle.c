@@ -47,6 +47,8 @@
 typedef struct {
   uint32_t Q, D;
   const uint64_t *K, *X; /* this epoch's [Q][D] tables */
+  const uint64_t *base;  /* this epoch's [D] pre-existing device loads, or NULL (all 0) */
+  const uint16_t *elig;  /* this epoch's [Q] eligible-device bit masks (0 = any), or NULL */
   uint64_t lo, hi;       /* mapping-index range [lo, hi) */
   uint64_t best_ms, best_m;
   int found;
@@ -68,8 +70,16 @@ static void oracle_scan_range(oracle_range_job *job) {
   job->best_ms = 0;
   job->best_m = 0;
   for (; m < job->hi; ++m) {
-    /* per-device loads from zero: queues on one device serialise (sum) */
-    for (uint32_t d = 0; d < D; ++d) load[d] = 0;
+    /* constrained variant (R11): a mapping that places a queue on a device
+       outside its eligible set is not a candidate (SCHED_OFF queues are "statically
+       mapped to the chosen device") */
+    int feasible = 1;
+    if (job->elig)
+      for (uint32_t q = 0; q < Q; ++q)
+        if (job->elig[q] != 0 && !((job->elig[q] >> digit[q]) & 1u)) feasible = 0;
+    /* per-device loads: the pre-existing load of the device (0 without base loads),
+       then every queue placed there -- queues on one device serialise (sum) */
+    for (uint32_t d = 0; d < D; ++d) load[d] = job->base ? job->base[d] : 0;
     for (uint32_t q = 0; q < Q; ++q) {
       uint32_t d = digit[q];
       load[d] += job->K[q * D + d] + job->X[q * D + d]; /* aggregate cost C = K + X */
@@ -79,7 +89,7 @@ static void oracle_scan_range(oracle_range_job *job) {
     for (uint32_t d = 0; d < D; ++d)
       if (load[d] > ms) ms = load[d];
     /* first strict minimum in increasing index order = lowest index among ties */
-    if (!job->found || ms < job->best_ms) {
+    if (feasible && (!job->found || ms < job->best_ms)) {
       job->found = 1;
       job->best_ms = ms;
       job->best_m = m;
@@ -120,10 +130,18 @@ static int oracle_pow(uint32_t D, uint32_t Q, uint64_t *out) {
  *   makespan_out[epochs] its makespan
  *   mapping_out [epochs][Q] its device tuple, or NULL
  * Returns ORACLE_OK, ORACLE_E_INVAL (Q, D, pointers, range) or ORACLE_E_RANGE.
+ *
+ * oracle_map_constrained additionally takes
+ *   base        [epochs][D] loads already on each device (queues pinned outside the pool:
+ *               SCHED_OFF queues), or NULL for all zero;
+ *   elig        [epochs][Q] bit masks of the devices each queue may use (bit d = device
+ *               d; 0 = any device), or NULL. Mappings outside the masks are not candidates.
+ * An epoch whose range holds no feasible mapping yields ORACLE_E_INVAL.
  */
-int oracle_map(uint32_t Q, uint32_t D, uint64_t epochs, const uint64_t *K, const uint64_t *X,
-               uint64_t lo, uint64_t hi, int threads, uint64_t *index_out, uint64_t *makespan_out,
-               uint8_t *mapping_out) {
+int oracle_map_constrained(uint32_t Q, uint32_t D, uint64_t epochs, const uint64_t *K,
+                           const uint64_t *X, const uint64_t *base, const uint16_t *elig,
+                           uint64_t lo, uint64_t hi, int threads, uint64_t *index_out,
+                           uint64_t *makespan_out, uint8_t *mapping_out) {
   if (Q == 0 || D == 0 || Q > ORACLE_MAX_Q || D > ORACLE_MAX_D) return ORACLE_E_INVAL;
   if (epochs == 0) return ORACLE_OK;
   if (!K || !X || !index_out || !makespan_out) return ORACLE_E_INVAL;
@@ -133,6 +151,9 @@ int oracle_map(uint32_t Q, uint32_t D, uint64_t epochs, const uint64_t *K, const
   if (lo >= hi || hi > N) return ORACLE_E_INVAL;
   for (uint64_t i = 0; i < epochs * Q * D; ++i)
     if (K[i] >= ORACLE_ENTRY_LIMIT || X[i] >= ORACLE_ENTRY_LIMIT) return ORACLE_E_RANGE;
+  if (base)
+    for (uint64_t i = 0; i < epochs * D; ++i)
+      if (base[i] >= ORACLE_ENTRY_LIMIT) return ORACLE_E_RANGE;
   if (threads < 1) threads = 1;
 
   /* work split: whole epochs per thread when there are enough epochs, otherwise every
@@ -149,6 +170,8 @@ int oracle_map(uint32_t Q, uint32_t D, uint64_t epochs, const uint64_t *K, const
       j->D = D;
       j->K = K + e * Q * D;
       j->X = X + e * Q * D;
+      j->base = base ? base + e * D : NULL;
+      j->elig = elig ? elig + e * Q : NULL;
       j->lo = lo + (hi - lo) * p / pieces;
       j->hi = lo + (hi - lo) * (p + 1) / pieces;
     }
@@ -197,9 +220,21 @@ int oracle_map(uint32_t Q, uint32_t D, uint64_t epochs, const uint64_t *K, const
         rest /= D;
       }
     }
+    if (!have) {  /* no feasible mapping in the range */
+      free(jobs);
+      return ORACLE_E_INVAL;
+    }
   }
   free(jobs);
   return ORACLE_OK;
+}
+
+/* The unconstrained mapper: no pre-existing loads, every device eligible. */
+int oracle_map(uint32_t Q, uint32_t D, uint64_t epochs, const uint64_t *K, const uint64_t *X,
+               uint64_t lo, uint64_t hi, int threads, uint64_t *index_out, uint64_t *makespan_out,
+               uint8_t *mapping_out) {
+  return oracle_map_constrained(Q, D, epochs, K, X, NULL, NULL, lo, hi, threads, index_out,
+                                makespan_out, mapping_out);
 }
 
 /* oracle_score: makespan of one given mapping (digit tuple). Used by
@@ -208,6 +243,19 @@ uint64_t oracle_score(uint32_t Q, uint32_t D, const uint64_t *K, const uint64_t 
                       const uint8_t *mapping) {
   uint64_t load[ORACLE_MAX_D];
   for (uint32_t d = 0; d < D; ++d) load[d] = 0;
+  for (uint32_t q = 0; q < Q; ++q) load[mapping[q]] += K[q * D + mapping[q]] + X[q * D + mapping[q]];
+  uint64_t ms = 0;
+  for (uint32_t d = 0; d < D; ++d)
+    if (load[d] > ms) ms = load[d];
+  return ms;
+}
+
+/* oracle_score_base: makespan of one mapping on devices that already carry `base` loads
+   ([D], or NULL for zero) -- the same definition with SCHED_OFF queues' loads included. */
+uint64_t oracle_score_base(uint32_t Q, uint32_t D, const uint64_t *K, const uint64_t *X,
+                           const uint64_t *base, const uint8_t *mapping) {
+  uint64_t load[ORACLE_MAX_D];
+  for (uint32_t d = 0; d < D; ++d) load[d] = base ? base[d] : 0;
   for (uint32_t q = 0; q < Q; ++q) load[mapping[q]] += K[q * D + mapping[q]] + X[q * D + mapping[q]];
   uint64_t ms = 0;
   for (uint32_t d = 0; d < D; ++d)

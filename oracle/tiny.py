@@ -39,3 +39,29 @@ def tiny_map(K, X):
     best = min(itertools.product(range(D), repeat=Q), key=lambda t: score(C, t))
     index = int(np.ravel_multi_index(best, (D,) * Q)) if Q > 0 else 0
     return index, score(C, best), tuple(best)
+
+
+def tiny_map_constrained(K, X, base=None, elig=None):
+    """Constrained definition: devices start at ``base`` loads; queue q may only use the
+    devices in its mask ``elig[q]`` (0 = any). Enumeration is over the eligible tuples in
+    lexicographic order (``itertools.product`` of the per-queue device lists), so ``min``'s
+    first-minimum rule is again the lowest full index."""
+    K = np.asarray(K, dtype=np.uint64)
+    X = np.asarray(X, dtype=np.uint64)
+    Q, D = K.shape
+    C = [[int(K[q, d]) + int(X[q, d]) for d in range(D)] for q in range(Q)]
+    b = [0] * D if base is None else [int(v) for v in base]
+    choices = []
+    for q in range(Q):
+        mask = 0 if elig is None else int(elig[q])
+        choices.append([d for d in range(D) if mask == 0 or (mask >> d) & 1])
+
+    def score_b(t):
+        load = list(b)
+        for q, d in enumerate(t):
+            load[d] += C[q][d]
+        return max(load)
+
+    best = min(itertools.product(*choices), key=score_b)
+    index = int(np.ravel_multi_index(best, (D,) * Q)) if Q > 0 else 0
+    return index, score_b(best), tuple(best)

@@ -27,17 +27,22 @@ def subset_sum_two_identical(w) -> int:
     return S - best
 
 
-def load_vector_dp(C) -> int:
+def load_vector_dp(C, base=None, elig=None) -> int:
     """Optimal makespan for unrelated devices by a DP over queues whose state is the set of
     reachable device-load vectors (the pseudo-polynomial 'dynamic programming' reading of
-    PAPER.md L1048-1052, reading R1). Only for small integer costs."""
+    PAPER.md L1048-1052, reading R1). Only for small integer costs. Optional
+    ``base`` (initial device loads) and ``elig`` (per-queue device masks, 0 = any) give the
+    constrained variant: the DP simply starts from ``base`` and only takes eligible moves."""
     C = [[int(v) for v in row] for row in C]
     D = len(C[0])
-    states = {tuple([0] * D)}
-    for row in C:
+    states = {tuple([0] * D) if base is None else tuple(int(v) for v in base)}
+    for q, row in enumerate(C):
+        mask = 0 if elig is None else int(elig[q])
         nxt = set()
         for s in states:
             for d in range(D):
+                if mask and not (mask >> d) & 1:
+                    continue
                 t = list(s)
                 t[d] += row[d]
                 nxt.add(tuple(t))
