@@ -98,6 +98,45 @@ mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t ep
                             const uint64_t* cost_kernel, const uint64_t* cost_xfer,
                             uint64_t* mapping_index, uint8_t* mapping, uint64_t* makespan);
 
+/*
+ * Constrained variant. The paper's runtime maps only the SCHED_AUTO queues
+ * of the pool; queues created with SCHED_OFF "will be statically mapped to the chosen
+ * device" and still occupy it. Here:
+ *   base_load : [E][D] uint64 or NULL -- load already on each device (e.g. the SCHED_OFF
+ *               queues' cost); every device's load starts from it. Entries < 2^48.
+ *   eligible  : [E][Q] uint16 or NULL -- bit d set = queue q may run on device d; 0 = any
+ *               device. A queue pinned to one device has a single bit.
+ * The result is the lowest index (in the full D^Q index space) among the mappings that
+ * respect every mask and minimise max_d (base_load[d] + sum of C over the queues on d).
+ * Either pointer may be NULL; both NULL is mcl_map_queues. Same buffer rules, sharding and
+ * errors as mcl_map_queues, plus MCL_E_INVAL when some queue has no eligible device < D.
+ * A shard-mode handle (world > 1, no communicator) whose index range holds no feasible
+ * mapping reports index = makespan = UINT64_MAX and mapping bytes 0xFF for that epoch.
+ */
+typedef struct {
+  const uint64_t* base_load; /* [E][D] or NULL */
+  const uint16_t* eligible;  /* [E][Q] or NULL */
+} mcl_constraints_t;
+
+mcl_status_t mcl_map_queues_constrained(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                                        const uint64_t* cost_kernel, const uint64_t* cost_xfer,
+                                        const mcl_constraints_t* constraints,
+                                        uint64_t* mapping_index, uint8_t* mapping,
+                                        uint64_t* makespan);
+
+/*
+ * Score GIVEN mappings: makespan[e] = max_d (base_load[e][d] + sum over queues q with
+ * mappings[e][q] == d of (cost_kernel + cost_xfer)[e][q][d]) -- e.g. a ROUND_ROBIN mapping
+ * ("the next available device when the scheduler is triggered") or a
+ * static hint-based choice (SS V.B), to compare a policy against the optimum.
+ *   mappings : [E][Q] uint8 device ids (< D, else MCL_E_INVAL); base_load may be NULL.
+ * Host or device pointers; synchronous; errors as mcl_map_queues.
+ */
+mcl_status_t mcl_score_mappings(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                                const uint64_t* cost_kernel, const uint64_t* cost_xfer,
+                                const uint64_t* base_load, const uint8_t* mappings,
+                                uint64_t* makespan);
+
 /* Destroy a handle (NULL-safe). Frees the handle's scratch; never the caller's buffers and
    never the NCCL communicator (its owner, e.g. the torch process group, keeps it). */
 void mcl_mapper_destroy(mcl_mapper_t* h);

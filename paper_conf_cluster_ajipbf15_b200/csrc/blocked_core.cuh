@@ -181,12 +181,13 @@ __device__ __forceinline__ void load_vec(T (&v)[D], const T* __restrict__ src) {
   for (int d = 0; d < D; ++d) v[d] = src[d];
 }
 
-// Prefix loads P of block `blk` (outer digits of queues 0..O-1), decoded from scratch.
+// Prefix loads P of block `blk` (outer digits of queues 0..O-1), decoded from scratch,
+// on top of the devices' base loads B0 (zero unless the call is constrained).
 template <typename T, int D>
 __device__ __forceinline__ void prefix_of(T (&P)[D], uint64_t blk, int O, const T* __restrict__ V,
-                                          uint32_t one) {
+                                          const T* __restrict__ B0, uint32_t one) {
 #pragma unroll
-  for (int d = 0; d < D; ++d) P[d] = 0;
+  for (int d = 0; d < D; ++d) P[d] = B0[d];
   for (int q = O - 1; q >= 0; --q) {
     const uint32_t dq = (uint32_t)(blk % D);
     blk /= D;
@@ -200,12 +201,14 @@ __device__ __forceinline__ void prefix_of(T (&P)[D], uint64_t blk, int O, const 
 // Score the blocks [b0, b0 + nleft) of one epoch for one thread, keeping the first strict
 // minimum: best = its block minimum, best_blk = the block holding it (kNone if none).
 // Tables (shared memory): in[8][D] (inner sums + the costs of queue O-1), V[O][D][D]
-// one-hot outer vectors, zero[D], dig[(O-1)][nthr] odometer digits of this thread.
+// one-hot outer vectors, zero[D], base0[D] device base loads (zero when unconstrained),
+// dig[(O-1)][nthr] odometer digits of this thread.
 template <typename T, int D>
 struct WalkCtx {
   const T* in;
   const T* V;
   const T* zero;
+  const T* base0;
   uint8_t* dig;
   int O;     // outer queues (Q - 3)
   int nthr;  // stride of the digit table
@@ -222,10 +225,11 @@ __device__ __forceinline__ void walk_blocks(const WalkCtx<T, D>& w, uint64_t b0,
   const T* in = w.in;
   const T* V = w.V;
   const T* zero = w.zero;
+  const T* B0 = w.base0;
   uint8_t* dig = w.dig;
   const bool chunked = kSuper && O >= 2;
   const uint64_t chunk = chunked ? (uint64_t)D * D : 1;
-if (nleft && chunked) {
+  if (nleft && chunked) {
     // Super-block path: queue O-1 = digit x (static, inside superblock_eval), queue
     // O-2 = digit y (uniform loop), queues 0..O-3 = the chunk index, decoded by a loop
     // whose trip count is the same for every lane (no divergent carries).
@@ -234,7 +238,7 @@ if (nleft && chunked) {
     uint64_t blk = b0;
     auto single = [&](uint64_t bk) {
       T P[D];
-      prefix_of<T, D>(P, bk, O, V, one);
+      prefix_of<T, D>(P, bk, O, V, B0, one);
       const T g = block_eval<T, D>(P, in, one);
       if (g < best) {
         best = g;
@@ -246,7 +250,7 @@ if (nleft && chunked) {
       uint64_t ch = blk / chunk;
       T base2[D];
 #pragma unroll
-      for (int d = 0; d < D; ++d) base2[d] = 0;
+      for (int d = 0; d < D; ++d) base2[d] = B0[d];
       for (int q = O - 3; q >= 0; --q) {
         const uint32_t dq = (uint32_t)(ch % D);
         ch /= D;
@@ -285,7 +289,7 @@ if (nleft && chunked) {
       uint64_t hi = b0 / D;
       T base[D];
 #pragma unroll
-      for (int d = 0; d < D; ++d) base[d] = 0;
+      for (int d = 0; d < D; ++d) base[d] = B0[d];
       for (int q = O - 2; q >= 0; --q) {
         const uint32_t dq = (uint32_t)(hi % D);
         hi /= D;

@@ -60,6 +60,8 @@ struct BlockedArgs {
   volatile uint32_t* flags;
   uint32_t one;
   size_t off_red, off_dig;
+  const uint64_t* base;  // [E][D] pre-existing device loads, or nullptr (constrained variant)
+  const uint16_t* elig;  // [E][Q] eligible-device masks (0 = any), or nullptr
 };
 
 // ceil(log2(N)): bits of the packed key's index field (N >= 1).
@@ -107,8 +109,16 @@ struct GenericArgs {
   EpochOut out;
   int ibits;
   volatile uint32_t* flags;
+  const uint64_t* base;  // [E][D] or nullptr (constrained variant)
+  const uint16_t* elig;  // [E][Q] or nullptr
 };
 size_t generic_smem_bytes(uint32_t Q, uint32_t D, int threads);
+
+// Scoring of given mappings (score.cu): makespan[e] of mapping[e][.] with optional base
+// loads; a device id >= D raises kFlagBadMapping.
+cudaError_t launch_score(uint32_t Q, uint32_t D, uint64_t E, const uint64_t* K, const uint64_t* X,
+                         const uint64_t* base, const uint8_t* mapping, uint64_t* makespan,
+                         volatile uint32_t* flags, cudaStream_t st);
 cudaError_t launch_generic(const GenericArgs& a, dim3 grid, int threads, size_t smem,
                            cudaStream_t st);
 

@@ -122,7 +122,7 @@ struct mcl_mapper {
   DevBuf done;             // uint32 per epoch, zero between calls
   DevBuf key, pair, gms, cand;
   DevBuf flat_keys, flat_done;  // flattened batched kernel: per-epoch key / block count
-  DevBuf in_k, in_x, out_idx, out_ms, out_map;  // staging for host pointers
+  DevBuf in_k, in_x, in_base, in_elig, out_idx, out_ms, out_map;  // staging for host pointers
   uint32_t* flags_host = nullptr;               // host-mapped status word
   uint32_t* flags_dev = nullptr;
   int timing = 0;               // 0 off, 1 search kernel, 2 search kernel + whole call
@@ -310,7 +310,7 @@ void mcl_mapper_destroy(mcl_mapper_t* h) {
     DeviceGuard g(h->device);
     if (h->stream) cudaStreamSynchronize(h->stream);
     for (DevBuf* b : {&h->scratch, &h->done, &h->key, &h->pair, &h->gms, &h->cand, &h->flat_keys,
-                      &h->flat_done, &h->in_k,
+                      &h->flat_done, &h->in_k, &h->in_base, &h->in_elig,
                       &h->in_x, &h->out_idx, &h->out_ms, &h->out_map})
       b->release();
     if (h->flags_host) cudaFreeHost(h->flags_host);
@@ -355,9 +355,27 @@ mcl_status_t mcl_last_kernel_time(const mcl_mapper_t* h, float* kernel_ms, float
   return MCL_OK;
 }
 
-mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
-                            const uint64_t* cost_kernel, const uint64_t* cost_xfer,
-                            uint64_t* mapping_index, uint8_t* mapping, uint64_t* makespan) {
+}  // extern "C"
+
+namespace {
+
+// Stage a host buffer of `bytes` into `buf` (device pointers are used in place).
+mcl_status_t stage_in(mcl_mapper* h, DevBuf& buf, const void* src, size_t bytes, bool on_device,
+                      const void** out) {
+  if (on_device) {
+    *out = src;
+    return MCL_OK;
+  }
+  MCL_CUDA(h, buf.ensure(bytes), "cudaMalloc(staging)");
+  MCL_CUDA(h, cudaMemcpyAsync(buf.p, src, bytes, cudaMemcpyHostToDevice, h->stream), "H2D");
+  *out = buf.p;
+  return MCL_OK;
+}
+
+mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                      const uint64_t* cost_kernel, const uint64_t* cost_xfer,
+                      const uint64_t* base_load, const uint16_t* eligible,
+                      uint64_t* mapping_index, uint8_t* mapping, uint64_t* makespan) {
   if (!h) return MCL_E_INVAL;
   h->last_err.clear();
   if (Q == 0 || D == 0 || Q > MCL_MAX_QUEUES || D > MCL_MAX_DEVICES) {
@@ -421,6 +439,24 @@ mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t ep
     MCL_CUDA(h, h->out_map.ensure(epochs * Q), "cudaMalloc(staging)");
     o_map = (uint8_t*)h->out_map.p;
   }
+  // constrained variant: base loads [E][D] and eligible masks [E][Q] (either may be NULL)
+  const bool constrained = base_load || eligible;
+  const uint64_t* Bd = nullptr;
+  const uint16_t* Ed = nullptr;
+  if (base_load) {
+    bool on;
+    if ((st = classify(h, base_load, &on)) != MCL_OK) return st;
+    const void* p = nullptr;
+    if ((st = stage_in(h, h->in_base, base_load, epochs * D * 8, on, &p)) != MCL_OK) return st;
+    Bd = (const uint64_t*)p;
+  }
+  if (eligible) {
+    bool on;
+    if ((st = classify(h, eligible, &on)) != MCL_OK) return st;
+    const void* p = nullptr;
+    if ((st = stage_in(h, h->in_elig, eligible, epochs * Q * 2, on, &p)) != MCL_OK) return st;
+    Ed = (const uint16_t*)p;
+  }
 
   const int ibits = mcl::index_bits_host(N);
   mcl::EpochOut out{o_idx, o_ms, o_map, nullptr, nullptr};
@@ -434,16 +470,17 @@ mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t ep
 
   // ---- choose the kernel ----
   const bool shard_mode = h->world > 1;  // NCCL collective or single-GPU shard test
+  // the small and flattened kernels take no constraints; the blocked and generic ones do
   int path;
-  if (!shard_mode && !multi && mcl::small_supported(Q, D)) path = 4;
+  if (!shard_mode && !multi && !constrained && mcl::small_supported(Q, D)) path = 4;
   else if (mcl::blocked_supported(Q, D)) path = 1;
   else path = 3;
   if (h->force_path) {
     const int f = h->force_path;
     const bool ok = (f == 3) || ((f == 1 || f == 2) && mcl::blocked_supported(Q, D)) ||
-                    (f == 5 && epochs > 1 && !shard_mode && !multi &&
+                    (f == 5 && epochs > 1 && !shard_mode && !multi && !constrained &&
                      mcl::flat_supported(Q, D, mcl::index_bits_host(N))) ||
-                    (f == 4 && !shard_mode && !multi && mcl::small_supported(Q, D));
+                    (f == 4 && !shard_mode && !multi && !constrained && mcl::small_supported(Q, D));
     if (!ok) {
       h->last_err = "forced kernel path does not support this shape / sharding";
       return MCL_E_INVAL;
@@ -501,6 +538,7 @@ mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t ep
       mcl::BlockedArgs a{};
       a.Q = Q; a.D = D; a.E = epochs; a.K = K; a.X = X; a.rlo = lo; a.rhi = hi;
       a.out = out; a.ibits = ibits; a.flags = h->flags_dev; a.one = 1;
+      a.base = Bd; a.elig = Ed;
       const size_t smem = mcl::blocked_smem_bytes(Q, D, wide, threads, &a.off_red, &a.off_dig);
       int occ = mcl::blocked_ctas_per_sm(D, wide, threads, smem);
       size_grid(h, epochs, hi - lo, occ, threads, &grid);
@@ -521,6 +559,7 @@ mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t ep
       mcl::GenericArgs a{};
       a.Q = Q; a.D = D; a.E = epochs; a.K = K; a.X = X; a.rlo = lo; a.rhi = hi;
       a.out = out; a.ibits = ibits; a.flags = h->flags_dev;
+      a.base = Bd; a.elig = Ed;
       const size_t smem = mcl::generic_smem_bytes(Q, D, threads);
       size_grid(h, epochs, hi - lo, 8, threads, &grid);
       if (grid.x > 1) {
@@ -549,8 +588,12 @@ mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t ep
     MCL_CUDA(h, cudaStreamSynchronize(s), "search kernel");
     const uint32_t flags = *(volatile uint32_t*)h->flags_host;
     if (flags & 1u) {
-      h->last_err = "a cost entry is >= 2^48";
+      h->last_err = "a cost entry or base load is >= 2^48";
       return MCL_E_RANGE;
+    }
+    if (flags & 8u) {
+      h->last_err = "a queue has no eligible device below D";
+      return MCL_E_INVAL;
     }
     if (flags & 2u) {  // some epoch's bound needs 64-bit loads: rerun the wide kernel
       if (path != 1 && path != 5) {
@@ -592,6 +635,88 @@ mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t ep
   h->timing_pending = h->timing > 0;  // elapsed times are read lazily (mcl_last_kernel_time)
   return MCL_OK;
 }
+
+}  // namespace
+
+extern "C" {
+
+mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                            const uint64_t* cost_kernel, const uint64_t* cost_xfer,
+                            uint64_t* mapping_index, uint8_t* mapping, uint64_t* makespan) {
+  return map_impl(h, Q, D, epochs, cost_kernel, cost_xfer, nullptr, nullptr, mapping_index,
+                  mapping, makespan);
+}
+
+mcl_status_t mcl_map_queues_constrained(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                                        const uint64_t* cost_kernel, const uint64_t* cost_xfer,
+                                        const mcl_constraints_t* constraints,
+                                        uint64_t* mapping_index, uint8_t* mapping,
+                                        uint64_t* makespan) {
+  return map_impl(h, Q, D, epochs, cost_kernel, cost_xfer,
+                  constraints ? constraints->base_load : nullptr,
+                  constraints ? constraints->eligible : nullptr, mapping_index, mapping, makespan);
+}
+
+mcl_status_t mcl_score_mappings(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                                const uint64_t* cost_kernel, const uint64_t* cost_xfer,
+                                const uint64_t* base_load, const uint8_t* mappings,
+                                uint64_t* makespan) {
+  if (!h) return MCL_E_INVAL;
+  h->last_err.clear();
+  if (Q == 0 || D == 0 || Q > MCL_MAX_QUEUES || D > MCL_MAX_DEVICES) {
+    h->last_err = "Q must be in [1, 32] and D in [1, 16]";
+    return MCL_E_INVAL;
+  }
+  if (epochs == 0) return MCL_OK;
+  if (!cost_kernel || !cost_xfer || !mappings || !makespan) {
+    h->last_err = "NULL required pointer";
+    return MCL_E_INVAL;
+  }
+  if (epochs > (1ull << 40) / ((uint64_t)Q * D)) {
+    h->last_err = "epochs too large";
+    return MCL_E_INVAL;
+  }
+  DeviceGuard g(h->device);
+  mcl_status_t st;
+  bool dk, dx, db = true, dmp, dm;
+  if ((st = classify(h, cost_kernel, &dk)) != MCL_OK) return st;
+  if ((st = classify(h, cost_xfer, &dx)) != MCL_OK) return st;
+  if (base_load && (st = classify(h, base_load, &db)) != MCL_OK) return st;
+  if ((st = classify(h, mappings, &dmp)) != MCL_OK) return st;
+  if ((st = classify(h, makespan, &dm)) != MCL_OK) return st;
+  const void *K, *X, *B = nullptr, *M;
+  const size_t in_bytes = (size_t)epochs * Q * D * 8;
+  if ((st = stage_in(h, h->in_k, cost_kernel, in_bytes, dk, &K)) != MCL_OK) return st;
+  if ((st = stage_in(h, h->in_x, cost_xfer, in_bytes, dx, &X)) != MCL_OK) return st;
+  if (base_load && (st = stage_in(h, h->in_base, base_load, epochs * D * 8, db, &B)) != MCL_OK)
+    return st;
+  if ((st = stage_in(h, h->in_elig, mappings, epochs * Q, dmp, &M)) != MCL_OK) return st;
+  uint64_t* o_ms = makespan;
+  if (!dm) {
+    MCL_CUDA(h, h->out_ms.ensure(epochs * 8), "cudaMalloc(staging)");
+    o_ms = (uint64_t*)h->out_ms.p;
+  }
+  *(volatile uint32_t*)h->flags_host = 0;
+  MCL_CUDA(h, mcl::launch_score(Q, D, epochs, (const uint64_t*)K, (const uint64_t*)X,
+                                (const uint64_t*)B, (const uint8_t*)M, o_ms, h->flags_dev, h->stream),
+           "score launch");
+  if (!dm) MCL_CUDA(h, cudaMemcpyAsync(makespan, o_ms, epochs * 8, cudaMemcpyDeviceToHost, h->stream), "D2H");
+  MCL_CUDA(h, cudaStreamSynchronize(h->stream), "score kernel");
+  const uint32_t flags = *(volatile uint32_t*)h->flags_host;
+  if (flags & 16u) {
+    h->last_err = "a mapping names a device >= D";
+    return MCL_E_INVAL;
+  }
+  if (flags & 1u) {
+    h->last_err = "a cost entry or base load is >= 2^48";
+    return MCL_E_RANGE;
+  }
+  return MCL_OK;
+}
+
+}  // extern "C"
+
+extern "C" {
 
 mcl_status_t mcl_probe_int_rate(int device, int op, double* lane_ops_per_s,
                                 double* lane_ops_per_clk_sm, double* eff_mhz) {

@@ -46,39 +46,37 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
   uint8_t* dig = reinterpret_cast<uint8_t*>(smem_raw) + a.off_dig;
   __shared__ __align__(16) T zero[D];
   if (threadIdx.x < D) zero[threadIdx.x] = 0;
-  __shared__ int s_bad;
+  __shared__ uint32_t s_status;
   __shared__ uint64_t s_ub;
+  __shared__ uint64_t s_feas;  // feasible bound of a constrained epoch (else kNone)
+  __shared__ uint64_t s_base[D];
+  __shared__ __align__(16) T base0[D];  // base loads in the search's arithmetic type
   constexpr bool kSuper = (sizeof(T) == 4 && D <= kSuperMaxD);
 
   for (uint64_t e = blockIdx.y; e < a.E; e += gridDim.y) {
     // ---- a1: cost composition C = K + X, range check, bound UB = sum_q max_d C ----
     __syncthreads();  // the previous epoch's tables are no longer read
-    if (tid == 0) { s_bad = 0; s_ub = 0; }
+    if (tid == 0) { s_status = 0; s_ub = 0; }
     __syncthreads();
     const uint64_t* Ke = a.K + e * Q * D;
     const uint64_t* Xe = a.X + e * Q * D;
     for (uint32_t t = tid; t < Q * D; t += nthr) {
       const uint64_t k = Ke[t], x = Xe[t];
-      if (k >= kEntryLimit || x >= kEntryLimit) s_bad = 1;
+      if (k >= kEntryLimit || x >= kEntryLimit) s_status = kFlagRange;
       C64[t] = k + x;
     }
     __syncthreads();
-    if (s_bad) {
-      if (tid == 0 && blockIdx.x == 0) raise_flag(a.flags, kFlagRange);
-      continue;
-    }
-    if (tid < 32) {  // one warp: per-queue row max, then the sum over queues
-      uint64_t part = 0;
-      for (uint32_t q = tid; q < Q; q += 32) {
-        uint64_t m = 0;
-        for (int d = 0; d < D; ++d) m = max2(m, C64[q * D + d]);
-        part += m;
-      }
-#pragma unroll
-      for (int off = 16; off > 0; off >>= 1) part += __shfl_xor_sync(0xffffffffu, part, off);
-      if (tid == 0) s_ub = part;
+    if (tid < 32) {  // one warp: base loads, eligibility masking, the bound UB
+      const uint64_t ub = epoch_prologue(C64, Q, D, a.base ? a.base + e * D : nullptr,
+                                         a.elig ? a.elig + e * Q : nullptr, s_base, &s_status,
+                                         &s_feas);
+      if (tid == 0) s_ub = ub;
     }
     __syncthreads();
+    if (s_status) {
+      if (tid == 0 && blockIdx.x == 0) raise_flag(a.flags, s_status);
+      continue;
+    }
     if (sizeof(T) == 4 && s_ub >= (1ull << 32)) {
       if (tid == 0 && blockIdx.x == 0) raise_flag(a.flags, kFlagNeedU64);
       continue;
@@ -95,6 +93,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
       in[6 * D + t] = (T)(A + B + Cc);
     }
     for (int t = tid; t < D; t += nthr) in[7 * D + t] = (O >= 1) ? (T)C64[(O - 1) * D + t] : (T)0;
+    for (int t = tid; t < D; t += nthr) base0[t] = (T)s_base[t];
     for (int t = tid; t < O * D * D; t += nthr) {
       const int q = t / (D * D), x = (t / D) % D, d = t % D;
       V[t] = (d == x) ? (T)C64[q * D + x] : (T)0;
@@ -123,7 +122,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
     T best = ~T(0);
     uint64_t best_blk = kNone;
     const uint32_t one = a.one;
-    const WalkCtx<T, D> wctx{in, V, zero, dig, O, nthr, tid, one};
+    const WalkCtx<T, D> wctx{in, V, zero, base0, dig, O, nthr, tid, one};
     walk_blocks<T, D>(wctx, b0, nleft, best, best_blk);
     // ---- a5: lowest index inside the best block, then warp / CTA / epoch argmin ----
     // Thread ranges ascend with the thread id, so the CTA's lowest-index optimum belongs to
@@ -152,7 +151,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
       __syncthreads();
       if ((uint32_t)tid == s_winner) {
         T P[D];
-        prefix_of<T, D>(P, best_blk, O, V, one);
+        prefix_of<T, D>(P, best_blk, O, V, base0, one);
         const uint32_t leaf = block_first<T, D>(P, in, one, best);
         s_cand = Cand{(uint64_t)best, best_blk * (uint64_t)(D * D * D) + leaf};
       }
@@ -160,7 +159,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
     }
     Cand c = s_cand;
     if (gridDim.x == 1) {
-      if (tid == 0) write_epoch(a.out, e, Q, D, a.ibits, c, a.flags);
+      if (tid == 0) write_epoch(a.out, e, Q, D, a.ibits, c, a.flags, s_feas);
       continue;
     }
     __shared__ bool s_last;
@@ -181,7 +180,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
       }
       r = block_min(r, red);
       if (tid == 0) {
-        write_epoch(a.out, e, Q, D, a.ibits, r, a.flags);
+        write_epoch(a.out, e, Q, D, a.ibits, r, a.flags, s_feas);
         a.done[e] = 0;  // self-reset for the next call
       }
     }

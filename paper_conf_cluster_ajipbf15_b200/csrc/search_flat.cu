@@ -43,7 +43,7 @@ __global__ void __launch_bounds__(32, (D <= 5) ? 16 : 8) search_flat_kernel(Flat
   };
   uint64_t f = split(w);
   const uint64_t fend = split(w + 1);
-  const WalkCtx<T, D> wctx{in, V, zero, dig, O, 32, lane, a.one};
+  const WalkCtx<T, D> wctx{in, V, zero, zero, dig, O, 32, lane, a.one};  // no base loads
 
   while (f < fend) {
     const uint64_t e = f / nb;
@@ -112,7 +112,7 @@ __global__ void __launch_bounds__(32, (D <= 5) ? 16 : 8) search_flat_kernel(Flat
     const uint32_t holders = __ballot_sync(0xffffffffu, bv != kNone && bv == wmin);
     if (holders && lane == __ffs(holders) - 1) {
       T P[D];
-      prefix_of<T, D>(P, best_blk, O, V, a.one);
+      prefix_of<T, D>(P, best_blk, O, V, zero, a.one);
       const uint32_t leaf = block_first<T, D>(P, in, a.one, best);
       const uint64_t idx = best_blk * (uint64_t)(D * D * D) + leaf;
       atomicMin((unsigned long long*)&a.keys[e], (unsigned long long)((bv << a.ibits) | idx));

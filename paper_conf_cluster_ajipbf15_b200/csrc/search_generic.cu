@@ -22,23 +22,29 @@ __global__ void __launch_bounds__(256) search_generic_kernel(GenericArgs a) {
   uint64_t* L = C64 + Q * D;
   Cand* red = reinterpret_cast<Cand*>(L + (size_t)D * nthr);
   uint8_t* dig = reinterpret_cast<uint8_t*>(red + 32);
-  __shared__ int s_bad;
+  __shared__ uint32_t s_status;
   __shared__ bool s_last;
+  __shared__ uint64_t s_base[kMaxDevices];
+  __shared__ uint64_t s_feas;
 
   for (uint64_t e = blockIdx.y; e < a.E; e += gridDim.y) {
     __syncthreads();
-    if (tid == 0) s_bad = 0;
+    if (tid == 0) s_status = 0;
     __syncthreads();
     const uint64_t* Ke = a.K + e * Q * D;
     const uint64_t* Xe = a.X + e * Q * D;
     for (uint32_t t = tid; t < Q * D; t += nthr) {
       const uint64_t k = Ke[t], x = Xe[t];
-      if (k >= kEntryLimit || x >= kEntryLimit) s_bad = 1;
+      if (k >= kEntryLimit || x >= kEntryLimit) s_status = kFlagRange;
       C64[t] = k + x;  // a1: aggregate cost
     }
     __syncthreads();
-    if (s_bad) {
-      if (tid == 0 && blockIdx.x == 0) raise_flag(a.flags, kFlagRange);
+    if (tid < 32)  // base loads and eligibility masking (constrained variant); 64-bit loads
+      epoch_prologue(C64, Q, D, a.base ? a.base + e * D : nullptr, a.elig ? a.elig + e * Q : nullptr,
+                     s_base, &s_status, &s_feas);
+    __syncthreads();
+    if (s_status) {
+      if (tid == 0 && blockIdx.x == 0) raise_flag(a.flags, s_status);
       continue;
     }
     const uint64_t nr = a.rhi - a.rlo;
@@ -51,7 +57,7 @@ __global__ void __launch_bounds__(256) search_generic_kernel(GenericArgs a) {
 
     Cand best{kNone, kNone};
     if (nleft) {
-      for (uint32_t d = 0; d < D; ++d) L[d * nthr + tid] = 0;
+      for (uint32_t d = 0; d < D; ++d) L[d * nthr + tid] = s_base[d];
       uint64_t r = row;
       for (int q = (int)Q - 2; q >= 0; --q) {  // decode the first row's digits
         const uint32_t dq = (uint32_t)(r % D);
@@ -83,7 +89,7 @@ __global__ void __launch_bounds__(256) search_generic_kernel(GenericArgs a) {
     }
     Cand c = block_min(best, red);
     if (gridDim.x == 1) {
-      if (tid == 0) write_epoch(a.out, e, Q, D, a.ibits, c, a.flags);
+      if (tid == 0) write_epoch(a.out, e, Q, D, a.ibits, c, a.flags, s_feas);
       continue;
     }
     if (tid == 0) {
@@ -102,7 +108,7 @@ __global__ void __launch_bounds__(256) search_generic_kernel(GenericArgs a) {
       }
       r = block_min(r, red);
       if (tid == 0) {
-        write_epoch(a.out, e, Q, D, a.ibits, r, a.flags);
+        write_epoch(a.out, e, Q, D, a.ibits, r, a.flags, s_feas);
         a.done[e] = 0;
       }
     }

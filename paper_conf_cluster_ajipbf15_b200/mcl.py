@@ -26,7 +26,12 @@ EXPORTED = [
     "mcl_set_timing", "mcl_last_kernel_time", "mcl_force_path", "mcl_probe_int_rate",
     "mcl_device_sms",
     "mcl_comm_unique_id", "mcl_comm_init", "mcl_comm_destroy",
+    "mcl_map_queues_constrained", "mcl_score_mappings",
 ]
+
+
+class mcl_constraints_t(ctypes.Structure):
+    _fields_ = [("base_load", ctypes.c_void_p), ("eligible", ctypes.c_void_p)]
 
 
 class mcl_config_t(ctypes.Structure):
@@ -81,6 +86,9 @@ def load_library(path: str | None = None) -> ctypes.CDLL:
         "mcl_comm_unique_id": (i32, [ctypes.c_char_p]),
         "mcl_comm_init": (i32, [i32, i32, i32, ctypes.c_char_p, ctypes.POINTER(vp)]),
         "mcl_comm_destroy": (i32, [vp]),
+        "mcl_map_queues_constrained": (i32, [vp, u32, u32, u64, vp, vp,
+                                             ctypes.POINTER(mcl_constraints_t), vp, vp, vp]),
+        "mcl_score_mappings": (i32, [vp, u32, u32, u64, vp, vp, vp, vp, vp]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -174,7 +182,7 @@ def _ptr_and_keepalive(x, dtype):
     except ImportError:  # pragma: no cover
         torch = None
     if torch is not None and isinstance(x, torch.Tensor):
-        want = {np.uint64: torch.uint64, np.uint8: torch.uint8}[dtype]
+        want = {np.uint64: torch.uint64, np.uint8: torch.uint8, np.uint16: torch.uint16}[dtype]
         if x.dtype != want or not x.is_contiguous():
             raise TypeError(f"expected a contiguous {want} tensor")
         return x.data_ptr(), x
@@ -244,6 +252,63 @@ class Mapper:
             ms = np.empty(E, dtype=np.uint64)
             mp = np.empty((E, Q), dtype=np.uint8) if with_mapping else None
         self.map_queues_into(K, X, idx, mp, ms)
+        return idx, mp, ms
+
+    def map_queues_constrained(self, K, X, base=None, eligible=None, with_mapping: bool = True):
+        """Constrained search (include/mcl.h mcl_map_queues_constrained): ``base`` [E, D]
+        uint64 device base loads or None, ``eligible`` [E, Q] uint16 device masks (0 = any)
+        or None. Outputs are allocated like K; returns (index, mapping or None, makespan)."""
+        if K.ndim == 2:
+            K, X = K[None], X[None]
+            base = None if base is None else base[None]
+            eligible = None if eligible is None else eligible[None]
+        E, Q, D = (int(s) for s in K.shape)
+        idx, mp, ms = self._alloc_outputs(K, E, Q, with_mapping)
+        pk, _k = _ptr_and_keepalive(K, np.uint64)
+        px, _x = _ptr_and_keepalive(X, np.uint64)
+        pb, _b = _ptr_and_keepalive(base, np.uint64) if base is not None else (None, None)
+        pe, _e = _ptr_and_keepalive(eligible, np.uint16) if eligible is not None else (None, None)
+        pi, _i = _ptr_and_keepalive(idx, np.uint64)
+        pm, _m = _ptr_and_keepalive(ms, np.uint64)
+        pmap = _ptr_and_keepalive(mp, np.uint8)[0] if mp is not None else None
+        c = mcl_constraints_t(pb, pe)
+        st = load_library().mcl_map_queues_constrained(self.handle, Q, D, E, pk, px, ctypes.byref(c),
+                                                       pi, pmap, pm)
+        if st != MCL_OK:
+            raise MclError(st, "mcl_map_queues_constrained", mcl_last_error_string(self.handle))
+        return idx, mp, ms
+
+    def score_mappings(self, K, X, mappings, base=None):
+        """Makespan of given mappings [E, Q] (uint8 device ids), optional base loads [E, D]."""
+        if K.ndim == 2:
+            K, X, mappings = K[None], X[None], mappings[None]
+            base = None if base is None else base[None]
+        E, Q, D = (int(s) for s in K.shape)
+        ms = self._alloc_outputs(K, E, Q, False)[2]
+        pk, _k = _ptr_and_keepalive(K, np.uint64)
+        px, _x = _ptr_and_keepalive(X, np.uint64)
+        pb, _b = _ptr_and_keepalive(base, np.uint64) if base is not None else (None, None)
+        pmp, _mp = _ptr_and_keepalive(mappings, np.uint8)
+        pm, _m = _ptr_and_keepalive(ms, np.uint64)
+        st = load_library().mcl_score_mappings(self.handle, Q, D, E, pk, px, pb, pmp, pm)
+        if st != MCL_OK:
+            raise MclError(st, "mcl_score_mappings", mcl_last_error_string(self.handle))
+        return ms
+
+    @staticmethod
+    def _alloc_outputs(K, E, Q, with_mapping):
+        try:
+            import torch
+        except ImportError:  # pragma: no cover
+            torch = None
+        if torch is not None and isinstance(K, torch.Tensor):
+            idx = torch.empty(E, dtype=torch.uint64, device=K.device)
+            ms = torch.empty(E, dtype=torch.uint64, device=K.device)
+            mp = torch.empty((E, Q), dtype=torch.uint8, device=K.device) if with_mapping else None
+        else:
+            idx = np.empty(E, dtype=np.uint64)
+            ms = np.empty(E, dtype=np.uint64)
+            mp = np.empty((E, Q), dtype=np.uint8) if with_mapping else None
         return idx, mp, ms
 
     def launch_info(self) -> dict:
