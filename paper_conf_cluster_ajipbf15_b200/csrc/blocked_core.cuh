@@ -181,6 +181,38 @@ __device__ __forceinline__ void load_vec(T (&v)[D], const T* __restrict__ src) {
   for (int d = 0; d < D; ++d) v[d] = src[d];
 }
 
+// Warp-cooperative form of block_first, called by all 32 lanes with the same (P, target):
+// lane l evaluates leaves l, l + 32, ... directly from the definition (runtime digits
+// i, j, k; loads P[d] plus the inner queues' costs on their devices; max over devices) and
+// a ballot per round finds the lowest leaf equal to `target`. Replaces a serial re-scan of
+// the whole block by one lane.
+template <typename T, int D>
+__device__ __forceinline__ uint32_t block_first_warp(const T (&P)[D], const T* __restrict__ in,
+                                                     T target) {
+  constexpr uint32_t kLeaves = (uint32_t)D * D * D;
+  const uint32_t lane = threadIdx.x & 31;
+  for (uint32_t r0 = 0; r0 < kLeaves; r0 += 32) {
+    const uint32_t l = r0 + lane;
+    bool hit = false;
+    if (l < kLeaves) {
+      const uint32_t i = l / (D * D), j = (l / D) % D, k = l % D;
+      T ms = 0;
+#pragma unroll
+      for (int d = 0; d < D; ++d) {
+        T L = P[d];
+        if (i == (uint32_t)d) L += in[0 * D + d];
+        if (j == (uint32_t)d) L += in[1 * D + d];
+        if (k == (uint32_t)d) L += in[2 * D + d];
+        ms = max2(ms, L);
+      }
+      hit = (ms == target);
+    }
+    const uint32_t b = __ballot_sync(0xffffffffu, hit);
+    if (b) return r0 + (uint32_t)(__ffs(b) - 1);
+  }
+  return 0xffffffffu;
+}
+
 // Prefix loads P of block `blk` (outer digits of queues 0..O-1), decoded from scratch,
 // on top of the devices' base loads B0 (zero unless the call is constrained).
 template <typename T, int D>

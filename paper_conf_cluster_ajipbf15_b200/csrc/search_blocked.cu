@@ -149,11 +149,15 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
       __syncthreads();
       if (bv != kNone && bv == s_gmin) atomicMin(&s_winner, (uint32_t)tid);
       __syncthreads();
-      if ((uint32_t)tid == s_winner) {
+      const uint32_t win = s_winner;
+      if (win != 0xffffffffu && (uint32_t)(tid >> 5) == (win >> 5)) {  // the winner's warp
+        const int wl = (int)(win & 31);
+        const uint64_t bb = __shfl_sync(0xffffffffu, best_blk, wl);
+        const T bt = __shfl_sync(0xffffffffu, best, wl);
         T P[D];
-        prefix_of<T, D>(P, best_blk, O, V, base0, one);
-        const uint32_t leaf = block_first<T, D>(P, in, one, best);
-        s_cand = Cand{(uint64_t)best, best_blk * (uint64_t)(D * D * D) + leaf};
+        prefix_of<T, D>(P, bb, O, V, base0, one);
+        const uint32_t leaf = block_first_warp<T, D>(P, in, bt);
+        if ((uint32_t)tid == win) s_cand = Cand{(uint64_t)bt, bb * (uint64_t)(D * D * D) + leaf};
       }
       __syncthreads();
     }

@@ -39,7 +39,10 @@ __global__ void __launch_bounds__(32, (D <= 5) ? 16 : 8) search_flat_kernel(Flat
   auto split = [&](uint64_t t) -> uint64_t {
     if (t >= nw) return W;
     const uint64_t per = W / nw, rem = W % nw;
-    return (t * per + (t < rem ? t : rem)) / chunk * chunk;
+    // align to 32 chunks (one per lane) where an epoch holds that many, so every piece
+    // keeps all lanes busy; otherwise to single chunks
+    const uint64_t unit = (nb % (32 * chunk) == 0) ? 32 * chunk : chunk;
+    return (t * per + (t < rem ? t : rem)) / unit * unit;
   };
   uint64_t f = split(w);
   const uint64_t fend = split(w + 1);
@@ -110,11 +113,14 @@ __global__ void __launch_bounds__(32, (D <= 5) ? 16 : 8) search_flat_kernel(Flat
 #pragma unroll
     for (int off = 16; off > 0; off >>= 1) wmin = min(wmin, __shfl_xor_sync(0xffffffffu, wmin, off));
     const uint32_t holders = __ballot_sync(0xffffffffu, bv != kNone && bv == wmin);
-    if (holders && lane == __ffs(holders) - 1) {
-      T P[D];
-      prefix_of<T, D>(P, best_blk, O, V, zero, a.one);
-      const uint32_t leaf = block_first<T, D>(P, in, a.one, best);
-      const uint64_t idx = best_blk * (uint64_t)(D * D * D) + leaf;
+    if (!holders) continue;
+    const int wl = __ffs(holders) - 1;
+    const uint64_t bb = __shfl_sync(0xffffffffu, best_blk, wl);
+    T P[D];
+    prefix_of<T, D>(P, bb, O, V, zero, a.one);
+    const uint32_t leaf = block_first_warp<T, D>(P, in, (T)wmin);
+    if (lane == wl) {
+      const uint64_t idx = bb * (uint64_t)(D * D * D) + leaf;
       atomicMin((unsigned long long*)&a.keys[e], (unsigned long long)((bv << a.ibits) | idx));
       __threadfence();
       // the warp that completes the epoch's block count publishes its result
