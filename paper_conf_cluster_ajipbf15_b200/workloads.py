@@ -155,3 +155,21 @@ def make(name: str, **kw):
     if name == "cfg1":
         return cfg1_npb(**kw)
     return {"cfg2": cfg2, "cfg3": cfg3, "cfg4": cfg4, "cfg5": cfg5}[name](**kw)
+
+
+def constraints(seed: int, E: int, Q: int, D: int, pin_frac: float = 0.25, mask_frac: float = 0.25,
+                base_hi: int = 1 << 20):
+    """Seeded constraints for the constrained variant (NEXT-3): per-device base loads
+    (queues outside the pool, SCHED_OFF) uniform in [0, base_hi), and per
+    queue an eligible-device mask: a fraction pinned to one device, a fraction restricted to
+    a random non-empty subset, the rest unconstrained (mask 0)."""
+    rng = np.random.default_rng(seed)
+    base = rng.integers(0, base_hi, size=(E, D), dtype=np.uint64)
+    elig = np.zeros((E, Q), dtype=np.uint16)
+    u = rng.random((E, Q))
+    pins = u < pin_frac
+    elig[pins] = (1 << rng.integers(0, D, size=int(pins.sum()))).astype(np.uint16)
+    sub = (u >= pin_frac) & (u < pin_frac + mask_frac)
+    masks = rng.integers(1, 1 << D, size=int(sub.sum())).astype(np.uint16)
+    elig[sub] = masks
+    return base, elig

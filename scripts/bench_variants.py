@@ -1,0 +1,80 @@
+"""Measure the NEXT-3 variants and the alternative batched kernel on one GPU (not the
+driver's bench line): constrained search, mapping scoring, CTA-per-epoch vs flattened
+batched kernel. Prints one JSON line per measurement.
+
+    python scripts/bench_variants.py [--reps 10]
+"""
+import argparse
+import json
+import os
+import statistics
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+from paper_conf_cluster_ajipbf15_b200 import Mapper, workloads  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--reps", type=int, default=10)
+args = ap.parse_args()
+dev = torch.device("cuda", 0)
+
+
+def t(x):
+    return torch.from_numpy(np.ascontiguousarray(x)).to(dev)
+
+
+def timed(m, fn, mappings):
+    for _ in range(3):
+        fn()
+    ks = []
+    for _ in range(args.reps):
+        fn()
+        ks.append(m.last_kernel_time_ms()[0])
+    k = statistics.median(ks)
+    return {"kernel_ms": k, "mappings_per_s": mappings / (k / 1e3)}
+
+
+with Mapper(0) as m:
+    m.set_timing(1)
+    for name in ("cfg5", "cfg4", "cfg2"):
+        K, X = workloads.make(name)
+        E, Q, D = K.shape
+        N = E * D**Q
+        base, elig = workloads.constraints(11, E, Q, D)
+        Kd, Xd, Bd, Ed = t(K), t(X), t(base), t(elig)
+        r0 = timed(m, lambda: m.map_queues(Kd, Xd), N)
+        r1 = timed(m, lambda: m.map_queues_constrained(Kd, Xd, Bd, Ed), N)
+        print(json.dumps({"measure": "constrained_vs_plain", "workload": name, "plain": r0,
+                          "constrained": r1, "path": m.launch_info()["path"],
+                          "constraints": "25% queues pinned, 25% masked, base loads U[0,2^20)"}), flush=True)
+    K, X = workloads.cfg2()
+    Kd, Xd = t(K), t(X)
+    for path, label in ((1, "cta_per_epoch"), (5, "flattened")):
+        m.force_path(path)
+        r = timed(m, lambda: m.map_queues(Kd, Xd), K.shape[0] * 4**8)
+        print(json.dumps({"measure": "batched_kernel", "workload": "cfg2", "kernel": label, **r}), flush=True)
+    m.force_path(0)
+    E, Q, D = 1_000_000, 8, 4
+    K, X = workloads.cfg2(E=E, seed=5)
+    mp = np.tile((np.arange(Q) % D).astype(np.uint8), (E, 1))
+    base = np.zeros((E, D), np.uint64)
+    Kd, Xd, Md, Bd = t(K), t(X), t(mp), t(base)
+    out = torch.empty(E, dtype=torch.uint64, device=dev)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    for _ in range(3):
+        m.score_mappings(Kd, Xd, Md, Bd)
+    ts = []
+    for _ in range(args.reps):
+        ev0.record()
+        m.score_mappings(Kd, Xd, Md, Bd)
+        ev1.record()
+        torch.cuda.synchronize()
+        ts.append(ev0.elapsed_time(ev1))
+    ms = statistics.median(ts)
+    nbytes = E * (2 * Q * D * 8 + D * 8 + Q + 8)
+    print(json.dumps({"measure": "score_mappings", "epochs": E, "Q": Q, "D": D, "call_ms": ms,
+                      "epochs_per_s": E / (ms / 1e3), "GB_per_s": nbytes / (ms / 1e3) / 1e9,
+                      "note": "call time incl. host overhead; round-robin mappings"}), flush=True)
