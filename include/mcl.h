@@ -125,6 +125,24 @@ mcl_status_t mcl_map_queues_constrained(mcl_mapper_t* h, uint32_t Q, uint32_t D,
                                         uint64_t* makespan);
 
 /*
+ * Exact search with pruning: returns exactly what
+ * mcl_map_queues_constrained returns (the lowest-index minimum-makespan mapping), found by
+ * a parallel depth-first branch and bound over the queue digits (lower bounds: the current
+ * max load, the largest remaining per-queue minimum cost, and the total work spread over D
+ * devices) instead of scoring all D^Q mappings. Its cost depends on the instance
+ * (time-to-solution, not mappings/s); random instances of 10^10-10^14 mappings typically
+ * need 10^2-10^6 nodes. Ineligible devices are skipped outright (a true mixed-radix
+ * search). The handle's sharding is ignored: every call solves the whole index space (a
+ * collective handle gets the same answer on every rank without communication).
+ * constraints may be NULL. mcl_last_launch_info's info[0] = 6 and info[7] = nodes visited.
+ * Same buffer rules and errors as mcl_map_queues_constrained.
+ */
+mcl_status_t mcl_map_queues_pruned(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                                   const uint64_t* cost_kernel, const uint64_t* cost_xfer,
+                                   const mcl_constraints_t* constraints, uint64_t* mapping_index,
+                                   uint8_t* mapping, uint64_t* makespan);
+
+/*
  * Score GIVEN mappings: makespan[e] = max_d (base_load[e][d] + sum over queues q with
  * mappings[e][q] == d of (cost_kernel + cost_xfer)[e][q][d]) -- e.g. a ROUND_ROBIN mapping
  * ("the next available device when the scheduler is triggered") or a

@@ -14,6 +14,7 @@ namespace mcl {
 
 constexpr uint64_t kNone = ~0ull;              // "no candidate" (both fields)
 constexpr int kMaxDevices = 16;                // D <= 16 (include/mcl.h)
+constexpr int kMaxQueues = 32;                 // Q <= 32
 constexpr uint64_t kEntryLimit = 1ull << 48;   // entries must be < 2^48 (reading R10)
 
 // Status bits written by kernels into the handle's host-mapped status word.

@@ -114,6 +114,27 @@ struct GenericArgs {
 };
 size_t generic_smem_bytes(uint32_t Q, uint32_t D, int threads);
 
+// Exact search with pruning (search_bnb.cu, NEXT-4): parallel depth-first branch and bound.
+struct BnbArgs {
+  uint32_t Q, D;
+  uint64_t E;
+  const uint64_t* K;
+  const uint64_t* X;
+  const uint64_t* base;  // [E][D] or nullptr
+  const uint16_t* elig;  // [E][Q] or nullptr
+  uint32_t k;            // subtree depth handed out by the per-epoch counter
+  uint64_t* next;        // [E] subtree counters, zero on entry, self-resetting
+  uint64_t* inc;         // [E] best (packed key or makespan) so far, all ones on entry, self-resetting
+  uint64_t* nodes;       // nodes visited (accumulated), or nullptr
+  Cand* scratch;         // [E][cpe]
+  uint32_t* done;        // [E]
+  EpochOut out;
+  int ibits;
+  volatile uint32_t* flags;
+};
+size_t bnb_smem_bytes(uint32_t Q, uint32_t D);
+cudaError_t launch_bnb(const BnbArgs& a, dim3 grid, int threads, cudaStream_t st);
+
 // Scoring of given mappings (score.cu): makespan[e] of mapping[e][.] with optional base
 // loads; a device id >= D raises kFlagBadMapping.
 cudaError_t launch_score(uint32_t Q, uint32_t D, uint64_t E, const uint64_t* K, const uint64_t* X,

@@ -99,6 +99,9 @@ struct DevBuf {
   }
 };
 
+// mcl_map_queues_pruned scores small index spaces exhaustively (measured crossover)
+constexpr uint64_t kPrunedMinMappings = 1ull << 24;
+
 bool mul_overflow_pow(uint32_t D, uint32_t Q, uint64_t limit, uint64_t* out) {
   uint64_t n = 1;
   for (uint32_t q = 0; q < Q; ++q) {
@@ -122,6 +125,7 @@ struct mcl_mapper {
   DevBuf done;             // uint32 per epoch, zero between calls
   DevBuf key, pair, gms, cand;
   DevBuf flat_keys, flat_done;  // flattened batched kernel: per-epoch key / block count
+  DevBuf bnb_next, bnb_inc, bnb_nodes;  // pruned search: subtree counters, incumbents, nodes
   DevBuf in_k, in_x, in_base, in_elig, out_idx, out_ms, out_map;  // staging for host pointers
   uint32_t* flags_host = nullptr;               // host-mapped status word
   uint32_t* flags_dev = nullptr;
@@ -310,7 +314,8 @@ void mcl_mapper_destroy(mcl_mapper_t* h) {
     DeviceGuard g(h->device);
     if (h->stream) cudaStreamSynchronize(h->stream);
     for (DevBuf* b : {&h->scratch, &h->done, &h->key, &h->pair, &h->gms, &h->cand, &h->flat_keys,
-                      &h->flat_done, &h->in_k, &h->in_base, &h->in_elig,
+                      &h->flat_done, &h->bnb_next, &h->bnb_inc, &h->bnb_nodes, &h->in_k,
+                      &h->in_base, &h->in_elig,
                       &h->in_x, &h->out_idx, &h->out_ms, &h->out_map})
       b->release();
     if (h->flags_host) cudaFreeHost(h->flags_host);
@@ -336,7 +341,7 @@ mcl_status_t mcl_set_timing(mcl_mapper_t* h, int enable) {
 }
 
 mcl_status_t mcl_force_path(mcl_mapper_t* h, int path) {
-  if (!h || path < 0 || path > 5) return MCL_E_INVAL;
+  if (!h || path < 0 || path > 6) return MCL_E_INVAL;
   h->force_path = path;
   return MCL_OK;
 }
@@ -475,7 +480,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
   if (!shard_mode && !multi && !constrained && mcl::small_supported(Q, D)) path = 4;
   else if (mcl::blocked_supported(Q, D)) path = 1;
   else path = 3;
-  if (h->force_path) {
+  if (h->force_path && h->force_path != 6) {  // 6 only affects mcl_map_queues_pruned
     const int f = h->force_path;
     const bool ok = (f == 3) || ((f == 1 || f == 2) && mcl::blocked_supported(Q, D)) ||
                     (f == 5 && epochs > 1 && !shard_mode && !multi && !constrained &&
@@ -655,6 +660,142 @@ mcl_status_t mcl_map_queues_constrained(mcl_mapper_t* h, uint32_t Q, uint32_t D,
   return map_impl(h, Q, D, epochs, cost_kernel, cost_xfer,
                   constraints ? constraints->base_load : nullptr,
                   constraints ? constraints->eligible : nullptr, mapping_index, mapping, makespan);
+}
+
+mcl_status_t mcl_map_queues_pruned(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                                   const uint64_t* cost_kernel, const uint64_t* cost_xfer,
+                                   const mcl_constraints_t* constraints, uint64_t* mapping_index,
+                                   uint8_t* mapping, uint64_t* makespan) {
+  if (!h) return MCL_E_INVAL;
+  h->last_err.clear();
+  if (Q == 0 || D == 0 || Q > MCL_MAX_QUEUES || D > MCL_MAX_DEVICES) {
+    h->last_err = "Q must be in [1, 32] and D in [1, 16]";
+    return MCL_E_INVAL;
+  }
+  uint64_t N = 0;
+  if (mul_overflow_pow(D, Q, 1ull << MCL_MAX_INDEX_BITS, &N)) {
+    h->last_err = "D^Q exceeds 2^48";
+    return MCL_E_RANGE;
+  }
+  if (epochs == 0) return MCL_OK;
+  if (!cost_kernel || !cost_xfer || !mapping_index || !makespan) {
+    h->last_err = "NULL required pointer";
+    return MCL_E_INVAL;
+  }
+  if (epochs > (1ull << 40) / ((uint64_t)Q * D)) {
+    h->last_err = "epochs too large";
+    return MCL_E_INVAL;
+  }
+  const uint64_t* base_load = constraints ? constraints->base_load : nullptr;
+  // Small index spaces: scoring every mapping is cheaper than a tree search (same result).
+  if (N < kPrunedMinMappings && h->comm == nullptr && h->world <= 1 && h->force_path != 6)
+    return map_impl(h, Q, D, epochs, cost_kernel, cost_xfer, base_load,
+                    constraints ? constraints->eligible : nullptr, mapping_index, mapping, makespan);
+  DeviceGuard g(h->device);
+  cudaStream_t s = h->stream;
+  mcl_status_t st;
+  const uint16_t* eligible = constraints ? constraints->eligible : nullptr;
+  bool dk, dx, db = true, de = true, di, dm, dmap = true;
+  if ((st = classify(h, cost_kernel, &dk)) != MCL_OK) return st;
+  if ((st = classify(h, cost_xfer, &dx)) != MCL_OK) return st;
+  if (base_load && (st = classify(h, base_load, &db)) != MCL_OK) return st;
+  if (eligible && (st = classify(h, eligible, &de)) != MCL_OK) return st;
+  if ((st = classify(h, mapping_index, &di)) != MCL_OK) return st;
+  if ((st = classify(h, makespan, &dm)) != MCL_OK) return st;
+  if (mapping && (st = classify(h, mapping, &dmap)) != MCL_OK) return st;
+  const size_t in_bytes = (size_t)epochs * Q * D * 8;
+  const void *K, *X, *B = nullptr, *El = nullptr;
+  if (h->timing >= 2) MCL_CUDA(h, cudaEventRecord(h->ev[2], s), "cudaEventRecord");
+  if ((st = stage_in(h, h->in_k, cost_kernel, in_bytes, dk, &K)) != MCL_OK) return st;
+  if ((st = stage_in(h, h->in_x, cost_xfer, in_bytes, dx, &X)) != MCL_OK) return st;
+  if (base_load && (st = stage_in(h, h->in_base, base_load, epochs * D * 8, db, &B)) != MCL_OK)
+    return st;
+  if (eligible && (st = stage_in(h, h->in_elig, eligible, epochs * Q * 2, de, &El)) != MCL_OK)
+    return st;
+  uint64_t* o_idx = mapping_index;
+  uint64_t* o_ms = makespan;
+  uint8_t* o_map = mapping;
+  if (!di) {
+    MCL_CUDA(h, h->out_idx.ensure(epochs * 8), "cudaMalloc(staging)");
+    o_idx = (uint64_t*)h->out_idx.p;
+  }
+  if (!dm) {
+    MCL_CUDA(h, h->out_ms.ensure(epochs * 8), "cudaMalloc(staging)");
+    o_ms = (uint64_t*)h->out_ms.p;
+  }
+  if (mapping && !dmap) {
+    MCL_CUDA(h, h->out_map.ensure(epochs * Q), "cudaMalloc(staging)");
+    o_map = (uint8_t*)h->out_map.p;
+  }
+  // per-epoch subtree counters (zero) and incumbents (all ones), self-resetting
+  if (h->bnb_next.cap < epochs * 8) {
+    MCL_CUDA(h, h->bnb_next.ensure(epochs * 8, true), "cudaMalloc(bnb)");
+    MCL_CUDA(h, h->bnb_inc.ensure(epochs * 8), "cudaMalloc(bnb)");
+    MCL_CUDA(h, cudaMemset(h->bnb_inc.p, 0xff, h->bnb_inc.cap), "cudaMemset(bnb)");
+  }
+  MCL_CUDA(h, h->bnb_nodes.ensure(8, true), "cudaMalloc(bnb)");
+  MCL_CUDA(h, cudaMemsetAsync(h->bnb_nodes.p, 0, 8, s), "cudaMemset(bnb)");
+  MCL_CUDA(h, h->done.ensure(epochs * sizeof(uint32_t), true), "cudaMalloc(done)");
+
+  // one CTA per SM shares an epoch's search when there are few epochs; the shared
+  // incumbent prunes so much that wider grids mostly add subtree-root checks
+  const int threads = 128;
+  const uint64_t slots = (uint64_t)h->num_sms;
+  uint64_t cpe = epochs >= slots ? 1 : (slots + epochs - 1) / epochs;
+  if (cpe > (N + threads - 1) / threads) cpe = std::max<uint64_t>(1, (N + threads - 1) / threads);
+  if (cpe > 65535) cpe = 65535;
+  dim3 grid((unsigned)cpe, (unsigned)std::min<uint64_t>(epochs, 65535), 1);
+  // subtree depth: about two subtrees per thread of an epoch
+  uint32_t k = 0;
+  uint64_t nsub = 1;
+  while (k < Q && nsub < 2ull * threads * cpe) {
+    nsub *= D;
+    ++k;
+  }
+  if (D == 1) k = Q;
+  mcl::BnbArgs a{};
+  a.Q = Q; a.D = D; a.E = epochs; a.K = (const uint64_t*)K; a.X = (const uint64_t*)X;
+  a.base = (const uint64_t*)B; a.elig = (const uint16_t*)El; a.k = k;
+  a.next = (uint64_t*)h->bnb_next.p; a.inc = (uint64_t*)h->bnb_inc.p;
+  a.nodes = (uint64_t*)h->bnb_nodes.p; a.done = (uint32_t*)h->done.p;
+  a.out = mcl::EpochOut{o_idx, o_ms, o_map, nullptr, nullptr};
+  a.ibits = mcl::index_bits_host(N); a.flags = h->flags_dev;
+  if (grid.x > 1) {
+    MCL_CUDA(h, h->scratch.ensure((size_t)epochs * grid.x * sizeof(Cand)), "cudaMalloc(scratch)");
+    a.scratch = (Cand*)h->scratch.p;
+  }
+  *(volatile uint32_t*)h->flags_host = 0;
+  if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[0], s), "cudaEventRecord");
+  MCL_CUDA(h, mcl::launch_bnb(a, grid, threads, s), "search_bnb launch");
+  if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[1], s), "cudaEventRecord");
+  uint64_t nodes = 0;
+  MCL_CUDA(h, cudaMemcpyAsync(&nodes, h->bnb_nodes.p, 8, cudaMemcpyDeviceToHost, s), "D2H");
+  MCL_CUDA(h, cudaStreamSynchronize(s), "search_bnb");
+  const uint32_t flags = *(volatile uint32_t*)h->flags_host;
+  if (flags & 1u) {
+    h->last_err = "a cost entry or base load is >= 2^48";
+    return MCL_E_RANGE;
+  }
+  if (flags & 8u) {
+    h->last_err = "a queue has no eligible device below D";
+    return MCL_E_INVAL;
+  }
+  h->info[0] = 6;
+  h->info[1] = 1;
+  h->info[2] = (int64_t)grid.x * grid.y;
+  h->info[3] = threads;
+  h->info[4] = 0;
+  h->info[5] = a.ibits;
+  h->info[6] = 0;
+  h->info[7] = (int64_t)nodes;
+  if (!di) MCL_CUDA(h, cudaMemcpyAsync(mapping_index, o_idx, epochs * 8, cudaMemcpyDeviceToHost, s), "D2H");
+  if (!dm) MCL_CUDA(h, cudaMemcpyAsync(makespan, o_ms, epochs * 8, cudaMemcpyDeviceToHost, s), "D2H");
+  if (mapping && !dmap)
+    MCL_CUDA(h, cudaMemcpyAsync(mapping, o_map, epochs * Q, cudaMemcpyDeviceToHost, s), "D2H");
+  if (h->timing >= 2) MCL_CUDA(h, cudaEventRecord(h->ev[3], s), "cudaEventRecord");
+  MCL_CUDA(h, cudaStreamSynchronize(s), "D2H");
+  h->timing_pending = h->timing > 0;
+  return MCL_OK;
 }
 
 mcl_status_t mcl_score_mappings(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,

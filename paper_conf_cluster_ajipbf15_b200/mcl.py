@@ -17,7 +17,8 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libmcl.so")
 
 MCL_OK, MCL_E_INVAL, MCL_E_RANGE, MCL_E_CUDA, MCL_E_NCCL, MCL_E_NOMEM = 0, -1, -2, -3, -4, -5
-PATH_NAMES = {1: "blocked_u32", 2: "blocked_u64", 3: "generic", 4: "small_batched", 5: "flat_u32"}
+PATH_NAMES = {1: "blocked_u32", 2: "blocked_u64", 3: "generic", 4: "small_batched", 5: "flat_u32",
+              6: "pruned"}
 
 # Every symbol the headers declare (tests check the library exports all of them).
 EXPORTED = [
@@ -26,7 +27,7 @@ EXPORTED = [
     "mcl_set_timing", "mcl_last_kernel_time", "mcl_force_path", "mcl_probe_int_rate",
     "mcl_device_sms",
     "mcl_comm_unique_id", "mcl_comm_init", "mcl_comm_destroy",
-    "mcl_map_queues_constrained", "mcl_score_mappings",
+    "mcl_map_queues_constrained", "mcl_score_mappings", "mcl_map_queues_pruned",
 ]
 
 
@@ -89,6 +90,8 @@ def load_library(path: str | None = None) -> ctypes.CDLL:
         "mcl_map_queues_constrained": (i32, [vp, u32, u32, u64, vp, vp,
                                              ctypes.POINTER(mcl_constraints_t), vp, vp, vp]),
         "mcl_score_mappings": (i32, [vp, u32, u32, u64, vp, vp, vp, vp, vp]),
+        "mcl_map_queues_pruned": (i32, [vp, u32, u32, u64, vp, vp,
+                                        ctypes.POINTER(mcl_constraints_t), vp, vp, vp]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -254,7 +257,13 @@ class Mapper:
         self.map_queues_into(K, X, idx, mp, ms)
         return idx, mp, ms
 
-    def map_queues_constrained(self, K, X, base=None, eligible=None, with_mapping: bool = True):
+    def map_queues_pruned(self, K, X, base=None, eligible=None, with_mapping: bool = True):
+        """Exact search with pruning (include/mcl.h mcl_map_queues_pruned): same result as
+        map_queues_constrained, time depends on the instance."""
+        return self.map_queues_constrained(K, X, base, eligible, with_mapping, _fn="mcl_map_queues_pruned")
+
+    def map_queues_constrained(self, K, X, base=None, eligible=None, with_mapping: bool = True,
+                               _fn: str = "mcl_map_queues_constrained"):
         """Constrained search (include/mcl.h mcl_map_queues_constrained): ``base`` [E, D]
         uint64 device base loads or None, ``eligible`` [E, Q] uint16 device masks (0 = any)
         or None. Outputs are allocated like K; returns (index, mapping or None, makespan)."""
@@ -272,10 +281,9 @@ class Mapper:
         pm, _m = _ptr_and_keepalive(ms, np.uint64)
         pmap = _ptr_and_keepalive(mp, np.uint8)[0] if mp is not None else None
         c = mcl_constraints_t(pb, pe)
-        st = load_library().mcl_map_queues_constrained(self.handle, Q, D, E, pk, px, ctypes.byref(c),
-                                                       pi, pmap, pm)
+        st = getattr(load_library(), _fn)(self.handle, Q, D, E, pk, px, ctypes.byref(c), pi, pmap, pm)
         if st != MCL_OK:
-            raise MclError(st, "mcl_map_queues_constrained", mcl_last_error_string(self.handle))
+            raise MclError(st, _fn, mcl_last_error_string(self.handle))
         return idx, mp, ms
 
     def score_mappings(self, K, X, mappings, base=None):
@@ -314,11 +322,13 @@ class Mapper:
     def launch_info(self) -> dict:
         i = mcl_last_launch_info(self.handle)
         return {"path": PATH_NAMES.get(i[0], str(i[0])), "launches": i[1], "ctas": i[2],
-                "threads": i[3], "allreduce": bool(i[4]), "index_bits": i[5], "two_step": bool(i[6])}
+                "threads": i[3], "allreduce": bool(i[4]), "index_bits": i[5], "two_step": bool(i[6]),
+                "nodes": i[7]}
 
     def force_path(self, path: int) -> None:
         """Testing aid: 0 auto, 1 blocked u32 (CTA per epoch), 2 blocked u64, 3 generic,
-        4 small batched, 5 flattened batched blocked u32."""
+        4 small batched, 5 flattened batched blocked u32, 6 branch-and-bound kernel in
+        map_queues_pruned even for small index spaces."""
         st = load_library().mcl_force_path(self.handle, path)
         if st != MCL_OK:
             raise MclError(st, "mcl_force_path")

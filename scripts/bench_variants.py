@@ -78,3 +78,27 @@ with Mapper(0) as m:
     print(json.dumps({"measure": "score_mappings", "epochs": E, "Q": Q, "D": D, "call_ms": ms,
                       "epochs_per_s": E / (ms / 1e3), "GB_per_s": nbytes / (ms / 1e3) / 1e9,
                       "note": "call time incl. host overhead; round-robin mappings"}), flush=True)
+
+# ---- NEXT-4: pruned exact search, time-to-solution vs exhaustive ----
+with Mapper(0) as m:
+    m.set_timing(1)
+    for name in ("cfg5", "cfg4", "cfg2", "cfg3"):
+        K, X = workloads.make(name)
+        E, Q, D = K.shape
+        Kd, Xd = t(K), t(X)
+        ex = timed(m, lambda: m.map_queues(Kd, Xd), E * D**Q)
+        pr = timed(m, lambda: m.map_queues_pruned(Kd, Xd), E * D**Q)
+        a = m.map_queues_pruned(Kd, Xd)
+        b = m.map_queues(Kd, Xd)
+        same = bool((a[0] == b[0]).all().item() and (a[2] == b[2]).all().item())
+        print(json.dumps({"measure": "pruned_vs_exhaustive", "workload": name,
+                          "exhaustive_kernel_ms": ex["kernel_ms"], "pruned_kernel_ms": pr["kernel_ms"],
+                          "speedup": ex["kernel_ms"] / pr["kernel_ms"], "nodes": m.launch_info()["nodes"],
+                          "identical_result": same}), flush=True)
+    for seed, (Q, D) in enumerate(((16, 8), (20, 4), (24, 3))):
+        K, X = workloads.random_tables(500 + seed, 1, Q, D, hi=1 << 22)
+        Kd, Xd = t(K), t(X)
+        pr = timed(m, lambda: m.map_queues_pruned(Kd, Xd), D**Q)
+        print(json.dumps({"measure": "pruned_large", "Q": Q, "D": D, "mappings": D**Q,
+                          "pruned_kernel_ms": pr["kernel_ms"], "nodes": m.launch_info()["nodes"],
+                          "exhaustive_estimate_ms": D**Q / 1.15e13 * 1e3}), flush=True)
