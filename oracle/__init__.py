@@ -20,16 +20,19 @@ import subprocess
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_SRC = os.path.join(_HERE, "oracle.c")
+_SRCS = [os.path.join(_HERE, "oracle.c"), os.path.join(_HERE, "costs.c")]
 _LIB = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
 
 def build(force: bool = False) -> str:
-    """Compile oracle.c into oracle/liboracle.so with gcc (plain C11 + pthreads)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+    """Compile oracle.c + costs.c into oracle/liboracle.so with gcc (plain C11 + pthreads;
+    no fused multiply-add, so the fp64 cost-model arithmetic is rounded as written)."""
+    stale = not os.path.exists(_LIB) or any(os.path.getmtime(_LIB) < os.path.getmtime(s) for s in _SRCS)
+    if force or stale:
         subprocess.check_call(
-            ["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-pthread", "-o", _LIB, _SRC]
+            ["gcc", "-O2", "-std=c11", "-ffp-contract=off", "-fPIC", "-shared", "-pthread", "-o", _LIB]
+            + _SRCS + ["-lm"]
         )
     return _LIB
 
@@ -54,6 +57,13 @@ def _load():
             ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p,
             ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_int,
             ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+        ]
+        lib.oracle_build_costs.restype = ctypes.c_int
+        lib.oracle_build_costs.argtypes = [
+            ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_uint32,
+            ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+            ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+            ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p,
         ]
         lib.oracle_score_base.restype = ctypes.c_uint64
         lib.oracle_score_base.argtypes = [
@@ -149,3 +159,33 @@ def oracle_score_base(K, X, base, mapping) -> int:
     b = None if base is None else np.ascontiguousarray(base, dtype=np.uint64)
     return int(_load().oracle_score_base(Q, D, K.ctypes.data, X.ctypes.data,
                                          None if b is None else b.ctypes.data, mpg.ctypes.data))
+
+
+def oracle_build_costs(Q: int, D: int, model: dict):
+    """Cost tables (NEXT-1) from a cost model dict with keys: profile [n_kernels, D] u64,
+    offsets [E*Q+1] u64, kernel_ids [nnz] u32, bytes [E, Q] u64, source [E, Q] i32
+    (-1 = host), cached [E, Q] u16 or None, sizes [M] u64, h2d_bw / d2h_bw [D, M] f64,
+    host_shared (int bit mask). Returns (K, X) uint64 [E, Q, D]."""
+    prof = np.ascontiguousarray(model["profile"], dtype=np.uint64)
+    off = np.ascontiguousarray(model["offsets"], dtype=np.uint64)
+    ids = np.ascontiguousarray(model["kernel_ids"], dtype=np.uint32)
+    nbytes = np.ascontiguousarray(model["bytes"], dtype=np.uint64)
+    src = np.ascontiguousarray(model["source"], dtype=np.int32)
+    cached = model.get("cached")
+    cached = None if cached is None else np.ascontiguousarray(cached, dtype=np.uint16)
+    sizes = np.ascontiguousarray(model["sizes"], dtype=np.uint64)
+    h2d = np.ascontiguousarray(model["h2d_bw"], dtype=np.float64)
+    d2h = np.ascontiguousarray(model["d2h_bw"], dtype=np.float64)
+    E = nbytes.shape[0]
+    K = np.zeros((E, Q, D), dtype=np.uint64)
+    X = np.zeros((E, Q, D), dtype=np.uint64)
+    ids_ptr = ids.ctypes.data if ids.size else None
+    rc = _load().oracle_build_costs(
+        Q, D, E, prof.shape[0], prof.ctypes.data, off.ctypes.data, ids_ptr, nbytes.ctypes.data,
+        src.ctypes.data, None if cached is None else cached.ctypes.data, sizes.shape[0],
+        sizes.ctypes.data, h2d.ctypes.data, d2h.ctypes.data, int(model.get("host_shared", 0)),
+        K.ctypes.data, X.ctypes.data,
+    )
+    if rc != 0:
+        raise OracleError(rc)
+    return K, X

@@ -582,6 +582,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
     h->info[4] = 0;
     h->info[5] = ibits;
     h->info[6] = 0;
+    h->info[7] = 0;
 
     if (multi) {
       ncclResult_t r = nccl().AllReduce(out.key, out.key, epochs, ncclUint64, ncclMin, h->comm, s);

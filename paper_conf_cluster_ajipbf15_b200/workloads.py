@@ -173,3 +173,39 @@ def constraints(seed: int, E: int, Q: int, D: int, pin_frac: float = 0.25, mask_
     masks = rng.integers(1, 1 << D, size=int(sub.sum())).astype(np.uint16)
     elig[sub] = masks
     return base, elig
+
+
+def cost_model(seed: int, E: int, Q: int, D: int, n_kernels: int = 64, max_kernels: int = 16,
+               cached_frac: float = 0.1):
+    """Seeded inputs of the cost-table construction step (NEXT-1), shaped by the paper:
+    a kernel profile table whose GPU/CPU time ratios span Fig. 3's
+    range (0.05x .. 4x, L1391-1401, L2058-2060); 1..max_kernels invocations per (epoch,
+    queue) (a kernel epoch, L1142-1158); working sets log-uniform in 1 KiB .. 256 MiB (Fig. 6
+    axis, L1854-1876) resident on the host or a GPU; bandwidth curves sampled at powers of
+    two from 1 KiB to 1 GiB, latency-bound at small sizes ("from being latency bound to
+    bandwidth bound", L896-898); device 0 is the CPU device working on host memory."""
+    rng = np.random.default_rng(seed)
+    cpu = rng.integers(100_000, 10_000_000, size=n_kernels)
+    profile = np.zeros((n_kernels, D), dtype=np.uint64)
+    profile[:, 0] = cpu
+    for d in range(1, D):
+        ratio = np.exp(rng.uniform(math.log(0.05), math.log(4.0), size=n_kernels))
+        profile[:, d] = np.maximum(1, np.rint(cpu * ratio)).astype(np.uint64)
+    counts = rng.integers(1, max_kernels + 1, size=E * Q)
+    offsets = np.zeros(E * Q + 1, dtype=np.uint64)
+    offsets[1:] = np.cumsum(counts)
+    kernel_ids = rng.integers(0, n_kernels, size=int(offsets[-1])).astype(np.uint32)
+    nbytes = np.exp(rng.uniform(math.log(1024), math.log(256 * MIB), size=(E, Q))).astype(np.uint64)
+    source = np.where(rng.random((E, Q)) < 0.5, -1, rng.integers(1, max(2, D), size=(E, Q))).astype(np.int32)
+    if D == 1:
+        source[:] = -1
+    cached = np.where(rng.random((E, Q)) < cached_frac, rng.integers(0, 1 << D, size=(E, Q)), 0).astype(np.uint16)
+    sizes = (1024 * (2 ** np.arange(21))).astype(np.uint64)
+    peak_h2d = rng.uniform(5.0, 12.0, size=D)      # GB/s == bytes/ns
+    peak_d2h = peak_h2d * rng.uniform(0.8, 1.0, size=D)
+    half = 65536.0
+    s = sizes.astype(np.float64)
+    h2d = (peak_h2d[:, None] * s[None, :] / (s[None, :] + half)).astype(np.float64)
+    d2h = (peak_d2h[:, None] * s[None, :] / (s[None, :] + half)).astype(np.float64)
+    return dict(profile=profile, offsets=offsets, kernel_ids=kernel_ids, bytes=nbytes, source=source,
+                cached=cached, sizes=sizes, h2d_bw=h2d, d2h_bw=d2h, host_shared=1)
