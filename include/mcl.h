@@ -143,6 +143,56 @@ mcl_status_t mcl_map_queues_pruned(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint
                                    uint8_t* mapping, uint64_t* makespan);
 
 /*
+ * Cost-table construction: the mapper's inputs built on the GPU from the
+ * runtime's profiles.
+ *   K[e][q][d] = sum over the kernel invocations enqueued to queue q in epoch e of
+ *                kernel_profile[kernel][d]  (kernel profiler: each kernel run once per
+ *                device; an epoch's "aggregate performance vector",
+ *                L1154-1158). Repeated invocations count each time.
+ *   X[e][q][d] = 0 if the queue's data is on device d (source == d) or a copy is cached
+ *                there (cached bit d, L1309-1321); else t_h2d(d) when the data is in host
+ *                memory (source == -1), or t_d2h(source) + t_h2d(d) when it is on another
+ *                device ("a D2H-H2D double operation via the host memory", L1293-1301). A
+ *                device with host_shared bit d set (an OpenCL CPU device on host memory)
+ *                has no H2D / D2H leg. t(curve, bytes) = ceil(bytes / bw(bytes)) ns with bw
+ *                (bytes per ns) linearly interpolated in bytes between the two neighbouring
+ *                sampled sizes and clamped outside them (device profiler: bandwidths over
+ *                sizes "from latency bound to bandwidth bound", "simple interpolation
+ *                techniques" for other sizes, L877-913); IEEE fp64, no fused multiply-add.
+ * Every array may be host or device memory (host arrays are staged).
+ */
+typedef struct {
+  uint32_t num_kernels;            /* rows of kernel_profile                             */
+  const uint64_t* kernel_profile;  /* [num_kernels][D] ns per invocation on each device  */
+  const uint64_t* offsets;         /* [E*Q + 1] CSR offsets of (e, q) into kernel_ids     */
+  const uint32_t* kernel_ids;      /* [num_invocations] kernel of each invocation         */
+  uint64_t num_invocations;        /* == offsets[E*Q]                                     */
+  const uint64_t* bytes;           /* [E][Q] working-set bytes of each queue              */
+  const int32_t* source;           /* [E][Q] device holding the data, -1 = host memory    */
+  const uint16_t* cached;          /* [E][Q] devices already holding a copy, or NULL      */
+  uint32_t num_sizes;              /* M sampled sizes, 1..64                              */
+  const uint64_t* sizes;           /* [M] strictly ascending bytes                        */
+  const double* h2d_bw;            /* [D][M] host->device bandwidth, bytes/ns, > 0        */
+  const double* d2h_bw;            /* [D][M] device->host bandwidth, bytes/ns, > 0        */
+  uint32_t host_shared;            /* bit d: device d works on host memory                */
+} mcl_cost_model_t;
+
+/* Build K and X ([E][Q][D] uint64, host or device outputs). Errors: MCL_E_INVAL (NULL
+   pointer, Q/D out of bounds, num_sizes outside 1..64, a kernel id >= num_kernels, a source
+   outside -1..D-1, bad offsets, sizes not ascending or a bandwidth <= 0), MCL_E_RANGE (a
+   cost >= 2^48), MCL_E_CUDA. */
+mcl_status_t mcl_build_costs(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                             const mcl_cost_model_t* model, uint64_t* cost_kernel,
+                             uint64_t* cost_xfer);
+
+/* The whole pipeline in one call: build K and X in handle-owned device memory, then run
+   mcl_map_queues_constrained on them (constraints may be NULL). Outputs as mcl_map_queues. */
+mcl_status_t mcl_map_from_profiles(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                                   const mcl_cost_model_t* model,
+                                   const mcl_constraints_t* constraints,
+                                   uint64_t* mapping_index, uint8_t* mapping, uint64_t* makespan);
+
+/*
  * Score GIVEN mappings: makespan[e] = max_d (base_load[e][d] + sum over queues q with
  * mappings[e][q] == d of (cost_kernel + cost_xfer)[e][q][d]) -- e.g. a ROUND_ROBIN mapping
  * ("the next available device when the scheduler is triggered") or a

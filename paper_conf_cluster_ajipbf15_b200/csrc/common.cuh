@@ -24,6 +24,7 @@ enum : uint32_t {
   kFlagNoPack = 4u,    // makespan does not fit beside the index in one u64 key (NCCL path)
   kFlagInfeasible = 8u,  // constrained call: some queue has no eligible device below D
   kFlagBadMapping = 16u, // scoring call: a mapping names a device >= D
+  kFlagBadModel = 32u,   // cost model: bad kernel id / source / offsets / curve
 };
 
 __device__ __forceinline__ bool cand_less(const Cand& a, const Cand& b) {

@@ -1,0 +1,164 @@
+// costs.cu -- cost-table construction: the mapper's inputs K and X built on
+// the GPU from the kernel profiles, the epochs' kernel lists and the device profiles.
+//
+//  K[e][q][d] = sum over the kernel invocations enqueued to queue q in epoch e of
+//               profile[kernel][d]   (kernel profiler; "the aggregate
+//               performance vector of the epoch", L1154-1158)
+//  X[e][q][d] = 0                                     data on d, or a copy cached on d
+//                                                     (data caching, L1309-1321)
+//             = t_h2d(d, bytes)                       data in host memory
+//             = t_d2h(src, bytes) + t_h2d(d, bytes)   data on another device: "a D2H-H2D
+//                                                     double operation via the host", L1293-1301
+//  with no H2D/D2H leg for a device flagged host_shared, and t(curve, b) = ceil(b / bw(b))
+//  ns, bw linearly interpolated between the sampled sizes and clamped at the ends ("simple
+//  interpolation techniques", L905-907). fp64 with explicitly rounded operations (no FMA
+//  contraction), so the result is bit-identical to a plain IEEE evaluation.
+//
+// Tiles of 256 (epoch, queue) pairs per CTA: the tile's CSR offsets and its contiguous
+// slice of kernel ids are staged in shared memory with coalesced loads (the profile table
+// too, when it fits), then one thread per pair sums its invocations' profile rows and
+// interpolates the curves (sizes and bandwidths in shared memory; one segment search serves
+// every device because the sample sizes are shared). Memory-bound: reads ids / offsets /
+// bytes / source / cached once, writes 2 x D x 8 bytes per pair.
+#include "common.cuh"
+#include "kernels.h"
+
+namespace mcl {
+
+namespace {
+
+__device__ __forceinline__ double lerp_bw(const double* __restrict__ bw, uint32_t i, double f,
+                                          bool clamp_lo, bool clamp_hi, uint32_t M) {
+  if (clamp_lo) return bw[0];
+  if (clamp_hi) return bw[M - 1];
+  return __dadd_rn(bw[i], __dmul_rn(f, __dsub_rn(bw[i + 1], bw[i])));
+}
+
+__device__ __forceinline__ uint64_t transfer_ns(uint64_t bytes, double bw) {
+  if (bytes == 0) return 0;
+  return (uint64_t)ceil(__ddiv_rn(__ull2double_rn(bytes), bw));
+}
+
+}  // namespace
+
+constexpr int kCostTile = 256;      // (epoch, queue) pairs per CTA tile (= blockDim.x)
+constexpr int kIdsCap = 8192;       // kernel ids of a tile staged in shared memory
+constexpr int kProfCapBytes = 32768;  // profile table staged when it fits
+
+__global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const uint32_t D = a.D, M = a.M;
+  const int tid = threadIdx.x;
+  // layout: sizes[M] u64 | h2d[D][M] f64 | d2h[D][M] f64 | off[kCostTile+1] u64 |
+  //         prof[num_kernels][D] u64 (if it fits) | ids[kIdsCap] u32
+  uint64_t* s_sizes = reinterpret_cast<uint64_t*>(smem_raw);
+  double* s_h2d = reinterpret_cast<double*>(s_sizes + M);
+  double* s_d2h = s_h2d + (size_t)D * M;
+  uint64_t* s_off = reinterpret_cast<uint64_t*>(s_d2h + (size_t)D * M);
+  uint64_t* s_prof = s_off + (kCostTile + 1);
+  const bool prof_in_smem = (size_t)a.num_kernels * D * 8 <= (size_t)kProfCapBytes;
+  uint32_t* s_ids = reinterpret_cast<uint32_t*>(s_prof + (prof_in_smem ? (size_t)a.num_kernels * D : 0));
+  for (uint32_t t = tid; t < M; t += blockDim.x) s_sizes[t] = a.sizes[t];
+  for (uint32_t t = tid; t < D * M; t += blockDim.x) {
+    s_h2d[t] = a.h2d[t];
+    s_d2h[t] = a.d2h[t];
+  }
+  if (prof_in_smem)
+    for (uint32_t t = tid; t < a.num_kernels * D; t += blockDim.x) s_prof[t] = a.profile[t];
+  __syncthreads();
+  const uint64_t* prof = prof_in_smem ? s_prof : a.profile;
+  uint32_t status = 0;
+  if (blockIdx.x == 0 && tid == 0) {  // model validation (once)
+    for (uint32_t i = 0; i + 1 < M; ++i)
+      if (!(s_sizes[i] < s_sizes[i + 1])) status |= kFlagBadModel;
+    for (uint32_t i = 0; i < D * M; ++i)
+      if (!(s_h2d[i] > 0.0) || !(s_d2h[i] > 0.0)) status |= kFlagBadModel;
+    if (a.offsets[a.EQ] != a.nnz) status |= kFlagBadModel;
+  }
+  const uint64_t ntiles = (a.EQ + kCostTile - 1) / kCostTile;
+  for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const uint64_t t0 = tile * kCostTile;
+    const uint32_t n = (uint32_t)((a.EQ - t0 < (uint64_t)kCostTile) ? a.EQ - t0 : kCostTile);
+    __syncthreads();  // the previous tile's staging is no longer read
+    for (uint32_t i = tid; i <= n; i += blockDim.x) s_off[i] = a.offsets[t0 + i];
+    __syncthreads();
+    // the tile's invocation lists are one contiguous slice of kernel_ids: stage it coalesced
+    const uint64_t lo = s_off[0], hi = s_off[n];
+    const bool ids_in_smem = hi >= lo && hi <= a.nnz && hi - lo <= (uint64_t)kIdsCap;
+    if (ids_in_smem)
+      for (uint64_t j = lo + tid; j < hi; j += blockDim.x) s_ids[j - lo] = a.ids[j];
+    __syncthreads();
+    if ((uint32_t)tid < n) {
+      const uint64_t eq = t0 + tid;
+      // ---- kernel part: sum of the invoked kernels' profile rows ----
+      uint64_t k[kMaxDevices];
+#pragma unroll
+      for (int d = 0; d < kMaxDevices; ++d) k[d] = 0;
+      const uint64_t j0 = s_off[tid], j1 = s_off[tid + 1];
+      bool ok = j0 <= j1 && j1 <= a.nnz;
+      for (uint64_t j = j0; ok && j < j1; ++j) {
+        const uint32_t kid = ids_in_smem ? s_ids[j - lo] : a.ids[j];
+        if (kid >= a.num_kernels) {
+          ok = false;
+          break;
+        }
+        const uint64_t* row = prof + (uint64_t)kid * D;
+#pragma unroll
+        for (int d = 0; d < kMaxDevices; ++d)
+          if (d < (int)D) k[d] += row[d];
+      }
+      // ---- transfer part ----
+      const uint64_t bytes = a.bytes[eq];
+      const int32_t src = a.source[eq];
+      const uint32_t cached = a.cached ? (uint32_t)a.cached[eq] : 0u;
+      ok = ok && src >= -1 && src < (int32_t)D;
+      if (!ok) status |= kFlagBadModel;
+      const bool clo = bytes <= s_sizes[0], chi = bytes >= s_sizes[M - 1];
+      uint32_t seg = 0;
+      double f = 0.0;
+      if (ok && !clo && !chi) {
+        while (!(s_sizes[seg] <= bytes && bytes < s_sizes[seg + 1])) ++seg;
+        f = __ddiv_rn(__ull2double_rn(bytes - s_sizes[seg]),
+                      __ull2double_rn(s_sizes[seg + 1] - s_sizes[seg]));
+      }
+      uint64_t down = 0;
+      if (ok && src >= 0 && !((a.host_shared >> src) & 1u))
+        down = transfer_ns(bytes, lerp_bw(s_d2h + (size_t)src * M, seg, f, clo, chi, M));
+#pragma unroll
+      for (int d = 0; d < kMaxDevices; ++d) {
+        if (d >= (int)D) break;
+        uint64_t x = 0;
+        if (ok && !(src == d || ((cached >> d) & 1u))) {
+          const uint64_t up = ((a.host_shared >> d) & 1u)
+                                  ? 0
+                                  : transfer_ns(bytes, lerp_bw(s_h2d + (size_t)d * M, seg, f, clo, chi, M));
+          x = down + up;
+        }
+        if (k[d] >= kEntryLimit || x >= kEntryLimit) status |= kFlagRange;
+        a.K[eq * D + d] = k[d];
+        a.X[eq * D + d] = x;
+      }
+    }
+  }
+  if (__any_sync(0xffffffffu, status != 0)) {
+    const uint32_t all = __reduce_or_sync(0xffffffffu, status);
+    if ((tid & 31) == 0) raise_flag(a.flags, all);
+  }
+}
+
+cudaError_t launch_build_costs(const CostArgs& a, int num_sms, cudaStream_t st) {
+  size_t smem = (size_t)a.M * 8 + 2 * (size_t)a.D * a.M * 8 + (kCostTile + 1) * 8;
+  if ((size_t)a.num_kernels * a.D * 8 <= (size_t)kProfCapBytes) smem += (size_t)a.num_kernels * a.D * 8;
+  smem += (size_t)kIdsCap * 4;
+  static SmemAttrCache cache;
+  cudaError_t err = ensure_smem(build_costs_kernel, smem, cache);
+  if (err != cudaSuccess) return err;
+  uint64_t grid = (a.EQ + kCostTile - 1) / kCostTile;
+  const uint64_t cap = (uint64_t)num_sms * 3;
+  if (grid > cap) grid = cap;
+  if (grid == 0) grid = 1;
+  build_costs_kernel<<<(unsigned)grid, kCostTile, smem, st>>>(a);
+  return cudaGetLastError();
+}
+
+}  // namespace mcl

@@ -135,6 +135,29 @@ struct BnbArgs {
 size_t bnb_smem_bytes(uint32_t Q, uint32_t D);
 cudaError_t launch_bnb(const BnbArgs& a, dim3 grid, int threads, cudaStream_t st);
 
+// Cost-table construction (costs.cu, NEXT-1).
+struct CostArgs {
+  uint32_t D;
+  uint64_t EQ;                // epochs x queues
+  uint32_t num_kernels;
+  const uint64_t* profile;    // [num_kernels][D]
+  const uint64_t* offsets;    // [EQ + 1]
+  const uint32_t* ids;        // [nnz]
+  uint64_t nnz;
+  const uint64_t* bytes;      // [EQ]
+  const int32_t* source;      // [EQ]
+  const uint16_t* cached;     // [EQ] or nullptr
+  uint32_t M;
+  const uint64_t* sizes;      // [M]
+  const double* h2d;          // [D][M]
+  const double* d2h;          // [D][M]
+  uint32_t host_shared;
+  uint64_t* K;                // [EQ][D] out
+  uint64_t* X;                // [EQ][D] out
+  volatile uint32_t* flags;
+};
+cudaError_t launch_build_costs(const CostArgs& a, int num_sms, cudaStream_t st);
+
 // Scoring of given mappings (score.cu): makespan[e] of mapping[e][.] with optional base
 // loads; a device id >= D raises kFlagBadMapping.
 cudaError_t launch_score(uint32_t Q, uint32_t D, uint64_t E, const uint64_t* K, const uint64_t* X,

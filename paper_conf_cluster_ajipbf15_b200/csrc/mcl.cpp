@@ -126,6 +126,7 @@ struct mcl_mapper {
   DevBuf key, pair, gms, cand;
   DevBuf flat_keys, flat_done;  // flattened batched kernel: per-epoch key / block count
   DevBuf bnb_next, bnb_inc, bnb_nodes;  // pruned search: subtree counters, incumbents, nodes
+  DevBuf model_buf[9], cost_k, cost_x;  // cost-table construction: staged model, built K / X
   DevBuf in_k, in_x, in_base, in_elig, out_idx, out_ms, out_map;  // staging for host pointers
   uint32_t* flags_host = nullptr;               // host-mapped status word
   uint32_t* flags_dev = nullptr;
@@ -316,8 +317,9 @@ void mcl_mapper_destroy(mcl_mapper_t* h) {
     for (DevBuf* b : {&h->scratch, &h->done, &h->key, &h->pair, &h->gms, &h->cand, &h->flat_keys,
                       &h->flat_done, &h->bnb_next, &h->bnb_inc, &h->bnb_nodes, &h->in_k,
                       &h->in_base, &h->in_elig,
-                      &h->in_x, &h->out_idx, &h->out_ms, &h->out_map})
+                      &h->in_x, &h->out_idx, &h->out_ms, &h->out_map, &h->cost_k, &h->cost_x})
       b->release();
+    for (DevBuf& b : h->model_buf) b.release();
     if (h->flags_host) cudaFreeHost(h->flags_host);
     for (auto& ev : h->ev)
       if (ev) cudaEventDestroy(ev);
@@ -797,6 +799,145 @@ mcl_status_t mcl_map_queues_pruned(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint
   MCL_CUDA(h, cudaStreamSynchronize(s), "D2H");
   h->timing_pending = h->timing > 0;
   return MCL_OK;
+}
+
+}  // extern "C"
+
+namespace {
+
+// Build K and X into device buffers Kd, Xd (each [E][Q][D]); stages host model arrays.
+mcl_status_t build_costs_dev(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                             const mcl_cost_model_t* m, uint64_t* Kd, uint64_t* Xd) {
+  if (!m || !m->kernel_profile || !m->offsets || !m->bytes || !m->source || !m->sizes ||
+      !m->h2d_bw || !m->d2h_bw || (m->num_invocations && !m->kernel_ids) ||
+      m->num_sizes == 0 || m->num_sizes > 64 || m->num_kernels == 0) {
+    h->last_err = "invalid cost model (NULL array, num_sizes outside 1..64 or no kernels)";
+    return MCL_E_INVAL;
+  }
+  const uint64_t EQ = epochs * Q;
+  const uint32_t M = m->num_sizes;
+  struct Arr {
+    const void* src;
+    size_t bytes;
+    DevBuf* buf;
+    const void* dev;
+  } arrs[9] = {
+      {m->kernel_profile, (size_t)m->num_kernels * D * 8, &h->model_buf[0], nullptr},
+      {m->offsets, (size_t)(EQ + 1) * 8, &h->model_buf[1], nullptr},
+      {m->kernel_ids, (size_t)m->num_invocations * 4, &h->model_buf[2], nullptr},
+      {m->bytes, (size_t)EQ * 8, &h->model_buf[3], nullptr},
+      {m->source, (size_t)EQ * 4, &h->model_buf[4], nullptr},
+      {m->cached, (size_t)EQ * 2, &h->model_buf[5], nullptr},
+      {m->sizes, (size_t)M * 8, &h->model_buf[6], nullptr},
+      {m->h2d_bw, (size_t)D * M * 8, &h->model_buf[7], nullptr},
+      {m->d2h_bw, (size_t)D * M * 8, &h->model_buf[8], nullptr},
+  };
+  mcl_status_t st;
+  for (auto& a : arrs) {
+    if (!a.src || a.bytes == 0) continue;
+    bool on = false;
+    if ((st = classify(h, a.src, &on)) != MCL_OK) return st;
+    if ((st = stage_in(h, *a.buf, a.src, a.bytes, on, &a.dev)) != MCL_OK) return st;
+  }
+  mcl::CostArgs c{};
+  c.D = D; c.EQ = EQ; c.num_kernels = m->num_kernels;
+  c.profile = (const uint64_t*)arrs[0].dev; c.offsets = (const uint64_t*)arrs[1].dev;
+  c.ids = (const uint32_t*)arrs[2].dev; c.nnz = m->num_invocations;
+  c.bytes = (const uint64_t*)arrs[3].dev; c.source = (const int32_t*)arrs[4].dev;
+  c.cached = (const uint16_t*)arrs[5].dev; c.M = M; c.sizes = (const uint64_t*)arrs[6].dev;
+  c.h2d = (const double*)arrs[7].dev; c.d2h = (const double*)arrs[8].dev;
+  c.host_shared = m->host_shared; c.K = Kd; c.X = Xd; c.flags = h->flags_dev;
+  MCL_CUDA(h, mcl::launch_build_costs(c, h->num_sms, h->stream), "build_costs launch");
+  return MCL_OK;
+}
+
+mcl_status_t cost_flags(mcl_mapper_t* h) {
+  const uint32_t flags = *(volatile uint32_t*)h->flags_host;
+  if (flags & 32u) {
+    h->last_err = "invalid cost model (kernel id, source, offsets, sizes or bandwidths)";
+    return MCL_E_INVAL;
+  }
+  if (flags & 1u) {
+    h->last_err = "a built cost is >= 2^48";
+    return MCL_E_RANGE;
+  }
+  return MCL_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+mcl_status_t mcl_build_costs(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                             const mcl_cost_model_t* model, uint64_t* cost_kernel,
+                             uint64_t* cost_xfer) {
+  if (!h) return MCL_E_INVAL;
+  h->last_err.clear();
+  if (Q == 0 || D == 0 || Q > MCL_MAX_QUEUES || D > MCL_MAX_DEVICES) {
+    h->last_err = "Q must be in [1, 32] and D in [1, 16]";
+    return MCL_E_INVAL;
+  }
+  if (epochs == 0) return MCL_OK;
+  if (!cost_kernel || !cost_xfer || epochs > (1ull << 40) / ((uint64_t)Q * D)) {
+    h->last_err = "NULL output or too many epochs";
+    return MCL_E_INVAL;
+  }
+  DeviceGuard g(h->device);
+  mcl_status_t st;
+  bool dk, dx;
+  if ((st = classify(h, cost_kernel, &dk)) != MCL_OK) return st;
+  if ((st = classify(h, cost_xfer, &dx)) != MCL_OK) return st;
+  const size_t out_bytes = (size_t)epochs * Q * D * 8;
+  uint64_t* Kd = cost_kernel;
+  uint64_t* Xd = cost_xfer;
+  if (!dk) {
+    MCL_CUDA(h, h->cost_k.ensure(out_bytes), "cudaMalloc(costs)");
+    Kd = (uint64_t*)h->cost_k.p;
+  }
+  if (!dx) {
+    MCL_CUDA(h, h->cost_x.ensure(out_bytes), "cudaMalloc(costs)");
+    Xd = (uint64_t*)h->cost_x.p;
+  }
+  *(volatile uint32_t*)h->flags_host = 0;
+  if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[0], h->stream), "cudaEventRecord");
+  if ((st = build_costs_dev(h, Q, D, epochs, model, Kd, Xd)) != MCL_OK) return st;
+  if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[1], h->stream), "cudaEventRecord");
+  if (!dk) MCL_CUDA(h, cudaMemcpyAsync(cost_kernel, Kd, out_bytes, cudaMemcpyDeviceToHost, h->stream), "D2H");
+  if (!dx) MCL_CUDA(h, cudaMemcpyAsync(cost_xfer, Xd, out_bytes, cudaMemcpyDeviceToHost, h->stream), "D2H");
+  MCL_CUDA(h, cudaStreamSynchronize(h->stream), "build_costs");
+  h->timing_pending = h->timing > 0;
+  return cost_flags(h);
+}
+
+mcl_status_t mcl_map_from_profiles(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                                   const mcl_cost_model_t* model,
+                                   const mcl_constraints_t* constraints,
+                                   uint64_t* mapping_index, uint8_t* mapping, uint64_t* makespan) {
+  if (!h) return MCL_E_INVAL;
+  h->last_err.clear();
+  if (Q == 0 || D == 0 || Q > MCL_MAX_QUEUES || D > MCL_MAX_DEVICES) {
+    h->last_err = "Q must be in [1, 32] and D in [1, 16]";
+    return MCL_E_INVAL;
+  }
+  if (epochs == 0) return MCL_OK;
+  if (epochs > (1ull << 40) / ((uint64_t)Q * D)) {
+    h->last_err = "epochs too large";
+    return MCL_E_INVAL;
+  }
+  DeviceGuard g(h->device);
+  const size_t bytes = (size_t)epochs * Q * D * 8;
+  MCL_CUDA(h, h->cost_k.ensure(bytes), "cudaMalloc(costs)");
+  MCL_CUDA(h, h->cost_x.ensure(bytes), "cudaMalloc(costs)");
+  *(volatile uint32_t*)h->flags_host = 0;
+  mcl_status_t st = build_costs_dev(h, Q, D, epochs, model, (uint64_t*)h->cost_k.p,
+                                    (uint64_t*)h->cost_x.p);
+  if (st != MCL_OK) return st;
+  // the search's own flag checks follow; model errors must be reported first
+  MCL_CUDA(h, cudaStreamSynchronize(h->stream), "build_costs");
+  if ((st = cost_flags(h)) != MCL_OK) return st;
+  return map_impl(h, Q, D, epochs, (const uint64_t*)h->cost_k.p, (const uint64_t*)h->cost_x.p,
+                  constraints ? constraints->base_load : nullptr,
+                  constraints ? constraints->eligible : nullptr, mapping_index, mapping, makespan);
 }
 
 mcl_status_t mcl_score_mappings(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,

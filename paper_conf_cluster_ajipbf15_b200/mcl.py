@@ -28,11 +28,23 @@ EXPORTED = [
     "mcl_device_sms",
     "mcl_comm_unique_id", "mcl_comm_init", "mcl_comm_destroy",
     "mcl_map_queues_constrained", "mcl_score_mappings", "mcl_map_queues_pruned",
+    "mcl_build_costs", "mcl_map_from_profiles",
 ]
 
 
 class mcl_constraints_t(ctypes.Structure):
     _fields_ = [("base_load", ctypes.c_void_p), ("eligible", ctypes.c_void_p)]
+
+
+class mcl_cost_model_t(ctypes.Structure):
+    _fields_ = [
+        ("num_kernels", ctypes.c_uint32), ("kernel_profile", ctypes.c_void_p),
+        ("offsets", ctypes.c_void_p), ("kernel_ids", ctypes.c_void_p),
+        ("num_invocations", ctypes.c_uint64), ("bytes", ctypes.c_void_p),
+        ("source", ctypes.c_void_p), ("cached", ctypes.c_void_p), ("num_sizes", ctypes.c_uint32),
+        ("sizes", ctypes.c_void_p), ("h2d_bw", ctypes.c_void_p), ("d2h_bw", ctypes.c_void_p),
+        ("host_shared", ctypes.c_uint32),
+    ]
 
 
 class mcl_config_t(ctypes.Structure):
@@ -91,6 +103,9 @@ def load_library(path: str | None = None) -> ctypes.CDLL:
                                              ctypes.POINTER(mcl_constraints_t), vp, vp, vp]),
         "mcl_score_mappings": (i32, [vp, u32, u32, u64, vp, vp, vp, vp, vp]),
         "mcl_map_queues_pruned": (i32, [vp, u32, u32, u64, vp, vp,
+                                        ctypes.POINTER(mcl_constraints_t), vp, vp, vp]),
+        "mcl_build_costs": (i32, [vp, u32, u32, u64, ctypes.POINTER(mcl_cost_model_t), vp, vp]),
+        "mcl_map_from_profiles": (i32, [vp, u32, u32, u64, ctypes.POINTER(mcl_cost_model_t),
                                         ctypes.POINTER(mcl_constraints_t), vp, vp, vp]),
     }
     for name, (res, args) in sig.items():
@@ -178,18 +193,23 @@ def mcl_comm_destroy(comm: int | None) -> None:
     load_library().mcl_comm_destroy(comm)
 
 
-def _ptr_and_keepalive(x, dtype):
-    """(pointer, owner) for a torch tensor or numpy array of the given numpy dtype."""
+def _ptr_and_keepalive(x, dtype, convert: bool = False):
+    """(pointer, owner) for a torch tensor or numpy array of the given numpy dtype. With
+    ``convert`` (read-only inputs) a numpy array is first made a contiguous copy of the
+    right dtype; outputs must already match."""
     try:
         import torch
     except ImportError:  # pragma: no cover
         torch = None
     if torch is not None and isinstance(x, torch.Tensor):
-        want = {np.uint64: torch.uint64, np.uint8: torch.uint8, np.uint16: torch.uint16}[dtype]
+        want = {np.uint64: torch.uint64, np.uint8: torch.uint8, np.uint16: torch.uint16,
+                np.uint32: torch.uint32, np.int32: torch.int32, np.float64: torch.float64}[dtype]
         if x.dtype != want or not x.is_contiguous():
             raise TypeError(f"expected a contiguous {want} tensor")
         return x.data_ptr(), x
     a = np.asarray(x)
+    if convert:
+        a = np.ascontiguousarray(a, dtype=dtype)
     if a.dtype != dtype or not a.flags.c_contiguous:
         raise TypeError(f"expected a C-contiguous {np.dtype(dtype)} array")
     return a.ctypes.data, a
@@ -255,6 +275,68 @@ class Mapper:
             ms = np.empty(E, dtype=np.uint64)
             mp = np.empty((E, Q), dtype=np.uint8) if with_mapping else None
         self.map_queues_into(K, X, idx, mp, ms)
+        return idx, mp, ms
+
+    @staticmethod
+    def _cost_model(model: dict, D: int):
+        """mcl_cost_model_t from a dict of arrays (numpy or torch, host or device); returns
+        (struct, keepalive list, E, Q)."""
+        keep = []
+
+        def p(name, dtype, optional=False):
+            v = model.get(name)
+            if v is None:
+                if optional:
+                    return None
+                raise KeyError(name)
+            ptr, owner = _ptr_and_keepalive(v, dtype, convert=True)
+            keep.append(owner)
+            return ptr
+
+        nb = model["bytes"]
+        E, Q = int(nb.shape[0]), int(nb.shape[1])
+        c = mcl_cost_model_t(
+            int(model["profile"].shape[0]), p("profile", np.uint64), p("offsets", np.uint64),
+            p("kernel_ids", np.uint32) if int(model["kernel_ids"].shape[0]) else None,
+            int(model["kernel_ids"].shape[0]), p("bytes", np.uint64), p("source", np.int32),
+            p("cached", np.uint16, optional=True), int(model["sizes"].shape[0]), p("sizes", np.uint64),
+            p("h2d_bw", np.float64), p("d2h_bw", np.float64), int(model.get("host_shared", 0)),
+        )
+        return c, keep, E, Q
+
+    def build_costs(self, model: dict, D: int, device_out: bool = False):
+        """Cost tables K, X [E, Q, D] from a cost model (include/mcl.h mcl_build_costs).
+        Returns numpy arrays, or CUDA tensors when device_out."""
+        c, keep, E, Q = self._cost_model(model, D)
+        if device_out:
+            import torch
+
+            K = torch.empty((E, Q, D), dtype=torch.uint64, device=f"cuda:{self.device}")
+            X = torch.empty_like(K)
+        else:
+            K = np.empty((E, Q, D), np.uint64)
+            X = np.empty((E, Q, D), np.uint64)
+        pk, _k = _ptr_and_keepalive(K, np.uint64)
+        px, _x = _ptr_and_keepalive(X, np.uint64)
+        st = load_library().mcl_build_costs(self.handle, Q, D, E, ctypes.byref(c), pk, px)
+        if st != MCL_OK:
+            raise MclError(st, "mcl_build_costs", mcl_last_error_string(self.handle))
+        return K, X
+
+    def map_from_profiles(self, model: dict, D: int, base=None, eligible=None):
+        """Build the cost tables and search in one call (mcl_map_from_profiles); host
+        (numpy) outputs (index, mapping, makespan)."""
+        c, keep, E, Q = self._cost_model(model, D)
+        pb, _b = _ptr_and_keepalive(base, np.uint64) if base is not None else (None, None)
+        pe, _e = _ptr_and_keepalive(eligible, np.uint16) if eligible is not None else (None, None)
+        cons = mcl_constraints_t(pb, pe)
+        idx = np.empty(E, np.uint64)
+        ms = np.empty(E, np.uint64)
+        mp = np.empty((E, Q), np.uint8)
+        st = load_library().mcl_map_from_profiles(self.handle, Q, D, E, ctypes.byref(c), ctypes.byref(cons),
+                                                  idx.ctypes.data, mp.ctypes.data, ms.ctypes.data)
+        if st != MCL_OK:
+            raise MclError(st, "mcl_map_from_profiles", mcl_last_error_string(self.handle))
         return idx, mp, ms
 
     def map_queues_pruned(self, K, X, base=None, eligible=None, with_mapping: bool = True):

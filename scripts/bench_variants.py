@@ -102,3 +102,23 @@ with Mapper(0) as m:
         print(json.dumps({"measure": "pruned_large", "Q": Q, "D": D, "mappings": D**Q,
                           "pruned_kernel_ms": pr["kernel_ms"], "nodes": m.launch_info()["nodes"],
                           "exhaustive_estimate_ms": D**Q / 1.15e13 * 1e3}), flush=True)
+
+# ---- NEXT-1: cost-table construction (HBM-bound) and the fused pipeline ----
+with Mapper(0) as m:
+    m.set_timing(1)
+    for E, Q, D in ((100_000, 8, 4), (1_000_000, 2, 3)):
+        model = workloads.cost_model(42, E, Q, D)
+        dm = {k: (t(v) if isinstance(v, np.ndarray) else v) for k, v in model.items()}
+        EQ = E * Q
+        nnz = int(model["kernel_ids"].shape[0])
+        alg = 4 * nnz + 8 * (EQ + 1) + 8 * EQ + 4 * EQ + 2 * EQ + 2 * 8 * D * EQ
+        for _ in range(3):
+            m.build_costs(dm, D, device_out=True)
+        ks = []
+        for _ in range(args.reps):
+            m.build_costs(dm, D, device_out=True)
+            ks.append(m.last_kernel_time_ms()[0])
+        k = statistics.median(ks)
+        print(json.dumps({"measure": "build_costs", "E": E, "Q": Q, "D": D, "invocations": nnz,
+                          "kernel_ms": k, "algorithmic_bytes": alg, "GB_per_s": alg / (k / 1e3) / 1e9,
+                          "frac_of_hbm": alg / (k / 1e3) / 1e9 / 6541.8}), flush=True)
