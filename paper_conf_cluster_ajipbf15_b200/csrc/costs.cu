@@ -45,9 +45,10 @@ constexpr int kCostTile = 256;      // (epoch, queue) pairs per CTA tile (= bloc
 constexpr int kIdsCap = 8192;       // kernel ids of a tile staged in shared memory
 constexpr int kProfCapBytes = 32768;  // profile table staged when it fits
 
+template <int D>
 __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  const uint32_t D = a.D, M = a.M;
+  const uint32_t M = a.M;
   const int tid = threadIdx.x;
   // layout: sizes[M] u64 | h2d[D][M] f64 | d2h[D][M] f64 | off[kCostTile+1] u64 |
   //         prof[num_kernels][D] u64 (if it fits) | ids[kIdsCap] u32
@@ -91,9 +92,9 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
     if ((uint32_t)tid < n) {
       const uint64_t eq = t0 + tid;
       // ---- kernel part: sum of the invoked kernels' profile rows ----
-      uint64_t k[kMaxDevices];
+      uint64_t k[D];
 #pragma unroll
-      for (int d = 0; d < kMaxDevices; ++d) k[d] = 0;
+      for (int d = 0; d < D; ++d) k[d] = 0;
       const uint64_t j0 = s_off[tid], j1 = s_off[tid + 1];
       bool ok = j0 <= j1 && j1 <= a.nnz;
       for (uint64_t j = j0; ok && j < j1; ++j) {
@@ -104,8 +105,7 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
         }
         const uint64_t* row = prof + (uint64_t)kid * D;
 #pragma unroll
-        for (int d = 0; d < kMaxDevices; ++d)
-          if (d < (int)D) k[d] += row[d];
+        for (int d = 0; d < D; ++d) k[d] += row[d];
       }
       // ---- transfer part ----
       const uint64_t bytes = a.bytes[eq];
@@ -117,7 +117,13 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
       uint32_t seg = 0;
       double f = 0.0;
       if (ok && !clo && !chi) {
-        while (!(s_sizes[seg] <= bytes && bytes < s_sizes[seg + 1])) ++seg;
+        // binary search for sizes[seg] <= bytes < sizes[seg + 1]
+        uint32_t l = 0, r = M - 1;  // sizes[l] <= bytes < sizes[r]
+        while (r - l > 1) {
+          const uint32_t mid = (l + r) >> 1;
+          if (s_sizes[mid] <= bytes) l = mid; else r = mid;
+        }
+        seg = l;
         f = __ddiv_rn(__ull2double_rn(bytes - s_sizes[seg]),
                       __ull2double_rn(s_sizes[seg + 1] - s_sizes[seg]));
       }
@@ -125,8 +131,7 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
       if (ok && src >= 0 && !((a.host_shared >> src) & 1u))
         down = transfer_ns(bytes, lerp_bw(s_d2h + (size_t)src * M, seg, f, clo, chi, M));
 #pragma unroll
-      for (int d = 0; d < kMaxDevices; ++d) {
-        if (d >= (int)D) break;
+      for (int d = 0; d < D; ++d) {
         uint64_t x = 0;
         if (ok && !(src == d || ((cached >> d) & 1u))) {
           const uint64_t up = ((a.host_shared >> d) & 1u)
@@ -146,19 +151,36 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
   }
 }
 
-cudaError_t launch_build_costs(const CostArgs& a, int num_sms, cudaStream_t st) {
-  size_t smem = (size_t)a.M * 8 + 2 * (size_t)a.D * a.M * 8 + (kCostTile + 1) * 8;
-  if ((size_t)a.num_kernels * a.D * 8 <= (size_t)kProfCapBytes) smem += (size_t)a.num_kernels * a.D * 8;
+namespace {
+template <int D>
+cudaError_t launch_build_costs_t(const CostArgs& a, int num_sms, cudaStream_t st) {
+  size_t smem = (size_t)a.M * 8 + 2 * (size_t)D * a.M * 8 + (kCostTile + 1) * 8;
+  if ((size_t)a.num_kernels * D * 8 <= (size_t)kProfCapBytes) smem += (size_t)a.num_kernels * D * 8;
   smem += (size_t)kIdsCap * 4;
+  auto k = build_costs_kernel<D>;
   static SmemAttrCache cache;
-  cudaError_t err = ensure_smem(build_costs_kernel, smem, cache);
+  cudaError_t err = ensure_smem(k, smem, cache);
   if (err != cudaSuccess) return err;
   uint64_t grid = (a.EQ + kCostTile - 1) / kCostTile;
-  const uint64_t cap = (uint64_t)num_sms * 3;
+  const uint64_t cap = (uint64_t)num_sms * 4;
   if (grid > cap) grid = cap;
   if (grid == 0) grid = 1;
-  build_costs_kernel<<<(unsigned)grid, kCostTile, smem, st>>>(a);
+  k<<<(unsigned)grid, kCostTile, smem, st>>>(a);
   return cudaGetLastError();
+}
+}  // namespace
+
+cudaError_t launch_build_costs(const CostArgs& a, int num_sms, cudaStream_t st) {
+  switch (a.D) {
+#define MCL_COST_CASE(DD) \
+  case DD: return launch_build_costs_t<DD>(a, num_sms, st);
+    MCL_COST_CASE(1) MCL_COST_CASE(2) MCL_COST_CASE(3) MCL_COST_CASE(4)
+    MCL_COST_CASE(5) MCL_COST_CASE(6) MCL_COST_CASE(7) MCL_COST_CASE(8)
+    MCL_COST_CASE(9) MCL_COST_CASE(10) MCL_COST_CASE(11) MCL_COST_CASE(12)
+    MCL_COST_CASE(13) MCL_COST_CASE(14) MCL_COST_CASE(15) MCL_COST_CASE(16)
+#undef MCL_COST_CASE
+    default: return cudaErrorInvalidValue;
+  }
 }
 
 }  // namespace mcl
