@@ -4,6 +4,7 @@
 #include <atomic>
 #include <cstddef>
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 namespace mcl {
@@ -44,6 +45,14 @@ cudaError_t ensure_smem(F* kernel, size_t smem, SmemAttrCache& cache) {
   cudaError_t err = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (err == cudaSuccess) g.store(smem + 1, std::memory_order_relaxed);
   return err;
+}
+
+// Integer tuning knob from the environment (read once by the caller), clamped to [lo, hi].
+inline int env_int(const char* name, int dflt, int lo, int hi) {
+  const char* v = getenv(name);
+  if (!v || !*v) return dflt;
+  const int x = atoi(v);
+  return x < lo ? lo : (x > hi ? hi : x);
 }
 
 // Register-blocked search (search_blocked.cu).

@@ -4,8 +4,8 @@
 // The work per epoch is a handful of integer ops; the kernel is bound by HBM (96 B of
 // costs in, 18 B of results out per epoch at Q=2, D=3). A persistent grid streams tiles of
 // blockDim.x epochs: one elected thread moves a tile's K and X slabs global -> shared with
-// cp.async.bulk (the TMA bulk-copy engine, SASS UBLKCP) completing on an mbarrier, six
-// stages deep so several tiles are in flight while the current one is scored. Each thread then
+// cp.async.bulk (the TMA bulk-copy engine, SASS UBLKCP) completing on mbarriers, several
+// stages deep so tiles are in flight while the current one is scored. Each thread then
 // scores its epoch's D^Q mappings from shared memory with compile-time digits (so every
 // load index is static), in increasing index order with a strict '<' (lowest index wins
 // ties, BASELINE.json north_star), and writes its outputs coalesced.
@@ -65,15 +65,15 @@ struct Pow<0, D> {
 
 }  // namespace
 
-constexpr int kSmallStages = 6;  // tiles in flight per CTA (TMA bulk copies)
+constexpr int kMaxSmallStages = 16;  // tiles in flight per CTA (TMA bulk copies), upper bound
 
 template <int Q, int D>
-__global__ void __launch_bounds__(128) search_small_kernel(SmallArgs a, int use_tma) {
+__global__ void __launch_bounds__(256) search_small_kernel(SmallArgs a, int use_tma, int kSmallStages) {
   constexpr int QD = Q * D;
   constexpr int N = Pow<Q, D>::N;
   constexpr bool kVec = (QD % 2) == 0;  // a row of QD u64 is a whole number of 16-B vectors
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  __shared__ __align__(8) uint64_t full[kSmallStages];
+  __shared__ __align__(8) uint64_t full[kMaxSmallStages];
   const int TE = blockDim.x, tid = threadIdx.x;
   const size_t slab = (size_t)TE * QD;  // u64 per array per stage
   uint64_t* sbase = reinterpret_cast<uint64_t*>(smem_raw);
@@ -193,31 +193,38 @@ namespace {
 template <int Q, int D>
 cudaError_t launch_small_t(const SmallArgs& a, int num_sms, cudaStream_t st, int* grid_out,
                            int* threads_out) {
-  // tile = one epoch per thread; tiny batches (cfg1: one epoch) get a single warp
-  const int threads = a.E >= 128 ? 128 : (int)((a.E + 31) / 32 * 32);
-  const size_t smem = (size_t)kSmallStages * 2 * threads * Q * D * 8;
+  // tile = one epoch per thread; tiny batches (cfg1: one epoch) get a single warp.
+  // Defaults from the cfg3 sweep (scripts/sweep_small.sh, profiles/r01/sweep_small.txt):
+  // 128-epoch tiles, 2 stages, 4 CTAs per SM (8 tiles in flight per SM) was fastest;
+  // MCL_SMALL_{THREADS,STAGES,CTAS_PER_SM} override them for tuning.
+  static const int kThreads = env_int("MCL_SMALL_THREADS", 128, 32, 256);
+  static const int kStages = env_int("MCL_SMALL_STAGES", 2, 1, kMaxSmallStages);
+  static const int kCtasCap = env_int("MCL_SMALL_CTAS_PER_SM", 4, 1, 32);
+  const int threads = a.E >= (uint64_t)kThreads ? kThreads : (int)((a.E + 31) / 32 * 32);
+  const size_t smem = (size_t)kStages * 2 * threads * Q * D * 8;
   auto k = search_small_kernel<Q, D>;
   static SmemAttrCache cache;
   cudaError_t err = ensure_smem(k, smem, cache);
   if (err != cudaSuccess) return err;
-  static std::atomic<int> occ128[64];  // CTAs per SM at 128 threads, per device (0 = unknown)
+  static std::atomic<int> occ_full[64];  // CTAs per SM at full tiles, per device (0 = unknown)
   int dev = 0;
   cudaGetDevice(&dev);
   int per_sm = 1;
-  if (threads == 128) {
-    per_sm = occ128[dev & 63].load(std::memory_order_relaxed);
+  if (threads == kThreads) {
+    per_sm = occ_full[dev & 63].load(std::memory_order_relaxed);
     if (per_sm == 0) {
       err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, threads, smem);
       if (err != cudaSuccess) return err;
       if (per_sm < 1) per_sm = 1;
-      occ128[dev & 63].store(per_sm, std::memory_order_relaxed);
+      occ_full[dev & 63].store(per_sm, std::memory_order_relaxed);
     }
+    if (per_sm > kCtasCap) per_sm = kCtasCap;
   }
   const uint64_t ntiles = (a.E + threads - 1) / threads;
   uint64_t grid = (uint64_t)num_sms * per_sm;
   if (grid > ntiles) grid = ntiles;
   const int use_tma = ((reinterpret_cast<uintptr_t>(a.K) | reinterpret_cast<uintptr_t>(a.X)) & 15) == 0;
-  k<<<(unsigned)grid, threads, smem, st>>>(a, use_tma);
+  k<<<(unsigned)grid, threads, smem, st>>>(a, use_tma, kStages);
   *grid_out = (int)grid;
   *threads_out = threads;
   return cudaGetLastError();
