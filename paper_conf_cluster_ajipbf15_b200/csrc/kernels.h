@@ -62,7 +62,9 @@ struct BlockedArgs {
   const uint64_t* K;
   const uint64_t* X;
   uint64_t rlo, rhi;  // this rank's block range [rlo, rhi), blocks of D^3 mappings
-  Cand* scratch;      // [E][cpe]
+  uint64_t e_full;    // epochs 0..e_full-1 get one CTA each
+  uint32_t tail_cpe;  // CTAs of each remaining epoch (1-D grid over the CTA index space)
+  Cand* scratch;      // [E - e_full][tail_cpe] (split epochs only)
   uint32_t* done;     // [E], zero on entry, self-resetting
   EpochOut out;
   int ibits;

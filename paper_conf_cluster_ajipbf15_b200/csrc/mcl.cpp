@@ -547,10 +547,32 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
       a.out = out; a.ibits = ibits; a.flags = h->flags_dev; a.one = 1;
       a.base = Bd; a.elig = Ed;
       const size_t smem = mcl::blocked_smem_bytes(Q, D, wide, threads, &a.off_red, &a.off_dig);
-      int occ = mcl::blocked_ctas_per_sm(D, wide, threads, smem);
-      size_grid(h, epochs, hi - lo, occ, threads, &grid);
-      if (grid.x > 1) {
-        MCL_CUDA(h, h->scratch.ensure((size_t)epochs * grid.x * sizeof(Cand)), "cudaMalloc(scratch)");
+      const int occ = mcl::blocked_ctas_per_sm(D, wide, threads, smem);
+      // Work layout (1-D grid): whole waves of epochs get one CTA each; the epochs of the
+      // last, partial wave are split over several CTAs so that wave is filled; a batch
+      // smaller than one wave spreads every epoch over the resident CTAs.
+      const uint64_t slots = (uint64_t)h->num_sms * std::max(1, occ);
+      const uint64_t units = hi - lo;
+      const uint64_t chunk = (D <= 5 && Q >= 5 && !wide) ? (uint64_t)D * D : 1;
+      uint64_t e_full = 0, tail_cpe = 1;
+      if (epochs >= slots) {
+        e_full = epochs / slots * slots;
+        const uint64_t rem = epochs - e_full;
+        // split only as far as every thread keeps at least one chunk
+        const uint64_t max_cpe = std::max<uint64_t>(1, units / ((uint64_t)threads * chunk));
+        tail_cpe = rem ? std::max<uint64_t>(1, std::min(slots / rem, max_cpe)) : 1;
+      } else {
+        tail_cpe = (slots + epochs - 1) / epochs;
+        tail_cpe = std::min<uint64_t>(tail_cpe, std::max<uint64_t>(1, (units + threads - 1) / threads));
+      }
+      tail_cpe = std::min<uint64_t>(tail_cpe, 65535);
+      a.e_full = e_full;
+      a.tail_cpe = (uint32_t)tail_cpe;
+      const uint64_t ncta = e_full + (epochs - e_full) * tail_cpe;
+      grid = dim3((unsigned)std::min<uint64_t>(ncta, 0x7fffffffu), 1, 1);
+      if (tail_cpe > 1) {
+        MCL_CUDA(h, h->scratch.ensure((size_t)(epochs - e_full) * tail_cpe * sizeof(Cand)),
+                 "cudaMalloc(scratch)");
         a.scratch = (Cand*)h->scratch.p;
       }
       a.done = (uint32_t*)h->done.p;

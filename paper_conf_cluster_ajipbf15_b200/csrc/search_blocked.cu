@@ -28,7 +28,10 @@
 namespace mcl {
 
 
-// Kernel: gridDim.x = CTAs per epoch (cpe), gridDim.y = epochs handled concurrently.
+// Kernel work layout over a 1-D grid of CTAs: the first e_full epochs get one CTA each; the
+// remaining E - e_full epochs (the "tail") get tail_cpe CTAs each, so the last wave of a
+// batch runs split epochs instead of idling (wave quantisation), and a single large epoch
+// (e_full = 0) spreads over every CTA. The grid strides over this CTA index space.
 template <typename T, int D>
 __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
     search_blocked_kernel(BlockedArgs a) {
@@ -53,7 +56,20 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
   __shared__ __align__(16) T base0[D];  // base loads in the search's arithmetic type
   constexpr bool kSuper = (sizeof(T) == 4 && D <= kSuperMaxD);
 
-  for (uint64_t e = blockIdx.y; e < a.E; e += gridDim.y) {
+  const uint64_t ncta = a.e_full + (a.E - a.e_full) * a.tail_cpe;
+  for (uint64_t cta = blockIdx.x; cta < ncta; cta += gridDim.x) {
+    uint64_t e;
+    uint32_t part, parts;
+    if (cta < a.e_full) {
+      e = cta;
+      part = 0;
+      parts = 1;
+    } else {
+      const uint64_t t = cta - a.e_full;
+      e = a.e_full + t / a.tail_cpe;
+      part = (uint32_t)(t % a.tail_cpe);
+      parts = a.tail_cpe;
+    }
     // ---- a1: cost composition C = K + X, range check, bound UB = sum_q max_d C ----
     __syncthreads();  // the previous epoch's tables are no longer read
     if (tid == 0) { s_status = 0; s_ub = 0; }
@@ -74,11 +90,11 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
     }
     __syncthreads();
     if (s_status) {
-      if (tid == 0 && blockIdx.x == 0) raise_flag(a.flags, s_status);
+      if (tid == 0 && part == 0) raise_flag(a.flags, s_status);
       continue;
     }
     if (sizeof(T) == 4 && s_ub >= (1ull << 32)) {
-      if (tid == 0 && blockIdx.x == 0) raise_flag(a.flags, kFlagNeedU64);
+      if (tid == 0 && part == 0) raise_flag(a.flags, kFlagNeedU64);
       continue;
     }
     // ---- tables: inner sums and one-hot outer vectors ----
@@ -104,8 +120,8 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
     // Split points are aligned to whole CHUNKS (D^2 blocks on the super-block path) so the
     // lanes of a warp walk chunks in lock-step; only the rank's two ends can be ragged.
     const uint64_t nb_rank = a.rhi - a.rlo;
-    const uint64_t T_all = (uint64_t)gridDim.x * nthr;
-    const uint64_t gt = (uint64_t)blockIdx.x * nthr + tid;
+    const uint64_t T_all = (uint64_t)parts * nthr;
+    const uint64_t gt = (uint64_t)part * nthr + tid;
     const bool chunked = kSuper && O >= 2;
     const uint64_t chunk = chunked ? (uint64_t)D * D : 1;
     auto split = [&](uint64_t t) -> uint64_t {
@@ -162,24 +178,25 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
       __syncthreads();
     }
     Cand c = s_cand;
-    if (gridDim.x == 1) {
+    if (parts == 1) {
       if (tid == 0) write_epoch(a.out, e, Q, D, a.ibits, c, a.flags, s_feas);
       continue;
     }
+    // a split epoch: per-CTA candidates in scratch; the last CTA to finish reduces them
     __shared__ bool s_last;
+    Cand* slots = a.scratch + (e - a.e_full) * parts;
     if (tid == 0) {
-      a.scratch[e * gridDim.x + blockIdx.x] = c;
+      slots[part] = c;
       __threadfence();
       const uint32_t prev = atomicAdd(&a.done[e], 1u);
-      s_last = (prev == gridDim.x - 1);
+      s_last = (prev == parts - 1);
     }
     __syncthreads();
     if (s_last) {
       __threadfence();
       Cand r{kNone, kNone};
-      for (uint32_t t = tid; t < gridDim.x; t += nthr) {
-        const volatile uint64_t* o =
-            reinterpret_cast<const volatile uint64_t*>(&a.scratch[e * gridDim.x + t]);
+      for (uint32_t t = tid; t < parts; t += nthr) {
+        const volatile uint64_t* o = reinterpret_cast<const volatile uint64_t*>(&slots[t]);
         r = cand_min(r, Cand{o[0], o[1]});
       }
       r = block_min(r, red);
