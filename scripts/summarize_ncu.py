@@ -77,8 +77,11 @@ def main(tag, workloads):
             rd = to_bytes(*d["dram__bytes_read.sum"])
             wr = to_bytes(*d["dram__bytes_write.sum"])
             wi = float(d["smsp__inst_executed.sum"][0].replace(",", ""))
-            lines += ["", f"thread instructions per mapping (warp instructions x 32 / mappings): "
-                          f"{wi * 32 / MAPPINGS[wl]:.3f}", ""]
+            if wl in MAPPINGS:
+                lines += ["", f"thread instructions per mapping (warp instructions x 32 / mappings): "
+                              f"{wi * 32 / MAPPINGS[wl]:.3f}", ""]
+            else:
+                lines += [""]
             traffic[wl] = {"dram_bytes_per_launch": rd + wr, "kernel": d["kernel"], "source": f"profiles/{tag}"}
         lp = os.path.join(ROOT, "gpurun_out", f"launches_{wl}.csv")
         if os.path.exists(lp):
@@ -89,4 +92,4 @@ def main(tag, workloads):
 
 
 if __name__ == "__main__":
-    main(sys.argv[1], sys.argv[2:] or ["cfg5", "cfg4", "cfg2", "cfg3"])
+    main(sys.argv[1], sys.argv[2:] or ["cfg5", "cfg4", "cfg2", "cfg3", "costs"])
