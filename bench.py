@@ -9,8 +9,10 @@ enumeration, per-device loads, makespan, argmin with lowest-index ties, the cros
 all-reduce when N > 1, and the output decode) on one synthetic workload already resident in
 HBM. Default workload: cfg5 = 12 queues x 8 devices (8^12 = 6.9e10 mappings, one epoch),
 the largest single-GPU configuration and the one BASELINE.json's scaling target names;
-at N GPUs its index space is sharded by contiguous ranges (strong scaling) and combined by
-one ncclAllReduce(MIN) over the packed (makespan, index) key.
+at N GPUs its index space is sharded by contiguous ranges (strong scaling) and the ranks'
+packed (makespan, index) keys are combined INSIDE the search kernel over NVLink peer memory
+(the fused exchange, include/mcl.h mcl_peer_import; `--collective nccl` uses
+ncclAllReduce(MIN) + a decode kernel instead).
 
 Rank 0 prints one JSON line. `value` is whole-job mappings/s from CUDA events over exactly
 K timed steps (L2 flushed between steps, outside the events), max over ranks; `e2e` is the
@@ -53,8 +55,10 @@ def parse():
     p.add_argument("--impl", default="mcl", choices=["mcl", "reference"])
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="CPU-oracle sample budget")
-    p.add_argument("--collective", action="store_true",
-                   help="use the NCCL all-reduce path even with one rank (exercises the N>1 code)")
+    p.add_argument("--collective", default="auto", choices=["auto", "fused", "nccl"],
+                   help="cross-GPU combine of a sharded single-epoch search: fused = in-kernel "
+                        "exchange over peer memory (NEXT-2), nccl = ncclAllReduce + decode kernel; "
+                        "auto = fused when N > 1. An explicit choice also runs it with one rank.")
     return p.parse_args()
 
 
@@ -217,12 +221,14 @@ def main():
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    if world > 1 or args.collective:
+    explicit = args.collective != "auto"
+    if world > 1 or explicit:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         os.environ.setdefault("MASTER_PORT", "29531")
         dist.init_process_group("nccl", device_id=dev, rank=rank, world_size=world)
+    sharded = (world > 1 or explicit) and not is_batched(w)
     comm = None
-    if (world > 1 or args.collective) and not is_batched(w):
+    if sharded:  # the NCCL communicator: the nccl path, and the fallback of the fused one
         obj = [mcl.mcl_comm_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         comm = mcl.mcl_comm_init(local, world, rank, obj[0])
@@ -241,6 +247,23 @@ def main():
     flush = torch.empty(L2_FLUSH_BYTES, dtype=torch.uint8, device=dev)
     mapper = Mapper(local, stream=stream.cuda_stream, nccl_comm=comm, rank=rank if comm else 0,
                     world=world if comm else 1)
+    combine = "nccl" if comm else "none"
+    if sharded and args.collective != "nccl":
+        # fused in-kernel exchange over NVLink peer memory; NCCL stays as the fallback if the
+        # slabs cannot be mapped (the choice is agreed by all ranks)
+        try:
+            mapper.connect_peers(max_epochs=max(1, w["E"]), timeout_ms=60_000)
+            ok = 1
+        except Exception as exc:  # pragma: no cover
+            print(f"[bench] fused exchange unavailable ({exc}); using NCCL", file=sys.stderr)
+            ok = 0
+        t_ok = torch.tensor([ok], dtype=torch.int32, device=dev)
+        dist.all_reduce(t_ok, op=dist.ReduceOp.MIN)
+        if int(t_ok[0]):
+            combine = "fused"
+        elif ok:  # another rank failed: drop the slabs everywhere
+            mapper.close()
+            mapper = Mapper(local, stream=stream.cuda_stream, nccl_comm=comm, rank=rank, world=world)
     mapper.set_timing(True)
 
     for _ in range(max(3, args.warmup)):
@@ -340,8 +363,11 @@ def main():
             "data": "synthetic",
             "config": {"workload": args.workload, "desc": w["desc"], "Q": Q, "D": w["D"],
                        "epochs": w["E"], "mappings_per_step": mappings_per_step,
-                       "parallelism": f"index-range shard x{world} + ncclAllReduce(min)" if (world > 1 and not is_batched(w))
+                       "parallelism": (f"index-range shard x{world} + " + (
+                           "in-kernel peer exchange (fused atomicMin over NVLink)" if combine == "fused"
+                           else "ncclAllReduce(min)")) if sharded
                        else (f"epoch replicas x{world}" if world > 1 else "1 GPU"),
+                       "combine": combine,
                        "l2": "flushed between timed steps (256 MiB write, outside the events)",
                        "path": info["path"], "ctas": info["ctas"], "threads": info["threads"],
                        "result": {"index": int(idx[0]), "makespan": int(msp[0])}},

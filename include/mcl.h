@@ -99,6 +99,35 @@ mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t ep
                             uint64_t* mapping_index, uint8_t* mapping, uint64_t* makespan);
 
 /*
+ * Fused cross-GPU exchange (no paper counterpart -- the paper's mapper is
+ * single-host). Replaces the NCCL all-reduce of a sharded handle by an
+ * exchange INSIDE the search kernel over NVLink / NVSwitch peer memory: each rank owns an
+ * exchange slab in its device memory, exported as a CUDA IPC handle and mapped by every
+ * other rank. When the rank's search is done, the kernel's last CTA adds its packed keys to
+ * every rank's slab with system-scope atomicMin, signals every rank, waits for all `world`
+ * signals and decodes the global result: one launch per call, no collective library, no
+ * extra kernel. The result is the same as the NCCL path's (including the two-step
+ * lexicographic reduction when a makespan does not fit beside the index).
+ * Setup, collective over the handle's `world` ranks (cfg->rank / cfg->world), once:
+ *   1. every rank: mcl_peer_export(h, max_epochs, handle_out) -> 64 opaque bytes
+ *      (allocates the slab: 2 * max_epochs + 8 words, max_epochs in [1, 2^20]);
+ *   2. the ranks exchange the bytes out of band (e.g. torch.distributed all_gather);
+ *   3. every rank: mcl_peer_import(h, handles, timeout_ms), handles = [world][64] bytes
+ *      in rank order (a rank's own entry is not opened; world == 1 exchanges with itself).
+ * Afterwards every mcl_map_queues / mcl_map_queues_constrained call on h with
+ * epochs <= max_epochs is COLLECTIVE through the slabs: all ranks must make the same calls,
+ * in the same order, with identical inputs. A communicator, if the handle has one, still
+ * serves larger calls. If some rank does not signal within timeout_ms (0 = 30 s), the call
+ * fails with MCL_E_NCCL ("peer exchange timed out") instead of hanging, and the handle's
+ * exchange is disabled. Destroy the handles of all ranks together (a rank's slab stays
+ * mapped by its peers until they destroy theirs).
+ * Errors: MCL_E_INVAL (bad arguments, world handles not matching, import before export),
+ *         MCL_E_CUDA (IPC export/open failed, e.g. no peer access between the devices).
+ */
+mcl_status_t mcl_peer_export(mcl_mapper_t* h, uint64_t max_epochs, uint8_t handle_out[64]);
+mcl_status_t mcl_peer_import(mcl_mapper_t* h, const uint8_t* handles, uint32_t timeout_ms);
+
+/*
  * Constrained variant. The paper's runtime maps only the SCHED_AUTO queues
  * of the pool; queues created with SCHED_OFF "will be statically mapped to the chosen
  * device" and still occupy it. Here:
@@ -223,8 +252,9 @@ const char* mcl_last_error_string(const mcl_mapper_t* h);
  *             search, 3 = generic search, 4 = small batched (thread per epoch),
  *             5 = register-blocked u32 over a flattened (epoch, block) space)
  *   info[1] = number of kernels launched by the call, info[2] = CTAs of the main kernel,
- *   info[3] = threads per CTA, info[4] = 1 if an NCCL all-reduce ran,
- *   info[5] = index bits of the packed key, info[6] = 1 if the two-step reduce ran.
+ *   info[3] = threads per CTA, info[4] = 1 if an NCCL all-reduce ran, 2 if the fused peer
+ *   exchange ran, info[5] = index bits of the packed key, info[6] = 1 if the two-step
+ *   reduce ran.
  */
 mcl_status_t mcl_last_launch_info(const mcl_mapper_t* h, int64_t info[8]);
 

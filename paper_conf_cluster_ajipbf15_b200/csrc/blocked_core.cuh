@@ -136,19 +136,6 @@ __device__ __forceinline__ T block_eval(const T (&P)[D], const T* __restrict__ i
   return block_eval<T, D>(s, max_of<T, D>(P));
 }
 
-// Lowest leaf of the block whose makespan equals `target` (the block is known to hold one).
-template <typename T, int D>
-__device__ __forceinline__ uint32_t block_first(const T (&P)[D], const T* __restrict__ in,
-                                                uint32_t one, T target) {
-  Sums<T, D> s;
-  make_sums<T, D>(s, P, in, one);
-  uint32_t first = 0xffffffffu;
-  for_each_leaf<T, D>(s, max_of<T, D>(P), [&](int leaf, T v) {
-    first = (v == target && first == 0xffffffffu) ? (uint32_t)leaf : first;
-  });
-  return first;
-}
-
 // A SUPER-BLOCK: the D blocks x = 0..D-1 of the fourth-innermost digit (queue Q-4) with
 // the same outer prefix `base`. Only device x's load changes between them, so the sums of
 // the other devices are shared and the block loop is unrolled with static x (used for
@@ -181,7 +168,8 @@ __device__ __forceinline__ void load_vec(T (&v)[D], const T* __restrict__ src) {
   for (int d = 0; d < D; ++d) v[d] = src[d];
 }
 
-// Warp-cooperative form of block_first, called by all 32 lanes with the same (P, target):
+// Lowest leaf of a block whose makespan equals `target` (the block is known to hold one),
+// found cooperatively: called by all 32 lanes with the same (P, target),
 // lane l evaluates leaves l, l + 32, ... directly from the definition (runtime digits
 // i, j, k; loads P[d] plus the inner queues' costs on their devices; max over devices) and
 // a ballot per round finds the lowest leaf equal to `target`. Replaces a serial re-scan of

@@ -17,16 +17,6 @@ constexpr int kMaxDevices = 16;                // D <= 16 (include/mcl.h)
 constexpr int kMaxQueues = 32;                 // Q <= 32
 constexpr uint64_t kEntryLimit = 1ull << 48;   // entries must be < 2^48 (reading R10)
 
-// Status bits written by kernels into the handle's host-mapped status word.
-enum : uint32_t {
-  kFlagRange = 1u,     // some cost entry >= 2^48
-  kFlagNeedU64 = 2u,   // some epoch's bound sum_q max_d C >= 2^32: rerun with 64-bit loads
-  kFlagNoPack = 4u,    // makespan does not fit beside the index in one u64 key (NCCL path)
-  kFlagInfeasible = 8u,  // constrained call: some queue has no eligible device below D
-  kFlagBadMapping = 16u, // scoring call: a mapping names a device >= D
-  kFlagBadModel = 32u,   // cost model: bad kernel id / source / offsets / curve
-};
-
 __device__ __forceinline__ bool cand_less(const Cand& a, const Cand& b) {
   return a.ms < b.ms || (a.ms == b.ms && a.idx < b.idx);
 }
@@ -65,13 +55,6 @@ __device__ __forceinline__ Cand block_min(Cand c, Cand* red) {
 
 __device__ __forceinline__ void raise_flag(volatile uint32_t* flags, uint32_t bit) {
   if (flags) atomicOr((uint32_t*)flags, bit);
-}
-
-// Bits needed to hold every index of an N-mapping space (N >= 1): ceil(log2(N)).
-__host__ __device__ __forceinline__ int index_bits(uint64_t N) {
-  int b = 0;
-  while (b < 64 && (N - 1) >> b) ++b;
-  return b;
 }
 
 // Epoch prologue, run by ONE WARP after C64[Q][D] = K + X is in shared memory (a1):
@@ -138,6 +121,22 @@ __device__ __forceinline__ uint64_t epoch_prologue(uint64_t* C64, uint32_t Q, ui
   return row + bmax;
 }
 
+// Public outputs of epoch e: index, makespan and (optionally) the index's base-D digits,
+// queue 0 most significant (reading R2); 0xFF bytes for "no mapping" (kNone).
+__device__ __forceinline__ void write_result(uint64_t* index, uint64_t* makespan, uint8_t* mapping,
+                                             uint64_t e, uint32_t Q, uint32_t D, uint64_t idx,
+                                             uint64_t ms) {
+  index[e] = idx;
+  makespan[e] = ms;
+  if (mapping) {
+    uint64_t rest = idx;
+    for (int q = (int)Q - 1; q >= 0; --q) {
+      mapping[e * Q + (uint64_t)q] = (idx == kNone) ? 0xFF : (uint8_t)(rest % D);
+      rest /= D;
+    }
+  }
+}
+
 // `feasible`: candidates above it are infeasible (constrained sub-range searches) and are
 // reported as (kNone, kNone); kNone when unconstrained.
 __device__ __forceinline__ void write_epoch(const EpochOut& o, uint64_t e, uint32_t Q, uint32_t D,
@@ -145,10 +144,13 @@ __device__ __forceinline__ void write_epoch(const EpochOut& o, uint64_t e, uint3
                                             uint64_t feasible = kNone) {
   if (c.ms != kNone && c.ms > feasible) c = Cand{kNone, kNone};
   if (o.key) {
-    // multi-GPU: publish the packed key; outputs are decoded after the all-reduce
+    // multi-GPU: publish the packed key; outputs are decoded after the all-reduce. A
+    // makespan that does not fit beside the index publishes kNone: it is larger than every
+    // key that fits, so it can only be the global minimum if no rank's candidate fits --
+    // which the decode step detects on the REDUCED key (identical on every rank, so every
+    // rank takes the same two-step decision; a local flag could differ between ranks).
     const bool none = (c.ms == kNone);
     const bool fits = none || (ibits == 0) || (c.ms < (1ull << (64 - ibits)));
-    if (!fits) raise_flag(flags, kFlagNoPack);
     o.key[e] = (fits && !none) ? ((ibits == 0 ? 0ull : (c.ms << ibits)) | c.idx) : kNone;
     if (o.pair) {
       o.pair[2 * e] = c.ms;
@@ -156,15 +158,7 @@ __device__ __forceinline__ void write_epoch(const EpochOut& o, uint64_t e, uint3
     }
     return;
   }
-  o.index[e] = c.idx;
-  o.makespan[e] = c.ms;
-  if (o.mapping) {
-    uint64_t rest = c.idx;
-    for (int q = (int)Q - 1; q >= 0; --q) {
-      o.mapping[e * Q + (uint64_t)q] = (c.idx == kNone) ? 0xFF : (uint8_t)(rest % D);
-      rest /= D;
-    }
-  }
+  write_result(o.index, o.makespan, o.mapping, e, Q, D, c.idx, c.ms);
 }
 
 }  // namespace mcl

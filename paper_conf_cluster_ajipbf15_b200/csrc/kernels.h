@@ -9,6 +9,34 @@
 
 namespace mcl {
 
+// Status bits written by kernels into the handle's host-mapped status word; mcl.cpp turns
+// them into an mcl_status_t after the stream sync.
+enum : uint32_t {
+  kFlagRange = 1u,       // some cost entry or base load >= 2^48
+  kFlagNeedU64 = 2u,     // some epoch's bound sum_q max_d C >= 2^32: rerun with 64-bit loads
+  kFlagNoPack = 4u,      // makespan does not fit beside the index in one u64 key (NCCL path)
+  kFlagInfeasible = 8u,  // constrained call: some queue has no eligible device below D
+  kFlagBadMapping = 16u, // scoring call: a mapping names a device >= D
+  kFlagBadModel = 32u,   // cost model: bad kernel id / source / offsets / curve
+  kFlagPeerTimeout = 64u,  // fused exchange: some rank did not signal in time
+  kFlagTwoStep = 128u,     // fused exchange ran the two-step reduction (informational)
+};
+
+// Fused cross-GPU exchange (peer.cuh). Slab of each rank, in u64 words:
+// [0] signal counter (every rank adds 1 per round), [1] rounds completed, [2] capacity (cap),
+// [3, 8) unused,
+// [8, 8 + cap) region 0, [8 + cap, 8 + 2 cap) region 1 (round R uses region R % 2).
+constexpr uint64_t kPeerHeaderWords = 8;
+struct PeerArgs {
+  int world;               // 0 = exchange off
+  uint64_t* const* slabs;  // [world] every rank's slab, mapped into this process (device array)
+  uint64_t* mine;          // this rank's slab
+  uint64_t cap;            // epochs per region
+  uint32_t* kdone;         // CTAs of the kernel that finished; zero on entry, self-resetting
+  uint64_t* gms;           // [cap] scratch: global makespans of the two-step reduction
+  uint64_t timeout_ns;
+};
+
 // Lexicographic (makespan, mapping index) candidate; see common.cuh.
 struct Cand {
   uint64_t ms;
@@ -73,6 +101,7 @@ struct BlockedArgs {
   size_t off_red, off_dig;
   const uint64_t* base;  // [E][D] pre-existing device loads, or nullptr (constrained variant)
   const uint16_t* elig;  // [E][Q] eligible-device masks (0 = any), or nullptr
+  PeerArgs peer;         // fused cross-GPU exchange (out.key / out.pair set), or world = 0
 };
 
 // ceil(log2(N)): bits of the packed key's index field (N >= 1).
@@ -122,6 +151,7 @@ struct GenericArgs {
   volatile uint32_t* flags;
   const uint64_t* base;  // [E][D] or nullptr (constrained variant)
   const uint16_t* elig;  // [E][Q] or nullptr
+  PeerArgs peer;         // as BlockedArgs::peer
 };
 size_t generic_smem_bytes(uint32_t Q, uint32_t D, int threads);
 
@@ -196,7 +226,7 @@ cudaError_t launch_small(const SmallArgs& a, int num_sms, cudaStream_t st, int* 
 // Multi-GPU epilogues (reduce.cu).
 cudaError_t launch_decode_key(const uint64_t* key, uint64_t E, uint32_t Q, uint32_t D, int ibits,
                               uint64_t* index, uint64_t* makespan, uint8_t* mapping,
-                              cudaStream_t st);
+                              volatile uint32_t* flags, cudaStream_t st);
 cudaError_t launch_pair_candidates(const uint64_t* pair, const uint64_t* gms, uint64_t E,
                                    uint64_t* cand, cudaStream_t st);
 cudaError_t launch_decode_pair(const uint64_t* gms, const uint64_t* gidx, uint64_t E, uint32_t Q,

@@ -15,6 +15,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <string>
+#include <vector>
 
 #include <cuda_runtime.h>
 #include <nccl.h>
@@ -128,6 +129,13 @@ struct mcl_mapper {
   DevBuf bnb_next, bnb_inc, bnb_nodes;  // pruned search: subtree counters, incumbents, nodes
   DevBuf model_buf[9], cost_k, cost_x;  // cost-table construction: staged model, built K / X
   DevBuf in_k, in_x, in_base, in_elig, out_idx, out_ms, out_map;  // staging for host pointers
+  // fused peer exchange (NEXT-2): own slab, kernel CTA counter, two-step scratch, and the
+  // device array of every rank's slab address (peers' slabs opened through CUDA IPC)
+  DevBuf peer_slab, peer_kdone, peer_gms, peer_ptrs;
+  std::vector<void*> peer_opened;
+  uint64_t peer_cap = 0;
+  uint64_t peer_timeout_ns = 0;
+  bool peer_ready = false;
   uint32_t* flags_host = nullptr;               // host-mapped status word
   uint32_t* flags_dev = nullptr;
   int timing = 0;               // 0 off, 1 search kernel, 2 search kernel + whole call
@@ -314,6 +322,8 @@ void mcl_mapper_destroy(mcl_mapper_t* h) {
   {
     DeviceGuard g(h->device);
     if (h->stream) cudaStreamSynchronize(h->stream);
+    for (void* p : h->peer_opened) cudaIpcCloseMemHandle(p);
+    for (DevBuf* b : {&h->peer_slab, &h->peer_kdone, &h->peer_gms, &h->peer_ptrs}) b->release();
     for (DevBuf* b : {&h->scratch, &h->done, &h->key, &h->pair, &h->gms, &h->cand, &h->flat_keys,
                       &h->flat_done, &h->bnb_next, &h->bnb_inc, &h->bnb_nodes, &h->in_k,
                       &h->in_base, &h->in_elig,
@@ -379,91 +389,157 @@ mcl_status_t stage_in(mcl_mapper* h, DevBuf& buf, const void* src, size_t bytes,
   return MCL_OK;
 }
 
+// Classify a caller buffer, then stage it in (`src` may be NULL: *out = NULL).
+mcl_status_t classify_stage_in(mcl_mapper* h, DevBuf& buf, const void* src, size_t bytes,
+                               const void** out) {
+  *out = nullptr;
+  if (!src) return MCL_OK;
+  bool on = false;
+  mcl_status_t st = classify(h, src, &on);
+  if (st != MCL_OK) return st;
+  return stage_in(h, buf, src, bytes, on, out);
+}
+
+// Argument checks shared by the entry points: Q in [1, 32], D in [1, 16], and an epoch
+// count whose [E][Q][D] tables stay addressable. With `N`, also *N = D^Q <= 2^48
+// (MCL_E_RANGE otherwise).
+mcl_status_t check_shape(mcl_mapper* h, uint32_t Q, uint32_t D, uint64_t epochs, uint64_t* N) {
+  if (Q == 0 || D == 0 || Q > MCL_MAX_QUEUES || D > MCL_MAX_DEVICES) {
+    h->last_err = "Q must be in [1, 32] and D in [1, 16]";
+    return MCL_E_INVAL;
+  }
+  if (N && mul_overflow_pow(D, Q, 1ull << MCL_MAX_INDEX_BITS, N)) {
+    h->last_err = "D^Q exceeds 2^48";
+    return MCL_E_RANGE;
+  }
+  if (epochs > (1ull << 40) / ((uint64_t)Q * D)) {
+    h->last_err = "epochs too large";
+    return MCL_E_INVAL;
+  }
+  return MCL_OK;
+}
+
+// Result buffers of a search call: device pointers are written in place, host pointers
+// through handle-owned device buffers that copy_outputs_back returns to the caller.
+struct Outputs {
+  uint64_t* idx = nullptr;  // where the kernels write
+  uint64_t* ms = nullptr;
+  uint8_t* map = nullptr;
+  uint64_t* user_idx = nullptr;  // the caller's buffers
+  uint64_t* user_ms = nullptr;
+  uint8_t* user_map = nullptr;
+};
+
+mcl_status_t stage_outputs(mcl_mapper* h, uint64_t epochs, uint32_t Q, uint64_t* index,
+                           uint8_t* mapping, uint64_t* makespan, Outputs* o) {
+  o->user_idx = index;
+  o->user_ms = makespan;
+  o->user_map = mapping;
+  bool di = true, dm = true, dmap = true;
+  mcl_status_t st;
+  if (index && (st = classify(h, index, &di)) != MCL_OK) return st;
+  if ((st = classify(h, makespan, &dm)) != MCL_OK) return st;
+  if (mapping && (st = classify(h, mapping, &dmap)) != MCL_OK) return st;
+  o->idx = index;
+  o->ms = makespan;
+  o->map = mapping;
+  if (!di) {
+    MCL_CUDA(h, h->out_idx.ensure(epochs * 8), "cudaMalloc(staging)");
+    o->idx = (uint64_t*)h->out_idx.p;
+  }
+  if (!dm) {
+    MCL_CUDA(h, h->out_ms.ensure(epochs * 8), "cudaMalloc(staging)");
+    o->ms = (uint64_t*)h->out_ms.p;
+  }
+  if (!dmap) {
+    MCL_CUDA(h, h->out_map.ensure(epochs * Q), "cudaMalloc(staging)");
+    o->map = (uint8_t*)h->out_map.p;
+  }
+  return MCL_OK;
+}
+
+// Enqueue the device-to-host copies of staged outputs (the caller syncs the stream).
+mcl_status_t copy_outputs_back(mcl_mapper* h, uint64_t epochs, uint32_t Q, const Outputs& o) {
+  cudaStream_t s = h->stream;
+  if (o.idx != o.user_idx)
+    MCL_CUDA(h, cudaMemcpyAsync(o.user_idx, o.idx, epochs * 8, cudaMemcpyDeviceToHost, s), "D2H");
+  if (o.ms != o.user_ms)
+    MCL_CUDA(h, cudaMemcpyAsync(o.user_ms, o.ms, epochs * 8, cudaMemcpyDeviceToHost, s), "D2H");
+  if (o.map != o.user_map)
+    MCL_CUDA(h, cudaMemcpyAsync(o.user_map, o.map, epochs * Q, cudaMemcpyDeviceToHost, s), "D2H");
+  return MCL_OK;
+}
+
+// The status word the kernels raised (read after the stream sync) as an mcl_status_t.
+// kFlagNeedU64 and kFlagNoPack are handled by the search itself, not reported.
+mcl_status_t status_from_flags(mcl_mapper* h) {
+  const uint32_t flags = *(volatile uint32_t*)h->flags_host;
+  if (flags & mcl::kFlagBadModel) {
+    h->last_err = "invalid cost model (kernel id, source, offsets, sizes or bandwidths)";
+    return MCL_E_INVAL;
+  }
+  if (flags & mcl::kFlagBadMapping) {
+    h->last_err = "a mapping names a device >= D";
+    return MCL_E_INVAL;
+  }
+  if (flags & mcl::kFlagRange) {
+    h->last_err = "a cost entry, built cost or base load is >= 2^48";
+    return MCL_E_RANGE;
+  }
+  if (flags & mcl::kFlagInfeasible) {
+    h->last_err = "a queue has no eligible device below D";
+    return MCL_E_INVAL;
+  }
+  if (flags & mcl::kFlagPeerTimeout) {
+    h->last_err = "peer exchange timed out (a rank did not make the same call); exchange disabled";
+    return MCL_E_NCCL;
+  }
+  return MCL_OK;
+}
+
+void clear_flags(mcl_mapper* h) { *(volatile uint32_t*)h->flags_host = 0; }
+
 mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
                       const uint64_t* cost_kernel, const uint64_t* cost_xfer,
                       const uint64_t* base_load, const uint16_t* eligible,
                       uint64_t* mapping_index, uint8_t* mapping, uint64_t* makespan) {
   if (!h) return MCL_E_INVAL;
   h->last_err.clear();
-  if (Q == 0 || D == 0 || Q > MCL_MAX_QUEUES || D > MCL_MAX_DEVICES) {
-    h->last_err = "Q must be in [1, 32] and D in [1, 16]";
-    return MCL_E_INVAL;
-  }
   uint64_t N = 0;
-  if (mul_overflow_pow(D, Q, 1ull << MCL_MAX_INDEX_BITS, &N)) {
-    h->last_err = "D^Q exceeds 2^48";
-    return MCL_E_RANGE;
-  }
-  if (epochs == 0) return MCL_OK;
+  mcl_status_t st = check_shape(h, Q, D, epochs, &N);
+  if (st != MCL_OK || epochs == 0) return st;
   if (!cost_kernel || !cost_xfer || !mapping_index || !makespan) {
     h->last_err = "NULL required pointer";
     return MCL_E_INVAL;
   }
-  if (epochs > (1ull << 40) / ((uint64_t)Q * D)) {
-    h->last_err = "epochs too large";
-    return MCL_E_INVAL;
-  }
   DeviceGuard g(h->device);
-  // With a communicator the call is collective (a 1-rank communicator exercises the same
-  // packed-key all-reduce path on a single GPU).
-  const bool multi = h->comm != nullptr;
+  // With a communicator or imported peer slabs the call is collective (a 1-rank
+  // communicator / slab set exercises the same exchange on a single GPU). The fused peer
+  // exchange (NEXT-2) takes precedence over NCCL for the calls its slabs can hold.
+  const bool fused = h->peer_ready && epochs <= h->peer_cap;
+  const bool use_nccl = !fused && h->comm != nullptr;
+  const bool multi = fused || use_nccl;
 
   // ---- where do the buffers live? host buffers are staged through device memory ----
-  bool dk, dx, di, dm, dmap = true;
-  mcl_status_t st;
-  if ((st = classify(h, cost_kernel, &dk)) != MCL_OK) return st;
-  if ((st = classify(h, cost_xfer, &dx)) != MCL_OK) return st;
-  if ((st = classify(h, mapping_index, &di)) != MCL_OK) return st;
-  if ((st = classify(h, makespan, &dm)) != MCL_OK) return st;
-  if (mapping && (st = classify(h, mapping, &dmap)) != MCL_OK) return st;
-  const size_t in_bytes = (size_t)epochs * Q * D * sizeof(uint64_t);
-  const uint64_t* K = cost_kernel;
-  const uint64_t* X = cost_xfer;
-  uint64_t* o_idx = mapping_index;
-  uint64_t* o_ms = makespan;
-  uint8_t* o_map = mapping;
   cudaStream_t s = h->stream;
   if (h->timing >= 2) MCL_CUDA(h, cudaEventRecord(h->ev[2], s), "cudaEventRecord");
-  if (!dk) {
-    MCL_CUDA(h, h->in_k.ensure(in_bytes), "cudaMalloc(staging)");
-    MCL_CUDA(h, cudaMemcpyAsync(h->in_k.p, cost_kernel, in_bytes, cudaMemcpyHostToDevice, s), "H2D");
-    K = (const uint64_t*)h->in_k.p;
-  }
-  if (!dx) {
-    MCL_CUDA(h, h->in_x.ensure(in_bytes), "cudaMalloc(staging)");
-    MCL_CUDA(h, cudaMemcpyAsync(h->in_x.p, cost_xfer, in_bytes, cudaMemcpyHostToDevice, s), "H2D");
-    X = (const uint64_t*)h->in_x.p;
-  }
-  if (!di) {
-    MCL_CUDA(h, h->out_idx.ensure(epochs * 8), "cudaMalloc(staging)");
-    o_idx = (uint64_t*)h->out_idx.p;
-  }
-  if (!dm) {
-    MCL_CUDA(h, h->out_ms.ensure(epochs * 8), "cudaMalloc(staging)");
-    o_ms = (uint64_t*)h->out_ms.p;
-  }
-  if (mapping && !dmap) {
-    MCL_CUDA(h, h->out_map.ensure(epochs * Q), "cudaMalloc(staging)");
-    o_map = (uint8_t*)h->out_map.p;
-  }
+  const size_t in_bytes = (size_t)epochs * Q * D * sizeof(uint64_t);
+  const void *Kp, *Xp, *Bp, *Ep;
+  if ((st = classify_stage_in(h, h->in_k, cost_kernel, in_bytes, &Kp)) != MCL_OK) return st;
+  if ((st = classify_stage_in(h, h->in_x, cost_xfer, in_bytes, &Xp)) != MCL_OK) return st;
   // constrained variant: base loads [E][D] and eligible masks [E][Q] (either may be NULL)
+  if ((st = classify_stage_in(h, h->in_base, base_load, epochs * D * 8, &Bp)) != MCL_OK) return st;
+  if ((st = classify_stage_in(h, h->in_elig, eligible, epochs * Q * 2, &Ep)) != MCL_OK) return st;
+  const uint64_t* K = (const uint64_t*)Kp;
+  const uint64_t* X = (const uint64_t*)Xp;
+  const uint64_t* Bd = (const uint64_t*)Bp;
+  const uint16_t* Ed = (const uint16_t*)Ep;
   const bool constrained = base_load || eligible;
-  const uint64_t* Bd = nullptr;
-  const uint16_t* Ed = nullptr;
-  if (base_load) {
-    bool on;
-    if ((st = classify(h, base_load, &on)) != MCL_OK) return st;
-    const void* p = nullptr;
-    if ((st = stage_in(h, h->in_base, base_load, epochs * D * 8, on, &p)) != MCL_OK) return st;
-    Bd = (const uint64_t*)p;
-  }
-  if (eligible) {
-    bool on;
-    if ((st = classify(h, eligible, &on)) != MCL_OK) return st;
-    const void* p = nullptr;
-    if ((st = stage_in(h, h->in_elig, eligible, epochs * Q * 2, on, &p)) != MCL_OK) return st;
-    Ed = (const uint16_t*)p;
-  }
+  Outputs o;
+  if ((st = stage_outputs(h, epochs, Q, mapping_index, mapping, makespan, &o)) != MCL_OK) return st;
+  uint64_t* o_idx = o.idx;
+  uint64_t* o_ms = o.ms;
+  uint8_t* o_map = o.map;
 
   const int ibits = mcl::index_bits_host(N);
   mcl::EpochOut out{o_idx, o_ms, o_map, nullptr, nullptr};
@@ -472,6 +548,16 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
     MCL_CUDA(h, h->pair.ensure(epochs * 16), "cudaMalloc(pair)");
     out.key = (uint64_t*)h->key.p;
     out.pair = (uint64_t*)h->pair.p;
+  }
+  mcl::PeerArgs peer{};  // world = 0: exchange off
+  if (fused) {
+    peer.world = h->world;
+    peer.slabs = (uint64_t* const*)h->peer_ptrs.p;
+    peer.mine = (uint64_t*)h->peer_slab.p;
+    peer.cap = h->peer_cap;
+    peer.kdone = (uint32_t*)h->peer_kdone.p;
+    peer.gms = (uint64_t*)h->peer_gms.p;
+    peer.timeout_ns = h->peer_timeout_ns;
   }
   MCL_CUDA(h, h->done.ensure(epochs * sizeof(uint32_t), true), "cudaMalloc(done)");
 
@@ -497,7 +583,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
 
   int nlaunch = 0;
   for (int attempt = 0; attempt < 2; ++attempt) {
-    *(volatile uint32_t*)h->flags_host = 0;
+    clear_flags(h);
     nlaunch = 0;
     dim3 grid(1, 1, 1);
     int threads = 0;
@@ -545,7 +631,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
       mcl::BlockedArgs a{};
       a.Q = Q; a.D = D; a.E = epochs; a.K = K; a.X = X; a.rlo = lo; a.rhi = hi;
       a.out = out; a.ibits = ibits; a.flags = h->flags_dev; a.one = 1;
-      a.base = Bd; a.elig = Ed;
+      a.base = Bd; a.elig = Ed; a.peer = peer;
       const size_t smem = mcl::blocked_smem_bytes(Q, D, wide, threads, &a.off_red, &a.off_dig);
       const int occ = mcl::blocked_ctas_per_sm(D, wide, threads, smem);
       // Work layout (1-D grid): whole waves of epochs get one CTA each; the epochs of the
@@ -588,7 +674,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
       mcl::GenericArgs a{};
       a.Q = Q; a.D = D; a.E = epochs; a.K = K; a.X = X; a.rlo = lo; a.rhi = hi;
       a.out = out; a.ibits = ibits; a.flags = h->flags_dev;
-      a.base = Bd; a.elig = Ed;
+      a.base = Bd; a.elig = Ed; a.peer = peer;
       const size_t smem = mcl::generic_smem_bytes(Q, D, threads);
       size_grid(h, epochs, hi - lo, 8, threads, &grid);
       if (grid.x > 1) {
@@ -608,24 +694,22 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
     h->info[6] = 0;
     h->info[7] = 0;
 
-    if (multi) {
+    if (use_nccl) {
       ncclResult_t r = nccl().AllReduce(out.key, out.key, epochs, ncclUint64, ncclMin, h->comm, s);
       if (r != ncclSuccess) return nccl_fail(h, r, "ncclAllReduce(key)");
-      MCL_CUDA(h, mcl::launch_decode_key(out.key, epochs, Q, D, ibits, o_idx, o_ms, o_map, s), "decode launch");
+      MCL_CUDA(h, mcl::launch_decode_key(out.key, epochs, Q, D, ibits, o_idx, o_ms, o_map, h->flags_dev, s), "decode launch");
       nlaunch += 1;
       h->info[4] = 1;
     }
     MCL_CUDA(h, cudaStreamSynchronize(s), "search kernel");
     const uint32_t flags = *(volatile uint32_t*)h->flags_host;
-    if (flags & 1u) {
-      h->last_err = "a cost entry or base load is >= 2^48";
-      return MCL_E_RANGE;
+    if (flags & mcl::kFlagPeerTimeout) h->peer_ready = false;  // the slabs' rounds diverged
+    if ((st = status_from_flags(h)) != MCL_OK) return st;
+    if (fused) {
+      h->info[4] = 2;
+      h->info[6] = (flags & mcl::kFlagTwoStep) ? 1 : 0;
     }
-    if (flags & 8u) {
-      h->last_err = "a queue has no eligible device below D";
-      return MCL_E_INVAL;
-    }
-    if (flags & 2u) {  // some epoch's bound needs 64-bit loads: rerun the wide kernel
+    if (flags & mcl::kFlagNeedU64) {  // some epoch's bound needs 64-bit loads: rerun the wide kernel
       if (path != 1 && path != 5) {
         h->last_err = "internal: 64-bit request from a 64-bit kernel";
         return MCL_E_CUDA;
@@ -633,7 +717,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
       path = 2;
       continue;
     }
-    if (multi && (flags & 4u)) {  // key does not pack: two-step lexicographic all-reduce
+    if (use_nccl && (flags & mcl::kFlagNoPack)) {  // key does not pack: two-step lexicographic all-reduce
       uint64_t* gms;
       uint64_t* cand;
       MCL_CUDA(h, h->gms.ensure(epochs * 8), "cudaMalloc(gms)");
@@ -656,10 +740,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
   h->info[1] = nlaunch;
 
   // ---- results back to host buffers ----
-  if (!di) MCL_CUDA(h, cudaMemcpyAsync(mapping_index, o_idx, epochs * 8, cudaMemcpyDeviceToHost, s), "D2H");
-  if (!dm) MCL_CUDA(h, cudaMemcpyAsync(makespan, o_ms, epochs * 8, cudaMemcpyDeviceToHost, s), "D2H");
-  if (mapping && !dmap)
-    MCL_CUDA(h, cudaMemcpyAsync(mapping, o_map, epochs * Q, cudaMemcpyDeviceToHost, s), "D2H");
+  if ((st = copy_outputs_back(h, epochs, Q, o)) != MCL_OK) return st;
   if (h->timing >= 2) MCL_CUDA(h, cudaEventRecord(h->ev[3], s), "cudaEventRecord");
   MCL_CUDA(h, cudaStreamSynchronize(s), "D2H");
   h->timing_pending = h->timing > 0;  // elapsed times are read lazily (mcl_last_kernel_time)
@@ -687,71 +768,108 @@ mcl_status_t mcl_map_queues_constrained(mcl_mapper_t* h, uint32_t Q, uint32_t D,
                   constraints ? constraints->eligible : nullptr, mapping_index, mapping, makespan);
 }
 
+mcl_status_t mcl_peer_export(mcl_mapper_t* h, uint64_t max_epochs, uint8_t handle_out[64]) {
+  static_assert(sizeof(cudaIpcMemHandle_t) == 64, "CUDA IPC handles are 64 bytes");
+  if (!h) return MCL_E_INVAL;
+  h->last_err.clear();
+  if (!handle_out || max_epochs == 0 || max_epochs > (1ull << 20)) {
+    h->last_err = "max_epochs must be in [1, 2^20]";
+    return MCL_E_INVAL;
+  }
+  DeviceGuard g(h->device);
+  MCL_CUDA(h, cudaStreamSynchronize(h->stream), "cudaStreamSynchronize");
+  for (void* p : h->peer_opened) cudaIpcCloseMemHandle(p);  // a new slab voids any import
+  h->peer_opened.clear();
+  h->peer_ready = false;
+  h->peer_slab.release();  // a fresh allocation: the handle names exactly this slab
+  const size_t words = mcl::kPeerHeaderWords + 2 * max_epochs;
+  MCL_CUDA(h, h->peer_slab.ensure(words * 8), "cudaMalloc(peer slab)");
+  MCL_CUDA(h, cudaMemset(h->peer_slab.p, 0xff, words * 8), "cudaMemset(peer slab)");  // regions = none
+  const uint64_t header[mcl::kPeerHeaderWords] = {0, 0, max_epochs, 0, 0, 0, 0, 0};
+  MCL_CUDA(h, cudaMemcpy(h->peer_slab.p, header, sizeof(header), cudaMemcpyHostToDevice), "H2D(slab)");
+  MCL_CUDA(h, h->peer_kdone.ensure(4), "cudaMalloc(peer)");
+  MCL_CUDA(h, cudaMemset(h->peer_kdone.p, 0, 4), "cudaMemset(peer)");
+  MCL_CUDA(h, h->peer_gms.ensure(max_epochs * 8), "cudaMalloc(peer)");
+  cudaIpcMemHandle_t ipc;
+  MCL_CUDA(h, cudaIpcGetMemHandle(&ipc, h->peer_slab.p), "cudaIpcGetMemHandle");
+  MCL_CUDA(h, cudaDeviceSynchronize(), "cudaDeviceSynchronize");  // memsets ran on the legacy stream
+  std::memcpy(handle_out, &ipc, sizeof(ipc));
+  h->peer_cap = max_epochs;
+  return MCL_OK;
+}
+
+mcl_status_t mcl_peer_import(mcl_mapper_t* h, const uint8_t* handles, uint32_t timeout_ms) {
+  if (!h) return MCL_E_INVAL;
+  h->last_err.clear();
+  if (!handles) {
+    h->last_err = "NULL handles";
+    return MCL_E_INVAL;
+  }
+  if (!h->peer_slab.p || h->peer_cap == 0) {
+    h->last_err = "mcl_peer_export must come first";
+    return MCL_E_INVAL;
+  }
+  DeviceGuard g(h->device);
+  for (void* p : h->peer_opened) cudaIpcCloseMemHandle(p);
+  h->peer_opened.clear();
+  h->peer_ready = false;
+  std::vector<uint64_t*> ptrs((size_t)h->world);
+  for (int r = 0; r < h->world; ++r) {
+    if (r == h->rank) {
+      ptrs[r] = (uint64_t*)h->peer_slab.p;
+      continue;
+    }
+    cudaIpcMemHandle_t ipc;
+    std::memcpy(&ipc, handles + 64 * (size_t)r, sizeof(ipc));
+    void* p = nullptr;
+    MCL_CUDA(h, cudaIpcOpenMemHandle(&p, ipc, cudaIpcMemLazyEnablePeerAccess), "cudaIpcOpenMemHandle");
+    h->peer_opened.push_back(p);
+    ptrs[r] = (uint64_t*)p;
+    uint64_t cap = 0;
+    MCL_CUDA(h, cudaMemcpy(&cap, (uint64_t*)p + 2, 8, cudaMemcpyDeviceToHost), "D2H(peer slab)");
+    if (cap != h->peer_cap) {
+      h->last_err = "ranks exported slabs of different max_epochs";
+      return MCL_E_INVAL;
+    }
+  }
+  MCL_CUDA(h, h->peer_ptrs.ensure((size_t)h->world * 8), "cudaMalloc(peer)");
+  MCL_CUDA(h, cudaMemcpy(h->peer_ptrs.p, ptrs.data(), (size_t)h->world * 8, cudaMemcpyHostToDevice),
+           "H2D(peer)");
+  h->peer_timeout_ns = (uint64_t)(timeout_ms ? timeout_ms : 30000) * 1000000ull;
+  h->peer_ready = true;
+  return MCL_OK;
+}
+
 mcl_status_t mcl_map_queues_pruned(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
                                    const uint64_t* cost_kernel, const uint64_t* cost_xfer,
                                    const mcl_constraints_t* constraints, uint64_t* mapping_index,
                                    uint8_t* mapping, uint64_t* makespan) {
   if (!h) return MCL_E_INVAL;
   h->last_err.clear();
-  if (Q == 0 || D == 0 || Q > MCL_MAX_QUEUES || D > MCL_MAX_DEVICES) {
-    h->last_err = "Q must be in [1, 32] and D in [1, 16]";
-    return MCL_E_INVAL;
-  }
   uint64_t N = 0;
-  if (mul_overflow_pow(D, Q, 1ull << MCL_MAX_INDEX_BITS, &N)) {
-    h->last_err = "D^Q exceeds 2^48";
-    return MCL_E_RANGE;
-  }
-  if (epochs == 0) return MCL_OK;
+  mcl_status_t st = check_shape(h, Q, D, epochs, &N);
+  if (st != MCL_OK || epochs == 0) return st;
   if (!cost_kernel || !cost_xfer || !mapping_index || !makespan) {
     h->last_err = "NULL required pointer";
     return MCL_E_INVAL;
   }
-  if (epochs > (1ull << 40) / ((uint64_t)Q * D)) {
-    h->last_err = "epochs too large";
-    return MCL_E_INVAL;
-  }
   const uint64_t* base_load = constraints ? constraints->base_load : nullptr;
+  const uint16_t* eligible = constraints ? constraints->eligible : nullptr;
   // Small index spaces: scoring every mapping is cheaper than a tree search (same result).
   if (N < kPrunedMinMappings && h->comm == nullptr && h->world <= 1 && h->force_path != 6)
-    return map_impl(h, Q, D, epochs, cost_kernel, cost_xfer, base_load,
-                    constraints ? constraints->eligible : nullptr, mapping_index, mapping, makespan);
+    return map_impl(h, Q, D, epochs, cost_kernel, cost_xfer, base_load, eligible, mapping_index,
+                    mapping, makespan);
   DeviceGuard g(h->device);
   cudaStream_t s = h->stream;
-  mcl_status_t st;
-  const uint16_t* eligible = constraints ? constraints->eligible : nullptr;
-  bool dk, dx, db = true, de = true, di, dm, dmap = true;
-  if ((st = classify(h, cost_kernel, &dk)) != MCL_OK) return st;
-  if ((st = classify(h, cost_xfer, &dx)) != MCL_OK) return st;
-  if (base_load && (st = classify(h, base_load, &db)) != MCL_OK) return st;
-  if (eligible && (st = classify(h, eligible, &de)) != MCL_OK) return st;
-  if ((st = classify(h, mapping_index, &di)) != MCL_OK) return st;
-  if ((st = classify(h, makespan, &dm)) != MCL_OK) return st;
-  if (mapping && (st = classify(h, mapping, &dmap)) != MCL_OK) return st;
-  const size_t in_bytes = (size_t)epochs * Q * D * 8;
-  const void *K, *X, *B = nullptr, *El = nullptr;
   if (h->timing >= 2) MCL_CUDA(h, cudaEventRecord(h->ev[2], s), "cudaEventRecord");
-  if ((st = stage_in(h, h->in_k, cost_kernel, in_bytes, dk, &K)) != MCL_OK) return st;
-  if ((st = stage_in(h, h->in_x, cost_xfer, in_bytes, dx, &X)) != MCL_OK) return st;
-  if (base_load && (st = stage_in(h, h->in_base, base_load, epochs * D * 8, db, &B)) != MCL_OK)
-    return st;
-  if (eligible && (st = stage_in(h, h->in_elig, eligible, epochs * Q * 2, de, &El)) != MCL_OK)
-    return st;
-  uint64_t* o_idx = mapping_index;
-  uint64_t* o_ms = makespan;
-  uint8_t* o_map = mapping;
-  if (!di) {
-    MCL_CUDA(h, h->out_idx.ensure(epochs * 8), "cudaMalloc(staging)");
-    o_idx = (uint64_t*)h->out_idx.p;
-  }
-  if (!dm) {
-    MCL_CUDA(h, h->out_ms.ensure(epochs * 8), "cudaMalloc(staging)");
-    o_ms = (uint64_t*)h->out_ms.p;
-  }
-  if (mapping && !dmap) {
-    MCL_CUDA(h, h->out_map.ensure(epochs * Q), "cudaMalloc(staging)");
-    o_map = (uint8_t*)h->out_map.p;
-  }
+  const size_t in_bytes = (size_t)epochs * Q * D * 8;
+  const void *K, *X, *B, *El;
+  if ((st = classify_stage_in(h, h->in_k, cost_kernel, in_bytes, &K)) != MCL_OK) return st;
+  if ((st = classify_stage_in(h, h->in_x, cost_xfer, in_bytes, &X)) != MCL_OK) return st;
+  if ((st = classify_stage_in(h, h->in_base, base_load, epochs * D * 8, &B)) != MCL_OK) return st;
+  if ((st = classify_stage_in(h, h->in_elig, eligible, epochs * Q * 2, &El)) != MCL_OK) return st;
+  Outputs o;
+  if ((st = stage_outputs(h, epochs, Q, mapping_index, mapping, makespan, &o)) != MCL_OK) return st;
   // per-epoch subtree counters (zero) and incumbents (all ones), self-resetting
   if (h->bnb_next.cap < epochs * 8) {
     MCL_CUDA(h, h->bnb_next.ensure(epochs * 8, true), "cudaMalloc(bnb)");
@@ -783,28 +901,20 @@ mcl_status_t mcl_map_queues_pruned(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint
   a.base = (const uint64_t*)B; a.elig = (const uint16_t*)El; a.k = k;
   a.next = (uint64_t*)h->bnb_next.p; a.inc = (uint64_t*)h->bnb_inc.p;
   a.nodes = (uint64_t*)h->bnb_nodes.p; a.done = (uint32_t*)h->done.p;
-  a.out = mcl::EpochOut{o_idx, o_ms, o_map, nullptr, nullptr};
+  a.out = mcl::EpochOut{o.idx, o.ms, o.map, nullptr, nullptr};
   a.ibits = mcl::index_bits_host(N); a.flags = h->flags_dev;
   if (grid.x > 1) {
     MCL_CUDA(h, h->scratch.ensure((size_t)epochs * grid.x * sizeof(Cand)), "cudaMalloc(scratch)");
     a.scratch = (Cand*)h->scratch.p;
   }
-  *(volatile uint32_t*)h->flags_host = 0;
+  clear_flags(h);
   if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[0], s), "cudaEventRecord");
   MCL_CUDA(h, mcl::launch_bnb(a, grid, threads, s), "search_bnb launch");
   if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[1], s), "cudaEventRecord");
   uint64_t nodes = 0;
   MCL_CUDA(h, cudaMemcpyAsync(&nodes, h->bnb_nodes.p, 8, cudaMemcpyDeviceToHost, s), "D2H");
   MCL_CUDA(h, cudaStreamSynchronize(s), "search_bnb");
-  const uint32_t flags = *(volatile uint32_t*)h->flags_host;
-  if (flags & 1u) {
-    h->last_err = "a cost entry or base load is >= 2^48";
-    return MCL_E_RANGE;
-  }
-  if (flags & 8u) {
-    h->last_err = "a queue has no eligible device below D";
-    return MCL_E_INVAL;
-  }
+  if ((st = status_from_flags(h)) != MCL_OK) return st;
   h->info[0] = 6;
   h->info[1] = 1;
   h->info[2] = (int64_t)grid.x * grid.y;
@@ -813,10 +923,7 @@ mcl_status_t mcl_map_queues_pruned(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint
   h->info[5] = a.ibits;
   h->info[6] = 0;
   h->info[7] = (int64_t)nodes;
-  if (!di) MCL_CUDA(h, cudaMemcpyAsync(mapping_index, o_idx, epochs * 8, cudaMemcpyDeviceToHost, s), "D2H");
-  if (!dm) MCL_CUDA(h, cudaMemcpyAsync(makespan, o_ms, epochs * 8, cudaMemcpyDeviceToHost, s), "D2H");
-  if (mapping && !dmap)
-    MCL_CUDA(h, cudaMemcpyAsync(mapping, o_map, epochs * Q, cudaMemcpyDeviceToHost, s), "D2H");
+  if ((st = copy_outputs_back(h, epochs, Q, o)) != MCL_OK) return st;
   if (h->timing >= 2) MCL_CUDA(h, cudaEventRecord(h->ev[3], s), "cudaEventRecord");
   MCL_CUDA(h, cudaStreamSynchronize(s), "D2H");
   h->timing_pending = h->timing > 0;
@@ -856,10 +963,8 @@ mcl_status_t build_costs_dev(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t e
   };
   mcl_status_t st;
   for (auto& a : arrs) {
-    if (!a.src || a.bytes == 0) continue;
-    bool on = false;
-    if ((st = classify(h, a.src, &on)) != MCL_OK) return st;
-    if ((st = stage_in(h, *a.buf, a.src, a.bytes, on, &a.dev)) != MCL_OK) return st;
+    if (a.bytes == 0) continue;
+    if ((st = classify_stage_in(h, *a.buf, a.src, a.bytes, &a.dev)) != MCL_OK) return st;
   }
   mcl::CostArgs c{};
   c.D = D; c.EQ = EQ; c.num_kernels = m->num_kernels;
@@ -873,19 +978,6 @@ mcl_status_t build_costs_dev(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t e
   return MCL_OK;
 }
 
-mcl_status_t cost_flags(mcl_mapper_t* h) {
-  const uint32_t flags = *(volatile uint32_t*)h->flags_host;
-  if (flags & 32u) {
-    h->last_err = "invalid cost model (kernel id, source, offsets, sizes or bandwidths)";
-    return MCL_E_INVAL;
-  }
-  if (flags & 1u) {
-    h->last_err = "a built cost is >= 2^48";
-    return MCL_E_RANGE;
-  }
-  return MCL_OK;
-}
-
 }  // namespace
 
 extern "C" {
@@ -895,17 +987,13 @@ mcl_status_t mcl_build_costs(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t e
                              uint64_t* cost_xfer) {
   if (!h) return MCL_E_INVAL;
   h->last_err.clear();
-  if (Q == 0 || D == 0 || Q > MCL_MAX_QUEUES || D > MCL_MAX_DEVICES) {
-    h->last_err = "Q must be in [1, 32] and D in [1, 16]";
-    return MCL_E_INVAL;
-  }
-  if (epochs == 0) return MCL_OK;
-  if (!cost_kernel || !cost_xfer || epochs > (1ull << 40) / ((uint64_t)Q * D)) {
-    h->last_err = "NULL output or too many epochs";
+  mcl_status_t st = check_shape(h, Q, D, epochs, nullptr);
+  if (st != MCL_OK || epochs == 0) return st;
+  if (!cost_kernel || !cost_xfer) {
+    h->last_err = "NULL output";
     return MCL_E_INVAL;
   }
   DeviceGuard g(h->device);
-  mcl_status_t st;
   bool dk, dx;
   if ((st = classify(h, cost_kernel, &dk)) != MCL_OK) return st;
   if ((st = classify(h, cost_xfer, &dx)) != MCL_OK) return st;
@@ -920,7 +1008,7 @@ mcl_status_t mcl_build_costs(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t e
     MCL_CUDA(h, h->cost_x.ensure(out_bytes), "cudaMalloc(costs)");
     Xd = (uint64_t*)h->cost_x.p;
   }
-  *(volatile uint32_t*)h->flags_host = 0;
+  clear_flags(h);
   if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[0], h->stream), "cudaEventRecord");
   if ((st = build_costs_dev(h, Q, D, epochs, model, Kd, Xd)) != MCL_OK) return st;
   if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[1], h->stream), "cudaEventRecord");
@@ -928,7 +1016,7 @@ mcl_status_t mcl_build_costs(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t e
   if (!dx) MCL_CUDA(h, cudaMemcpyAsync(cost_xfer, Xd, out_bytes, cudaMemcpyDeviceToHost, h->stream), "D2H");
   MCL_CUDA(h, cudaStreamSynchronize(h->stream), "build_costs");
   h->timing_pending = h->timing > 0;
-  return cost_flags(h);
+  return status_from_flags(h);
 }
 
 mcl_status_t mcl_map_from_profiles(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
@@ -937,26 +1025,18 @@ mcl_status_t mcl_map_from_profiles(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint
                                    uint64_t* mapping_index, uint8_t* mapping, uint64_t* makespan) {
   if (!h) return MCL_E_INVAL;
   h->last_err.clear();
-  if (Q == 0 || D == 0 || Q > MCL_MAX_QUEUES || D > MCL_MAX_DEVICES) {
-    h->last_err = "Q must be in [1, 32] and D in [1, 16]";
-    return MCL_E_INVAL;
-  }
-  if (epochs == 0) return MCL_OK;
-  if (epochs > (1ull << 40) / ((uint64_t)Q * D)) {
-    h->last_err = "epochs too large";
-    return MCL_E_INVAL;
-  }
+  mcl_status_t st = check_shape(h, Q, D, epochs, nullptr);
+  if (st != MCL_OK || epochs == 0) return st;
   DeviceGuard g(h->device);
   const size_t bytes = (size_t)epochs * Q * D * 8;
   MCL_CUDA(h, h->cost_k.ensure(bytes), "cudaMalloc(costs)");
   MCL_CUDA(h, h->cost_x.ensure(bytes), "cudaMalloc(costs)");
-  *(volatile uint32_t*)h->flags_host = 0;
-  mcl_status_t st = build_costs_dev(h, Q, D, epochs, model, (uint64_t*)h->cost_k.p,
-                                    (uint64_t*)h->cost_x.p);
+  clear_flags(h);
+  st = build_costs_dev(h, Q, D, epochs, model, (uint64_t*)h->cost_k.p, (uint64_t*)h->cost_x.p);
   if (st != MCL_OK) return st;
   // the search's own flag checks follow; model errors must be reported first
   MCL_CUDA(h, cudaStreamSynchronize(h->stream), "build_costs");
-  if ((st = cost_flags(h)) != MCL_OK) return st;
+  if ((st = status_from_flags(h)) != MCL_OK) return st;
   return map_impl(h, Q, D, epochs, (const uint64_t*)h->cost_k.p, (const uint64_t*)h->cost_x.p,
                   constraints ? constraints->base_load : nullptr,
                   constraints ? constraints->eligible : nullptr, mapping_index, mapping, makespan);
@@ -968,55 +1048,28 @@ mcl_status_t mcl_score_mappings(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_
                                 uint64_t* makespan) {
   if (!h) return MCL_E_INVAL;
   h->last_err.clear();
-  if (Q == 0 || D == 0 || Q > MCL_MAX_QUEUES || D > MCL_MAX_DEVICES) {
-    h->last_err = "Q must be in [1, 32] and D in [1, 16]";
-    return MCL_E_INVAL;
-  }
-  if (epochs == 0) return MCL_OK;
+  mcl_status_t st = check_shape(h, Q, D, epochs, nullptr);
+  if (st != MCL_OK || epochs == 0) return st;
   if (!cost_kernel || !cost_xfer || !mappings || !makespan) {
     h->last_err = "NULL required pointer";
     return MCL_E_INVAL;
   }
-  if (epochs > (1ull << 40) / ((uint64_t)Q * D)) {
-    h->last_err = "epochs too large";
-    return MCL_E_INVAL;
-  }
   DeviceGuard g(h->device);
-  mcl_status_t st;
-  bool dk, dx, db = true, dmp, dm;
-  if ((st = classify(h, cost_kernel, &dk)) != MCL_OK) return st;
-  if ((st = classify(h, cost_xfer, &dx)) != MCL_OK) return st;
-  if (base_load && (st = classify(h, base_load, &db)) != MCL_OK) return st;
-  if ((st = classify(h, mappings, &dmp)) != MCL_OK) return st;
-  if ((st = classify(h, makespan, &dm)) != MCL_OK) return st;
-  const void *K, *X, *B = nullptr, *M;
+  const void *K, *X, *B, *M;
   const size_t in_bytes = (size_t)epochs * Q * D * 8;
-  if ((st = stage_in(h, h->in_k, cost_kernel, in_bytes, dk, &K)) != MCL_OK) return st;
-  if ((st = stage_in(h, h->in_x, cost_xfer, in_bytes, dx, &X)) != MCL_OK) return st;
-  if (base_load && (st = stage_in(h, h->in_base, base_load, epochs * D * 8, db, &B)) != MCL_OK)
-    return st;
-  if ((st = stage_in(h, h->in_elig, mappings, epochs * Q, dmp, &M)) != MCL_OK) return st;
-  uint64_t* o_ms = makespan;
-  if (!dm) {
-    MCL_CUDA(h, h->out_ms.ensure(epochs * 8), "cudaMalloc(staging)");
-    o_ms = (uint64_t*)h->out_ms.p;
-  }
-  *(volatile uint32_t*)h->flags_host = 0;
+  if ((st = classify_stage_in(h, h->in_k, cost_kernel, in_bytes, &K)) != MCL_OK) return st;
+  if ((st = classify_stage_in(h, h->in_x, cost_xfer, in_bytes, &X)) != MCL_OK) return st;
+  if ((st = classify_stage_in(h, h->in_base, base_load, epochs * D * 8, &B)) != MCL_OK) return st;
+  if ((st = classify_stage_in(h, h->in_elig, mappings, epochs * Q, &M)) != MCL_OK) return st;
+  Outputs o;
+  if ((st = stage_outputs(h, epochs, Q, nullptr, nullptr, makespan, &o)) != MCL_OK) return st;
+  clear_flags(h);
   MCL_CUDA(h, mcl::launch_score(Q, D, epochs, (const uint64_t*)K, (const uint64_t*)X,
-                                (const uint64_t*)B, (const uint8_t*)M, o_ms, h->flags_dev, h->stream),
+                                (const uint64_t*)B, (const uint8_t*)M, o.ms, h->flags_dev, h->stream),
            "score launch");
-  if (!dm) MCL_CUDA(h, cudaMemcpyAsync(makespan, o_ms, epochs * 8, cudaMemcpyDeviceToHost, h->stream), "D2H");
+  if ((st = copy_outputs_back(h, epochs, Q, o)) != MCL_OK) return st;
   MCL_CUDA(h, cudaStreamSynchronize(h->stream), "score kernel");
-  const uint32_t flags = *(volatile uint32_t*)h->flags_host;
-  if (flags & 16u) {
-    h->last_err = "a mapping names a device >= D";
-    return MCL_E_INVAL;
-  }
-  if (flags & 1u) {
-    h->last_err = "a cost entry or base load is >= 2^48";
-    return MCL_E_RANGE;
-  }
-  return MCL_OK;
+  return status_from_flags(h);
 }
 
 }  // extern "C"

@@ -1,11 +1,12 @@
-// reduce.cu -- epilogues of the cross-GPU argmin.
+// reduce.cu -- epilogues of the cross-GPU argmin over NCCL.
 //
 // Each rank's search kernel leaves, per epoch, a packed key (makespan << index_bits | index)
 // and the raw (makespan, index) pair. After ncclAllReduce(MIN) on the keys every rank holds
 // the global lexicographic minimum; these kernels turn it back into the public outputs.
-// When the makespan does not fit beside the index, the two-step path is used instead:
-// all-reduce MIN of the makespans, then all-reduce MIN of the indices of the ranks whose
-// local makespan equals the global one.
+// When no rank's makespan fits beside the index (the reduced key is kNone), the two-step
+// path is used instead: all-reduce MIN of the makespans, then all-reduce MIN of the
+// indices of the ranks whose local makespan equals the global one. (The fused peer
+// exchange, peer.cuh, does the same inside the search kernel.)
 #include "common.cuh"
 #include "kernels.h"
 
@@ -13,29 +14,17 @@ namespace mcl {
 
 namespace {
 
-__device__ __forceinline__ void write_outputs(uint64_t e, uint32_t Q, uint32_t D, uint64_t idx,
-                                              uint64_t ms, uint64_t* index, uint64_t* makespan,
-                                              uint8_t* mapping) {
-  index[e] = idx;
-  makespan[e] = ms;
-  if (mapping) {
-    uint64_t rest = idx;
-    for (int q = (int)Q - 1; q >= 0; --q) {
-      mapping[e * Q + (uint64_t)q] = (uint8_t)(rest % D);
-      rest /= D;
-    }
-  }
-}
-
 __global__ void decode_key_kernel(const uint64_t* __restrict__ key, uint64_t E, uint32_t Q,
                                   uint32_t D, int ibits, uint64_t* index, uint64_t* makespan,
-                                  uint8_t* mapping) {
+                                  uint8_t* mapping, volatile uint32_t* flags) {
   for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < E;
        e += (uint64_t)gridDim.x * blockDim.x) {
     const uint64_t k = key[e];
+    // no rank's candidate fitted the packed key (see write_epoch): the same on every rank
+    if (k == kNone) raise_flag(flags, kFlagNoPack);
     const uint64_t mask = (ibits >= 64) ? ~0ull : ((1ull << ibits) - 1);
     const uint64_t ms = (ibits == 0) ? k : (ibits >= 64 ? 0 : (k >> ibits));
-    write_outputs(e, Q, D, k & mask, ms, index, makespan, mapping);
+    write_result(index, makespan, mapping, e, Q, D, k & mask, ms);
   }
 }
 
@@ -59,7 +48,7 @@ __global__ void decode_pair_kernel(const uint64_t* __restrict__ gms,
                                    uint8_t* mapping) {
   for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < E;
        e += (uint64_t)gridDim.x * blockDim.x)
-    write_outputs(e, Q, D, gidx[e], gms[e], index, makespan, mapping);
+    write_result(index, makespan, mapping, e, Q, D, gidx[e], gms[e]);
 }
 
 unsigned grid_for(uint64_t E) {
@@ -71,8 +60,9 @@ unsigned grid_for(uint64_t E) {
 
 cudaError_t launch_decode_key(const uint64_t* key, uint64_t E, uint32_t Q, uint32_t D, int ibits,
                               uint64_t* index, uint64_t* makespan, uint8_t* mapping,
-                              cudaStream_t st) {
-  decode_key_kernel<<<grid_for(E), 256, 0, st>>>(key, E, Q, D, ibits, index, makespan, mapping);
+                              volatile uint32_t* flags, cudaStream_t st) {
+  decode_key_kernel<<<grid_for(E), 256, 0, st>>>(key, E, Q, D, ibits, index, makespan, mapping,
+                                                 flags);
   return cudaGetLastError();
 }
 

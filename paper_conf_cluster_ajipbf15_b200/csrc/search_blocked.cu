@@ -24,6 +24,7 @@
 // queues 0..Q-5 live in shared memory and update the base load vector by one-hot vectors
 // V[q][x] (V[q][x][d] = C[q][x] if d == x else 0) so every register index stays static.
 #include "blocked_core.cuh"
+#include "peer.cuh"
 
 namespace mcl {
 
@@ -206,6 +207,8 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
       }
     }
   }
+  // fused cross-GPU exchange (NEXT-2): the last CTA reduces over every rank and decodes
+  if (a.peer.world) peer_finish(a.peer, a.out, a.E, Q, D, a.ibits, a.flags);
 }
 
 template <typename T, int D>

@@ -10,6 +10,7 @@
 // (serialise on a device, concurrent across devices).
 #include "common.cuh"
 #include "kernels.h"
+#include "peer.cuh"
 
 namespace mcl {
 
@@ -113,6 +114,7 @@ __global__ void __launch_bounds__(256) search_generic_kernel(GenericArgs a) {
       }
     }
   }
+  if (a.peer.world) peer_finish(a.peer, a.out, a.E, Q, D, a.ibits, a.flags);  // NEXT-2
 }
 
 size_t generic_smem_bytes(uint32_t Q, uint32_t D, int threads) {

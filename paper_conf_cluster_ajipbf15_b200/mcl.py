@@ -29,6 +29,7 @@ EXPORTED = [
     "mcl_comm_unique_id", "mcl_comm_init", "mcl_comm_destroy",
     "mcl_map_queues_constrained", "mcl_score_mappings", "mcl_map_queues_pruned",
     "mcl_build_costs", "mcl_map_from_profiles",
+    "mcl_peer_export", "mcl_peer_import",
 ]
 
 
@@ -107,6 +108,8 @@ def load_library(path: str | None = None) -> ctypes.CDLL:
         "mcl_build_costs": (i32, [vp, u32, u32, u64, ctypes.POINTER(mcl_cost_model_t), vp, vp]),
         "mcl_map_from_profiles": (i32, [vp, u32, u32, u64, ctypes.POINTER(mcl_cost_model_t),
                                         ctypes.POINTER(mcl_constraints_t), vp, vp, vp]),
+        "mcl_peer_export": (i32, [vp, u64, ctypes.c_char_p]),
+        "mcl_peer_import": (i32, [vp, ctypes.c_char_p, u32]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -404,8 +407,37 @@ class Mapper:
     def launch_info(self) -> dict:
         i = mcl_last_launch_info(self.handle)
         return {"path": PATH_NAMES.get(i[0], str(i[0])), "launches": i[1], "ctas": i[2],
-                "threads": i[3], "allreduce": bool(i[4]), "index_bits": i[5], "two_step": bool(i[6]),
-                "nodes": i[7]}
+                "threads": i[3], "allreduce": bool(i[4]), "fused_exchange": i[4] == 2,
+                "index_bits": i[5], "two_step": bool(i[6]), "nodes": i[7]}
+
+    def peer_export(self, max_epochs: int = 1) -> bytes:
+        """Allocate this rank's exchange slab for the fused cross-GPU exchange and return
+        its 64-byte CUDA IPC handle (include/mcl.h mcl_peer_export)."""
+        buf = ctypes.create_string_buffer(64)
+        st = load_library().mcl_peer_export(self.handle, max_epochs, buf)
+        if st != MCL_OK:
+            raise MclError(st, "mcl_peer_export", mcl_last_error_string(self.handle))
+        return buf.raw
+
+    def peer_import(self, handles: list[bytes], timeout_ms: int = 0) -> None:
+        """Map every rank's slab (handles in rank order, 64 bytes each); afterwards calls
+        of up to max_epochs epochs exchange results inside the search kernel."""
+        if any(len(h) != 64 for h in handles):
+            raise ValueError("every handle is 64 bytes")
+        st = load_library().mcl_peer_import(self.handle, b"".join(handles), timeout_ms)
+        if st != MCL_OK:
+            raise MclError(st, "mcl_peer_import", mcl_last_error_string(self.handle))
+
+    def connect_peers(self, group=None, max_epochs: int = 1, timeout_ms: int = 0) -> None:
+        """Collective over a torch.distributed group: export, all-gather the handles
+        (plumbing only), import."""
+        import torch.distributed as dist
+
+        mine = self.peer_export(max_epochs)
+        world = dist.get_world_size(group)
+        got: list = [None] * world
+        dist.all_gather_object(got, mine, group=group)
+        self.peer_import(got, timeout_ms)
 
     def force_path(self, path: int) -> None:
         """Testing aid: 0 auto, 1 blocked u32 (CTA per epoch), 2 blocked u64, 3 generic,
