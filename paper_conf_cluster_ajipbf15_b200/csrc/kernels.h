@@ -32,7 +32,8 @@ struct PeerArgs {
   uint64_t* const* slabs;  // [world] every rank's slab, mapped into this process (device array)
   uint64_t* mine;          // this rank's slab
   uint64_t cap;            // epochs per region
-  uint32_t* kdone;         // CTAs of the kernel that finished; zero on entry, self-resetting
+  uint32_t* kdone;         // [2]: CTAs of the kernel that finished, "some CTA abandoned its
+                           // search" (input error / 64-bit rerun); zero on entry, self-resetting
   uint64_t* gms;           // [cap] scratch: global makespans of the two-step reduction
   uint64_t timeout_ns;
 };

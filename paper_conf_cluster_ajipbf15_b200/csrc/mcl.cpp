@@ -787,8 +787,8 @@ mcl_status_t mcl_peer_export(mcl_mapper_t* h, uint64_t max_epochs, uint8_t handl
   MCL_CUDA(h, cudaMemset(h->peer_slab.p, 0xff, words * 8), "cudaMemset(peer slab)");  // regions = none
   const uint64_t header[mcl::kPeerHeaderWords] = {0, 0, max_epochs, 0, 0, 0, 0, 0};
   MCL_CUDA(h, cudaMemcpy(h->peer_slab.p, header, sizeof(header), cudaMemcpyHostToDevice), "H2D(slab)");
-  MCL_CUDA(h, h->peer_kdone.ensure(4), "cudaMalloc(peer)");
-  MCL_CUDA(h, cudaMemset(h->peer_kdone.p, 0, 4), "cudaMemset(peer)");
+  MCL_CUDA(h, h->peer_kdone.ensure(8), "cudaMalloc(peer)");
+  MCL_CUDA(h, cudaMemset(h->peer_kdone.p, 0, 8), "cudaMemset(peer)");
   MCL_CUDA(h, h->peer_gms.ensure(max_epochs * 8), "cudaMalloc(peer)");
   cudaIpcMemHandle_t ipc;
   MCL_CUDA(h, cudaIpcGetMemHandle(&ipc, h->peer_slab.p), "cudaIpcGetMemHandle");

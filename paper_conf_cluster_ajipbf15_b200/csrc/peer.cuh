@@ -38,8 +38,35 @@ __device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t* p) {
   return v;
 }
 
+__device__ __forceinline__ uint64_t ld_relaxed_gpu(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// Reductions without a returned value (RED): no round trip per contribution.
+__device__ __forceinline__ void red_min_relaxed_sys(uint64_t* p, uint64_t v) {
+  asm volatile("red.relaxed.sys.global.min.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ void red_add_relaxed_sys(uint64_t* p, uint64_t v) {
+  asm volatile("red.relaxed.sys.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ void fence_acq_rel_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
+
+__device__ __forceinline__ uint32_t atom_add_acq_rel_gpu(uint32_t* p, uint32_t v) {
+  uint32_t old;
+  asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+  return old;
+}
+
 // One exchange round (steps 1-3), run by the whole last CTA. value(e) is this rank's
 // contribution for epoch e. Returns false if some rank did not signal within the timeout.
+// Ordering: the contributions (relaxed, system scope, any thread of the CTA) come before
+// the barrier; thread 0 then fences (acq_rel, system scope) and signals every rank, so a rank whose
+// ACQUIRE load sees the signal also sees every contribution (causality through the CTA
+// barrier and the release/acquire pair, PTX memory model).
 template <typename F>
 static __device__ bool peer_round(const PeerArgs& p, uint64_t R, uint64_t E, F value) {
   const uint64_t region = kPeerHeaderWords + (R & 1) * p.cap;
@@ -48,16 +75,13 @@ static __device__ bool peer_round(const PeerArgs& p, uint64_t R, uint64_t E, F v
     const uint64_t e = i / (uint64_t)p.world;
     const int r = (int)(i % (uint64_t)p.world);
     const uint64_t v = value(e);
-    if (v != kNone)
-      atomicMin_system(reinterpret_cast<unsigned long long*>(p.slabs[r] + region + e),
-                       (unsigned long long)v);
+    if (v != kNone) red_min_relaxed_sys(p.slabs[r] + region + e, v);
   }
   __syncthreads();
   __shared__ int s_ok;
   if (threadIdx.x == 0) {
-    __threadfence_system();  // every contribution of this CTA before the signal
-    for (int r = 0; r < p.world; ++r)
-      atomicAdd_system(reinterpret_cast<unsigned long long*>(p.slabs[r]), 1ull);
+    fence_acq_rel_sys();  // release pattern: one fence, then relaxed signals to every rank
+    for (int r = 0; r < p.world; ++r) red_add_relaxed_sys(p.slabs[r], 1ull);
     const uint64_t want = (R + 1) * (uint64_t)p.world;
     const uint64_t t0 = global_ns();
     int ok = 1;
@@ -84,26 +108,39 @@ __device__ __forceinline__ uint64_t peer_take(const PeerArgs& p, uint64_t R, uin
 
 // Called by EVERY CTA of a sharded search kernel after its last epoch. The last CTA to get
 // here runs the exchange and writes the public outputs o.index / o.makespan / o.mapping
-// from the global result. A search abandoned on an input error or for the 64-bit rerun
-// (status flags; identical on every rank since all ranks see the same inputs) skips it.
-static __device__ __forceinline__ void peer_finish(const PeerArgs& p, const EpochOut& o, uint64_t E, uint32_t Q,
-                            uint32_t D, int ibits, volatile uint32_t* flags) {
+// from the global result. `abandoned`: this CTA skipped an epoch on an input error or for
+// the 64-bit rerun; then the whole exchange is skipped (identical on every rank, since all
+// ranks see the same inputs). Only GPU-scope ordering is needed up to here: the other CTAs'
+// keys (written by their thread 0) are read by this GPU's last CTA alone, so an acq_rel
+// counter increment replaces fences. Measured on one B200 (scripts/collective_compare.sh,
+// scripts/peer_tail_bench.cu): a system-scope fence per CTA plus a read of the host-mapped
+// status word made the tail ~17 us; as written it adds ~6 us to the search kernel at
+// world = 1 -- a chain of dependent memory round trips (round counter, keys, reduction,
+// fence, signal, poll, read-back, outputs), of which the counting and one round alone are
+// ~2 us in isolation.
+static __device__ __forceinline__ void peer_finish(const PeerArgs& p, const EpochOut& o, uint64_t E,
+                                                   uint32_t Q, uint32_t D, int ibits,
+                                                   volatile uint32_t* flags, bool abandoned) {
   __shared__ bool s_last;
   __syncthreads();
   if (threadIdx.x == 0) {
-    __threadfence_system();  // this CTA's keys (and raised flags) before the count
-    s_last = (atomicAdd(p.kdone, 1u) == gridDim.x * gridDim.y * gridDim.z - 1);
+    if (abandoned) atomicOr(&p.kdone[1], 1u);
+    s_last = (atom_add_acq_rel_gpu(&p.kdone[0], 1u) == gridDim.x * gridDim.y * gridDim.z - 1);
   }
   __syncthreads();
   if (!s_last) return;
-  __threadfence_system();
-  if (threadIdx.x == 0) *p.kdone = 0;  // self-reset for the next call
-  if (*flags & (kFlagRange | kFlagNeedU64 | kFlagInfeasible)) return;
+  const bool skip = *reinterpret_cast<volatile uint32_t*>(&p.kdone[1]) != 0;
+  __syncthreads();
+  if (threadIdx.x == 0) {  // self-reset for the next call
+    p.kdone[0] = 0;
+    p.kdone[1] = 0;
+  }
+  if (skip) return;
 
   uint64_t R = *reinterpret_cast<volatile uint64_t*>(p.mine + 1);
   const uint64_t mask = (ibits >= 64) ? ~0ull : ((1ull << ibits) - 1);
   // round A: packed keys
-  if (!peer_round(p, R, E, [&](uint64_t e) { return o.key[e]; })) {
+  if (!peer_round(p, R, E, [&](uint64_t e) { return ld_relaxed_gpu(o.key + e); })) {
     if (threadIdx.x == 0) raise_flag(flags, kFlagPeerTimeout);
     return;
   }
@@ -120,7 +157,7 @@ static __device__ __forceinline__ void peer_finish(const PeerArgs& p, const Epoc
   ++R;
   if (__syncthreads_or(unpacked)) {
     // round B: global makespans
-    if (!peer_round(p, R, E, [&](uint64_t e) { return o.pair[2 * e]; })) {
+    if (!peer_round(p, R, E, [&](uint64_t e) { return ld_relaxed_gpu(o.pair + 2 * e); })) {
       if (threadIdx.x == 0) raise_flag(flags, kFlagPeerTimeout);
       return;
     }
@@ -128,7 +165,7 @@ static __device__ __forceinline__ void peer_finish(const PeerArgs& p, const Epoc
     ++R;
     // round C: lowest index among the ranks holding the global makespan
     if (!peer_round(p, R, E, [&](uint64_t e) {
-          return (o.pair[2 * e] == p.gms[e]) ? o.pair[2 * e + 1] : kNone;
+          return (ld_relaxed_gpu(o.pair + 2 * e) == p.gms[e]) ? ld_relaxed_gpu(o.pair + 2 * e + 1) : kNone;
         })) {
       if (threadIdx.x == 0) raise_flag(flags, kFlagPeerTimeout);
       return;

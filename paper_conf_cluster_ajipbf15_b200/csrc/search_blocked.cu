@@ -58,6 +58,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
   constexpr bool kSuper = (sizeof(T) == 4 && D <= kSuperMaxD);
 
   const uint64_t ncta = a.e_full + (a.E - a.e_full) * a.tail_cpe;
+  bool abandoned = false;  // an epoch skipped on an input error / for the 64-bit rerun
   for (uint64_t cta = blockIdx.x; cta < ncta; cta += gridDim.x) {
     uint64_t e;
     uint32_t part, parts;
@@ -92,10 +93,12 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
     __syncthreads();
     if (s_status) {
       if (tid == 0 && part == 0) raise_flag(a.flags, s_status);
+      abandoned = true;
       continue;
     }
     if (sizeof(T) == 4 && s_ub >= (1ull << 32)) {
       if (tid == 0 && part == 0) raise_flag(a.flags, kFlagNeedU64);
+      abandoned = true;
       continue;
     }
     // ---- tables: inner sums and one-hot outer vectors ----
@@ -208,7 +211,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
     }
   }
   // fused cross-GPU exchange (NEXT-2): the last CTA reduces over every rank and decodes
-  if (a.peer.world) peer_finish(a.peer, a.out, a.E, Q, D, a.ibits, a.flags);
+  if (a.peer.world) peer_finish(a.peer, a.out, a.E, Q, D, a.ibits, a.flags, abandoned);
 }
 
 template <typename T, int D>

@@ -28,6 +28,7 @@ __global__ void __launch_bounds__(256) search_generic_kernel(GenericArgs a) {
   __shared__ uint64_t s_base[kMaxDevices];
   __shared__ uint64_t s_feas;
 
+  bool abandoned = false;  // an epoch skipped on an input error (peer exchange skipped too)
   for (uint64_t e = blockIdx.y; e < a.E; e += gridDim.y) {
     __syncthreads();
     if (tid == 0) s_status = 0;
@@ -46,6 +47,7 @@ __global__ void __launch_bounds__(256) search_generic_kernel(GenericArgs a) {
     __syncthreads();
     if (s_status) {
       if (tid == 0 && blockIdx.x == 0) raise_flag(a.flags, s_status);
+      abandoned = true;
       continue;
     }
     const uint64_t nr = a.rhi - a.rlo;
@@ -114,7 +116,7 @@ __global__ void __launch_bounds__(256) search_generic_kernel(GenericArgs a) {
       }
     }
   }
-  if (a.peer.world) peer_finish(a.peer, a.out, a.E, Q, D, a.ibits, a.flags);  // NEXT-2
+  if (a.peer.world) peer_finish(a.peer, a.out, a.E, Q, D, a.ibits, a.flags, abandoned);  // NEXT-2
 }
 
 size_t generic_smem_bytes(uint32_t Q, uint32_t D, int threads) {
