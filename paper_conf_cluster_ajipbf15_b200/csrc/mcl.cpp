@@ -740,9 +740,11 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
   h->info[1] = nlaunch;
 
   // ---- results back to host buffers ----
+  const bool staged = o.idx != o.user_idx || o.ms != o.user_ms || o.map != o.user_map;
   if ((st = copy_outputs_back(h, epochs, Q, o)) != MCL_OK) return st;
   if (h->timing >= 2) MCL_CUDA(h, cudaEventRecord(h->ev[3], s), "cudaEventRecord");
-  MCL_CUDA(h, cudaStreamSynchronize(s), "D2H");
+  // the stream is already idle unless copies or the call-end event were enqueued
+  if (staged || h->timing >= 2) MCL_CUDA(h, cudaStreamSynchronize(s), "D2H");
   h->timing_pending = h->timing > 0;  // elapsed times are read lazily (mcl_last_kernel_time)
   return MCL_OK;
 }

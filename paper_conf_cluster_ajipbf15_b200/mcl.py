@@ -196,17 +196,30 @@ def mcl_comm_destroy(comm: int | None) -> None:
     load_library().mcl_comm_destroy(comm)
 
 
+_TORCH = None  # (torch.Tensor, {numpy dtype: torch dtype}) once torch is importable
+
+
+def _torch_types():
+    global _TORCH
+    if _TORCH is None:
+        try:
+            import torch
+        except ImportError:  # pragma: no cover
+            _TORCH = (type(None), {})
+        else:
+            _TORCH = (torch.Tensor, {np.uint64: torch.uint64, np.uint8: torch.uint8,
+                                     np.uint16: torch.uint16, np.uint32: torch.uint32,
+                                     np.int32: torch.int32, np.float64: torch.float64})
+    return _TORCH
+
+
 def _ptr_and_keepalive(x, dtype, convert: bool = False):
     """(pointer, owner) for a torch tensor or numpy array of the given numpy dtype. With
     ``convert`` (read-only inputs) a numpy array is first made a contiguous copy of the
     right dtype; outputs must already match."""
-    try:
-        import torch
-    except ImportError:  # pragma: no cover
-        torch = None
-    if torch is not None and isinstance(x, torch.Tensor):
-        want = {np.uint64: torch.uint64, np.uint8: torch.uint8, np.uint16: torch.uint16,
-                np.uint32: torch.uint32, np.int32: torch.int32, np.float64: torch.float64}[dtype]
+    tensor_type, dtypes = _TORCH or _torch_types()
+    if isinstance(x, tensor_type):
+        want = dtypes[dtype]
         if x.dtype != want or not x.is_contiguous():
             raise TypeError(f"expected a contiguous {want} tensor")
         return x.data_ptr(), x
@@ -247,7 +260,7 @@ class Mapper:
         """Run the search writing into caller-owned outputs. K, X: [E, Q, D] uint64;
         index, makespan: [E] uint64; mapping: [E, Q] uint8 or None. Tensors may live on the
         handle's CUDA device or on the host."""
-        E, Q, D = (int(s) for s in K.shape)
+        E, Q, D = K.shape
         pk, _k = _ptr_and_keepalive(K, np.uint64)
         px, _x = _ptr_and_keepalive(X, np.uint64)
         pi, _i = _ptr_and_keepalive(index, np.uint64)
@@ -255,7 +268,7 @@ class Mapper:
         pmap = None
         if mapping is not None:
             pmap, _mp = _ptr_and_keepalive(mapping, np.uint8)
-        st = mcl_map_queues(self.handle, Q, D, E, pk, px, pi, pmap, pm)
+        st = (_lib or load_library()).mcl_map_queues(self.handle, Q, D, E, pk, px, pi, pmap, pm)
         if st != MCL_OK:
             raise MclError(st, "mcl_map_queues", mcl_last_error_string(self.handle))
 
