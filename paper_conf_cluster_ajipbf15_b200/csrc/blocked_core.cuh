@@ -18,7 +18,7 @@
 // sm_100a three-input minimum (VIMNMX3: two mappings per ALU instruction), so the floor is
 // 1.5 ALU instructions per mapping. The block minimum is compared
 // with the thread's running best (strict <, blocks visited in increasing index order);
-// only the single best block is re-scanned at the end to recover the lowest leaf index.
+// only the best block (or super-block) is re-scanned at the end for the lowest leaf index.
 //
 // The outer digits walk an odometer: digit x (queue Q-4) is the block loop, the digits of
 // queues 0..Q-5 live in shared memory and update the base load vector by one-hot vectors
@@ -110,23 +110,36 @@ __device__ __forceinline__ void for_each_leaf(const Sums<T, D>& s, T M, F&& f) {
       }
 }
 
-// Minimum makespan over one block, folded two leaves per three-input min.
+// Fold one block's leaves into a running 4-way minimum, two leaves per three-input min.
+// `first` = the number of leaves folded before this block in the same run (a compile-time
+// constant after unrolling), so the pairing continues across the blocks of a super-block.
+template <typename T, int D>
+__device__ __forceinline__ void block_fold(const Sums<T, D>& s, T M, int first, T (&acc)[4], T& pend) {
+  for_each_leaf<T, D>(s, M, [&](int leaf, T v) {
+    const int n = first + leaf;
+    if (n & 1) {
+      acc[(n >> 1) & 3] = min3(acc[(n >> 1) & 3], pend, v);
+    } else {
+      pend = v;
+    }
+  });
+}
+
+template <typename T>
+__device__ __forceinline__ T fold_result(const T (&acc)[4], T pend, int leaves) {
+  T g = min3(acc[0], acc[1], min2(acc[2], acc[3]));
+  if (leaves & 1) g = min2(g, pend);
+  return g;
+}
+
+// Minimum makespan over one block.
 template <typename T, int D>
 __device__ __forceinline__ T block_eval(const Sums<T, D>& s, T M) {
   constexpr T kMax = ~T(0);
   T acc[4] = {kMax, kMax, kMax, kMax};
   T pend = kMax;
-  for_each_leaf<T, D>(s, M, [&](int leaf, T v) {
-    if (leaf & 1) {
-      acc[(leaf >> 1) & 3] = min3(acc[(leaf >> 1) & 3], pend, v);
-    } else {
-      pend = v;
-    }
-  });
-  constexpr int kLeaves = D * D * D;
-  T g = min3(acc[0], acc[1], min2(acc[2], acc[3]));
-  if (kLeaves & 1) g = min2(g, pend);
-  return g;
+  block_fold<T, D>(s, M, 0, acc, pend);
+  return fold_result<T>(acc, pend, D * D * D);
 }
 
 template <typename T, int D>
@@ -139,10 +152,16 @@ __device__ __forceinline__ T block_eval(const T (&P)[D], const T* __restrict__ i
 // A SUPER-BLOCK: the D blocks x = 0..D-1 of the fourth-innermost digit (queue Q-4) with
 // the same outer prefix `base`. Only device x's load changes between them, so the sums of
 // the other devices are shared and the block loop is unrolled with static x (used for
-// small D, where a D^3 block alone is too short to amortise its setup).
+// small D, where a D^3 block alone is too short to amortise its setup). All D^4 leaves fold
+// into ONE running minimum (one finalisation and one comparison with the thread's best per
+// super-block); the rare new best is located by re-scanning the super-block at the end.
 template <typename T, int D>
-__device__ __forceinline__ void superblock_eval(const T (&base)[D], const T* __restrict__ in,
-                                                const T* __restrict__ c4, uint32_t one, T (&g)[D]) {
+__device__ __forceinline__ T superblock_eval(const T (&base)[D], const T* __restrict__ in,
+                                             const T* __restrict__ c4, uint32_t one) {
+  constexpr T kMax = ~T(0);
+  constexpr int kLeaves = D * D * D;
+  T acc[4] = {kMax, kMax, kMax, kMax};
+  T pend = kMax;
   Sums<T, D> sb;
   make_sums<T, D>(sb, base, in, one);
   const T Mb = max_of<T, D>(base);
@@ -158,8 +177,9 @@ __device__ __forceinline__ void superblock_eval(const T (&base)[D], const T* __r
     s.bc[x] = add_f(sb.bc[x], cx, one);
     s.abc[x] = add_f(sb.abc[x], cx, one);
     const T M = max2(Mb, add_f(base[x], cx, one));
-    g[x] = block_eval<T, D>(s, M);
+    block_fold<T, D>(s, M, x * kLeaves, acc, pend);
   }
+  return fold_result<T>(acc, pend, D * kLeaves);
 }
 
 template <typename T, int D>
@@ -236,9 +256,27 @@ struct WalkCtx {
   uint32_t one;
 };
 
+// Lowest mapping index in blocks [bb, bb + span) whose makespan equals `target` (the span
+// is known to hold one): blocks in increasing order, each re-scanned by the whole warp.
+// Called by all 32 lanes with the same arguments.
+template <typename T, int D>
+__device__ __forceinline__ uint64_t span_first_warp(uint64_t bb, uint32_t span, int O,
+                                                    const T* __restrict__ V, const T* __restrict__ B0,
+                                                    const T* __restrict__ in, T target, uint32_t one) {
+  for (uint32_t t = 0; t < span; ++t) {
+    T P[D];
+    prefix_of<T, D>(P, bb + t, O, V, B0, one);
+    const uint32_t leaf = block_first_warp<T, D>(P, in, target);
+    if (leaf != 0xffffffffu) return (bb + t) * (uint64_t)(D * D * D) + leaf;
+  }
+  return kNone;
+}
+
+// best_span: the number of blocks starting at best_blk that hold the best (1, or D for a
+// super-block).
 template <typename T, int D>
 __device__ __forceinline__ void walk_blocks(const WalkCtx<T, D>& w, uint64_t b0, uint64_t nleft,
-                                            T& best, uint64_t& best_blk) {
+                                            T& best, uint64_t& best_blk, uint32_t& best_span) {
   constexpr bool kSuper = (sizeof(T) == 4 && D <= kSuperMaxD);
   const int O = w.O, nthr = w.nthr, tid = w.tid;
   const uint32_t one = w.one;
@@ -263,6 +301,7 @@ __device__ __forceinline__ void walk_blocks(const WalkCtx<T, D>& w, uint64_t b0,
       if (g < best) {
         best = g;
         best_blk = bk;
+        best_span = 1;
       }
     };
     for (; nleft && (blk % chunk) != 0; ++blk, --nleft) single(blk);
@@ -283,17 +322,11 @@ __device__ __forceinline__ void walk_blocks(const WalkCtx<T, D>& w, uint64_t b0,
         load_vec<T, D>(vy, Vy + y * D);
 #pragma unroll
         for (int d = 0; d < D; ++d) base[d] = add_f(base2[d], vy[d], one);
-        T g[D];
-        superblock_eval<T, D>(base, in, c4, one, g);
-        T gs = g[0];
-#pragma unroll
-        for (int t = 1; t < D; ++t) gs = min2(gs, g[t]);
-        if (gs < best) {  // rare: locate the first block holding the new minimum
+        const T gs = superblock_eval<T, D>(base, in, c4, one);
+        if (gs < best) {
           best = gs;
-          const uint64_t bb = blk + (uint64_t)y * D;
-#pragma unroll
-          for (int t = D - 1; t >= 0; --t)
-            if (g[t] == gs) best_blk = bb + t;
+          best_blk = blk + (uint64_t)y * D;
+          best_span = D;
         }
       }
     }
@@ -321,16 +354,11 @@ __device__ __forceinline__ void walk_blocks(const WalkCtx<T, D>& w, uint64_t b0,
       uint64_t blk = b0;
       while (true) {
         if (kSuper && x == 0 && nleft >= (uint64_t)D) {
-          T g[D];
-          superblock_eval<T, D>(base, in, c4, one, g);
-          T gs = g[0];
-#pragma unroll
-          for (int t = 1; t < D; ++t) gs = min2(gs, g[t]);
-          if (gs < best) {  // rare: locate the first block holding the new minimum
+          const T gs = superblock_eval<T, D>(base, in, c4, one);
+          if (gs < best) {
             best = gs;
-#pragma unroll
-            for (int t = D - 1; t >= 0; --t)
-              if (g[t] == gs) best_blk = blk + t;
+            best_blk = blk;
+            best_span = D;
           }
           x = D;
           nleft -= D;
@@ -345,6 +373,7 @@ __device__ __forceinline__ void walk_blocks(const WalkCtx<T, D>& w, uint64_t b0,
           if (g < best) {
             best = g;
             best_blk = blk;
+            best_span = 1;
           }
         }
         if (!nleft) break;

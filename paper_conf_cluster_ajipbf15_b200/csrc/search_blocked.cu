@@ -141,9 +141,10 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
 
     T best = ~T(0);
     uint64_t best_blk = kNone;
+    uint32_t best_span = 1;
     const uint32_t one = a.one;
     const WalkCtx<T, D> wctx{in, V, zero, base0, dig, O, nthr, tid, one};
-    walk_blocks<T, D>(wctx, b0, nleft, best, best_blk);
+    walk_blocks<T, D>(wctx, b0, nleft, best, best_blk, best_span);
     // ---- a5: lowest index inside the best block, then warp / CTA / epoch argmin ----
     // Thread ranges ascend with the thread id, so the CTA's lowest-index optimum belongs to
     // the LOWEST thread whose best equals the CTA minimum; only that thread re-scans its
@@ -173,11 +174,10 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
       if (win != 0xffffffffu && (uint32_t)(tid >> 5) == (win >> 5)) {  // the winner's warp
         const int wl = (int)(win & 31);
         const uint64_t bb = __shfl_sync(0xffffffffu, best_blk, wl);
+        const uint32_t span = __shfl_sync(0xffffffffu, best_span, wl);
         const T bt = __shfl_sync(0xffffffffu, best, wl);
-        T P[D];
-        prefix_of<T, D>(P, bb, O, V, base0, one);
-        const uint32_t leaf = block_first_warp<T, D>(P, in, bt);
-        if ((uint32_t)tid == win) s_cand = Cand{(uint64_t)bt, bb * (uint64_t)(D * D * D) + leaf};
+        const uint64_t idx = span_first_warp<T, D>(bb, span, O, V, base0, in, bt, one);
+        if ((uint32_t)tid == win) s_cand = Cand{(uint64_t)bt, idx};
       }
       __syncthreads();
     }

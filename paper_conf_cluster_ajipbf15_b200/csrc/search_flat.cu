@@ -104,7 +104,8 @@ __global__ void __launch_bounds__(32, (D <= 5) ? 16 : 8) search_flat_kernel(Flat
     const uint64_t s1 = (b_lo + c_hi * chunk < b_lo + len) ? b_lo + c_hi * chunk : b_lo + len;
     T best = ~T(0);
     uint64_t best_blk = kNone;
-    if (s1 > s0) walk_blocks<T, D>(wctx, s0, s1 - s0, best, best_blk);
+    uint32_t best_span = 1;
+    if (s1 > s0) walk_blocks<T, D>(wctx, s0, s1 - s0, best, best_blk, best_span);
 
     // ---- a5: warp argmin; lanes ascend with the index, so the lowest lane holding the
     // minimum owns the piece's lowest-index optimum and alone re-scans its best block ----
@@ -116,11 +117,9 @@ __global__ void __launch_bounds__(32, (D <= 5) ? 16 : 8) search_flat_kernel(Flat
     if (!holders) continue;
     const int wl = __ffs(holders) - 1;
     const uint64_t bb = __shfl_sync(0xffffffffu, best_blk, wl);
-    T P[D];
-    prefix_of<T, D>(P, bb, O, V, zero, a.one);
-    const uint32_t leaf = block_first_warp<T, D>(P, in, (T)wmin);
+    const uint32_t span = __shfl_sync(0xffffffffu, best_span, wl);
+    const uint64_t idx = span_first_warp<T, D>(bb, span, O, V, zero, in, (T)wmin, a.one);
     if (lane == wl) {
-      const uint64_t idx = bb * (uint64_t)(D * D * D) + leaf;
       atomicMin((unsigned long long*)&a.keys[e], (unsigned long long)((bv << a.ibits) | idx));
       __threadfence();
       // the warp that completes the epoch's block count publishes its result
