@@ -41,6 +41,11 @@ UNIT = "mappings/s"
 ALU_LANES_PER_CLK_SM = 64       # B200 ALU pipe: 16 lanes x 4 SMSPs per SM per clock (measured: probe)
 ALU_INSTR_PER_MAPPING = 1.5     # floor: 1 VIMNMX forms the makespan + 1/2 VIMNMX3 folds it
 L2_FLUSH_BYTES = 256 << 20      # > 126 MB L2
+HOLD_US = 200                   # spin ahead of each kernel-duration launch (> host launch latency)
+KERNEL_TIMING = ("CUDA events on the mapper's stream around the search launch, in a pass of `steps` "
+                 "launches after the timed steps, each preceded by a 200 us spin kernel so the events "
+                 "measure device execution (kernel_ms_in_step: the same events inside the timed steps, "
+                 "where an idle GPU adds the host launch latency)")
 KERNEL_NAMES = {"blocked_u32": "search_blocked_kernel<u32, D>", "blocked_u64": "search_blocked_kernel<u64, D>",
                 "generic": "search_generic_kernel", "flat_u32": "search_flat_kernel<u32, D>",
                 "small_batched": "search_small_kernel<Q, D>"}
@@ -245,6 +250,14 @@ def main():
     msp = torch.empty(E, dtype=torch.uint64, device=dev)
     mpg = torch.empty((E, Q), dtype=torch.uint8, device=dev)
     flush = torch.empty(L2_FLUSH_BYTES, dtype=torch.uint8, device=dev)
+    flush64 = flush.view(torch.int64)
+
+    def flush_l2(i):
+        # write a buffer larger than L2, then read it back: the write evicts everything of
+        # ours, the read evicts the write's dirty lines (written back here, not charged to
+        # the next kernel's DRAM traffic), leaving L2 clean and holding none of the inputs
+        flush.fill_(i & 0xFF)
+        flush64.sum()
     mapper = Mapper(local, stream=stream.cuda_stream, nccl_comm=comm, rank=rank if comm else 0,
                     world=world if comm else 1)
     combine = "nccl" if comm else "none"
@@ -278,7 +291,7 @@ def main():
     torch.cuda.synchronize(dev)
     with ClockSampler(local) as clk:
         for i in range(args.steps):
-            flush.fill_(i & 0xFF)  # L2 flush between timed steps, outside the events
+            flush_l2(i)  # L2 flush between timed steps, outside the events
             starts[i].record(stream)
             mapper.map_queues_into(Kd, Xd, idx, mpg, msp)
             ends[i].record(stream)
@@ -289,11 +302,22 @@ def main():
         dist.barrier()
     step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
     total_ms = sum(step_ms)
-    kern_mean = statistics.mean(kernel_ms)
-    t = torch.tensor([total_ms, kern_mean], dtype=torch.float64, device=dev)
+    kern_step_mean = statistics.mean(kernel_ms)
+    # Kernel-duration pass (outside the timed steps, same launches): a spin kernel holds the
+    # stream while the host enqueues the start event and the launch, so the events bracket
+    # the search kernel's device execution, not the host launch latency an idle GPU adds.
+    mapper.set_timing(True, hold_us=HOLD_US)
+    kernel_dev = []
+    for i in range(args.steps):
+        flush_l2(i)
+        mapper.map_queues_into(Kd, Xd, idx, mpg, msp)
+        kernel_dev.append(mapper.last_kernel_time_ms()[0])
+    mapper.set_timing(True, hold_us=0)
+    kern_mean = statistics.mean(kernel_dev)
+    t = torch.tensor([total_ms, kern_mean, kern_step_mean], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    total_ms, kern_mean = float(t[0]), float(t[1])
+    total_ms, kern_mean, kern_step_mean = float(t[0]), float(t[1]), float(t[2])
     ms_per_step = total_ms / args.steps
     mappings_per_step = w["E"] * w["N"] * (world if is_batched(w) else 1)
     value = mappings_per_step / (ms_per_step / 1e3)
@@ -339,6 +363,7 @@ def main():
             roof = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tops/s",
                     "frac": achieved / peak, "traffic": traffic_from_profiles(args.workload),
                     "kernel": KERNEL_NAMES.get(info["path"], info["path"]), "kernel_ms": kern_mean,
+                    "kernel_ms_in_step": kern_step_mean, "kernel_timing": KERNEL_TIMING,
                     "algorithmic": f"{ALU_INSTR_PER_MAPPING} ALU lane-instructions per mapping x "
                                    f"{mappings_per_launch:.4g} mappings per launch",
                     "peak_basis": f"derived: {ALU_LANES_PER_CLK_SM} ALU lanes/clk/SM x {sms} SMs x "
@@ -355,7 +380,8 @@ def main():
             peak = measured_hbm()
             roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                     "frac": achieved / peak, "traffic": traffic_from_profiles(args.workload),
-                    "kernel": "search_small_kernel", "kernel_ms": kern_mean}
+                    "kernel": "search_small_kernel", "kernel_ms": kern_mean,
+                    "kernel_ms_in_step": kern_step_mean, "kernel_timing": KERNEL_TIMING}
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
@@ -368,7 +394,7 @@ def main():
                            else "ncclAllReduce(min)")) if sharded
                        else (f"epoch replicas x{world}" if world > 1 else "1 GPU"),
                        "combine": combine,
-                       "l2": "flushed between timed steps (256 MiB write, outside the events)",
+                       "l2": "flushed between timed steps (256 MiB write + read-back, outside the events)",
                        "path": info["path"], "ctas": info["ctas"], "threads": info["threads"],
                        "result": {"index": int(idx[0]), "makespan": int(msp[0])}},
             "clocks": clocks,

@@ -26,6 +26,13 @@ mcl_status_t mcl_set_timing(mcl_mapper_t* h, int enable);
    else 0). enable: 0 = off, 1 = search kernel only (two events), 2 = kernel and call. */
 mcl_status_t mcl_last_kernel_time(const mcl_mapper_t* h, float* kernel_ms, float* call_ms);
 
+/* Measurement aid for the timing events (not part of any step): with hold_us > 0, every
+   timed launch is preceded on the same stream by a one-thread kernel that spins for
+   hold_us microseconds (%globaltimer), so the host-side launch latency elapses while the
+   stream is busy and the kernel_ms events bracket the search kernel's device execution
+   only. 0 (default) disables it. Has no effect unless timing is enabled. */
+mcl_status_t mcl_set_timing_hold(mcl_mapper_t* h, uint32_t hold_us);
+
 /*
  * Integer-pipe throughput probe on `device` (op: 0 = 2-input min/max VIMNMX, 1 = 3-input
  * VIMNMX3, 2 = IADD3, 3 = IMAD, 4 = VIMNMX3 and IMAD interleaved). Runs for ~1 ms at full

@@ -116,6 +116,8 @@ bool blocked_supported(uint32_t Q, uint32_t D);
 int blocked_ctas_per_sm(uint32_t D, bool wide, int threads, size_t smem);
 size_t blocked_smem_bytes(uint32_t Q, uint32_t D, bool wide, int threads, size_t* off_red,
                           size_t* off_dig);
+// one-thread kernel spinning for `ns` nanoseconds of %globaltimer (timing aid, probe.cu)
+cudaError_t launch_hold(uint64_t ns, cudaStream_t st);
 cudaError_t launch_blocked(const BlockedArgs& a, bool wide, dim3 grid, int threads, size_t smem,
                            cudaStream_t st);
 

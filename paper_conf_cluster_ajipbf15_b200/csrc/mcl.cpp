@@ -139,6 +139,7 @@ struct mcl_mapper {
   uint32_t* flags_host = nullptr;               // host-mapped status word
   uint32_t* flags_dev = nullptr;
   int timing = 0;               // 0 off, 1 search kernel, 2 search kernel + whole call
+  uint32_t hold_us = 0;         // timing aid: spin kernel ahead of the start event
   bool timing_pending = false;  // events recorded, elapsed times not read yet
   int force_path = 0;
   cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
@@ -344,6 +345,12 @@ mcl_status_t mcl_last_launch_info(const mcl_mapper_t* h, int64_t info[8]) {
   return MCL_OK;
 }
 
+mcl_status_t mcl_set_timing_hold(mcl_mapper_t* h, uint32_t hold_us) {
+  if (!h || hold_us > 1000000u) return MCL_E_INVAL;
+  h->hold_us = hold_us;
+  return MCL_OK;
+}
+
 mcl_status_t mcl_set_timing(mcl_mapper_t* h, int enable) {
   if (!h) return MCL_E_INVAL;
   if (enable < 0 || enable > 2) return MCL_E_INVAL;
@@ -499,6 +506,16 @@ mcl_status_t status_from_flags(mcl_mapper* h) {
 
 void clear_flags(mcl_mapper* h) { *(volatile uint32_t*)h->flags_host = 0; }
 
+// start event of a timed launch; with a hold the stream is kept busy until the launch is
+// enqueued, so the events bracket device execution only (mcl_set_timing_hold)
+cudaError_t record_start(mcl_mapper* h, cudaStream_t s) {
+  if (h->hold_us) {
+    const cudaError_t e = mcl::launch_hold((uint64_t)h->hold_us * 1000u, s);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaEventRecord(h->ev[0], s);
+}
+
 mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
                       const uint64_t* cost_kernel, const uint64_t* cost_xfer,
                       const uint64_t* base_load, const uint16_t* eligible,
@@ -587,7 +604,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
     nlaunch = 0;
     dim3 grid(1, 1, 1);
     int threads = 0;
-    if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[0], s), "cudaEventRecord");
+    if (h->timing) MCL_CUDA(h, record_start(h, s), "cudaEventRecord(start)");
     if (path == 4) {
       mcl::SmallArgs a{Q, D, epochs, K, X, o_idx, o_ms, o_map, h->flags_dev};
       int gx = 0;
@@ -910,7 +927,7 @@ mcl_status_t mcl_map_queues_pruned(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint
     a.scratch = (Cand*)h->scratch.p;
   }
   clear_flags(h);
-  if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[0], s), "cudaEventRecord");
+  if (h->timing) MCL_CUDA(h, record_start(h, s), "cudaEventRecord(start)");
   MCL_CUDA(h, mcl::launch_bnb(a, grid, threads, s), "search_bnb launch");
   if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[1], s), "cudaEventRecord");
   uint64_t nodes = 0;
@@ -1011,7 +1028,7 @@ mcl_status_t mcl_build_costs(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t e
     Xd = (uint64_t*)h->cost_x.p;
   }
   clear_flags(h);
-  if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[0], h->stream), "cudaEventRecord");
+  if (h->timing) MCL_CUDA(h, record_start(h, h->stream), "cudaEventRecord(start)");
   if ((st = build_costs_dev(h, Q, D, epochs, model, Kd, Xd)) != MCL_OK) return st;
   if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[1], h->stream), "cudaEventRecord");
   if (!dk) MCL_CUDA(h, cudaMemcpyAsync(cost_kernel, Kd, out_bytes, cudaMemcpyDeviceToHost, h->stream), "D2H");

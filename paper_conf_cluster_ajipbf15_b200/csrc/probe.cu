@@ -121,4 +121,20 @@ cudaError_t probe_alu(int op, int sms, cudaStream_t st, double* rate, double* pe
   }
 }
 
+// Timing aid (mcl_set_timing_hold): keeps the stream busy while the host enqueues the
+// start event and the search launch, so the events measure device execution only.
+__global__ void hold_kernel(uint64_t ns) {
+  uint64_t t0, t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  do {
+    __nanosleep(500);
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  } while (t - t0 < ns);
+}
+
+cudaError_t launch_hold(uint64_t ns, cudaStream_t st) {
+  hold_kernel<<<1, 1, 0, st>>>(ns);
+  return cudaGetLastError();
+}
+
 }  // namespace mcl

@@ -24,7 +24,7 @@ PATH_NAMES = {1: "blocked_u32", 2: "blocked_u64", 3: "generic", 4: "small_batche
 EXPORTED = [
     "mcl_mapper_create", "mcl_map_queues", "mcl_mapper_destroy", "mcl_status_string",
     "mcl_last_error_string", "mcl_last_launch_info", "mcl_version",
-    "mcl_set_timing", "mcl_last_kernel_time", "mcl_force_path", "mcl_probe_int_rate",
+    "mcl_set_timing", "mcl_set_timing_hold", "mcl_last_kernel_time", "mcl_force_path", "mcl_probe_int_rate",
     "mcl_device_sms",
     "mcl_comm_unique_id", "mcl_comm_init", "mcl_comm_destroy",
     "mcl_map_queues_constrained", "mcl_score_mappings", "mcl_map_queues_pruned",
@@ -92,6 +92,7 @@ def load_library(path: str | None = None) -> ctypes.CDLL:
         "mcl_last_launch_info": (i32, [vp, ctypes.POINTER(ctypes.c_int64)]),
         "mcl_version": (ctypes.c_char_p, []),
         "mcl_set_timing": (i32, [vp, i32]),
+        "mcl_set_timing_hold": (i32, [vp, u32]),
         "mcl_force_path": (i32, [vp, i32]),
         "mcl_last_kernel_time": (i32, [vp, ctypes.POINTER(ctypes.c_float), ctypes.POINTER(ctypes.c_float)]),
         "mcl_probe_int_rate": (i32, [i32, i32, ctypes.POINTER(ctypes.c_double),
@@ -460,8 +461,12 @@ class Mapper:
         if st != MCL_OK:
             raise MclError(st, "mcl_force_path")
 
-    def set_timing(self, enable: bool = True) -> None:
-        load_library().mcl_set_timing(self.handle, 1 if enable else 0)
+    def set_timing(self, enable: bool = True, hold_us: int = 0) -> None:
+        """CUDA-event timing of the search kernel; hold_us > 0 precedes each timed launch
+        with a spin kernel so the events exclude host launch latency (measurement only)."""
+        lib = load_library()
+        lib.mcl_set_timing(self.handle, 1 if enable else 0)
+        lib.mcl_set_timing_hold(self.handle, int(hold_us))
 
     def last_kernel_time_ms(self) -> tuple[float, float]:
         k, c = ctypes.c_float(), ctypes.c_float()

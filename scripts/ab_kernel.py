@@ -1,0 +1,73 @@
+"""A/B kernel timing of several builds of libmcl.so on the same GPU (not the bench line).
+
+    python scripts/ab_kernel.py --libs ab/libmcl_head.so paper_conf_cluster_ajipbf15_b200/libmcl.so \
+        --workloads cfg5 cfg4 cfg2 --rounds 3
+
+Each (round, library) pair runs in its own subprocess (the binding loads one library per
+process); libraries alternate within a round so clock drift hits them alike. Prints the
+median kernel time (CUDA events around the search launch) per library and workload, and
+checks that every build returns the same result.
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+CHILD = r"""
+import json, sys, statistics
+sys.path.insert(0, {root!r})
+import torch
+from paper_conf_cluster_ajipbf15_b200 import mcl, Mapper, workloads
+mcl.load_library({lib!r})
+out = {{}}
+with Mapper(0) as m:
+    m.set_timing(1)
+    for name in {wls!r}:
+        K, X = workloads.make(name)
+        Kd, Xd = torch.from_numpy(K).cuda(), torch.from_numpy(X).cuda()
+        reps = 5 if name == "cfg5" else 20
+        for _ in range(3):
+            idx, mp, ms = m.map_queues(Kd, Xd)
+        ts = []
+        for _ in range(reps):
+            idx, mp, ms = m.map_queues(Kd, Xd)
+            ts.append(m.last_kernel_time_ms()[0])
+        out[name] = {{"ms": statistics.median(ts), "min": min(ts),
+                      "res": [int(idx[:64].sum()), int(ms[:64].sum())]}}
+print(json.dumps(out))
+"""
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--libs", nargs="+", required=True)
+    ap.add_argument("--workloads", nargs="+", default=["cfg5", "cfg4", "cfg2"])
+    ap.add_argument("--rounds", type=int, default=3)
+    args = ap.parse_args()
+    res = {lib: {w: [] for w in args.workloads} for lib in args.libs}
+    results = {}
+    for r in range(args.rounds):
+        for lib in (args.libs if r % 2 == 0 else args.libs[::-1]):
+            code = CHILD.format(root=ROOT, lib=os.path.abspath(lib), wls=args.workloads)
+            p = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True)
+            if p.returncode:
+                print(lib, "failed:", p.stderr[-2000:])
+                continue
+            d = json.loads(p.stdout.strip().splitlines()[-1])
+            for w, v in d.items():
+                res[lib][w].append(v["ms"])
+                results.setdefault(w, set()).add(tuple(v["res"]))
+    for w in args.workloads:
+        line = {"workload": w, "same_result": len(results.get(w, ())) == 1}
+        for lib in args.libs:
+            line[os.path.basename(lib)] = {"median_ms": statistics.median(res[lib][w]) if res[lib][w] else None,
+                                           "all": [round(x, 4) for x in res[lib][w]]}
+        print(json.dumps(line), flush=True)
+
+
+if __name__ == "__main__":
+    main()
