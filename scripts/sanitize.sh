@@ -5,7 +5,7 @@ mkdir -p gpurun_out
 CS=/usr/local/cuda/bin/compute-sanitizer
 run() {  # tool, workload, reps, [epochs]
   timeout 900 $CS --tool $1 --error-exitcode 9 python scripts/profile_run.py $2 $3 $4 > gpurun_out/sanitize_$1_$2.log 2>&1
-  echo "$1 $2 rc=$? $(grep -c 'ERROR SUMMARY: 0 errors' gpurun_out/sanitize_$1_$2.log) $(grep 'ERROR SUMMARY' gpurun_out/sanitize_$1_$2.log | tail -1)"
+  echo "$1 $2 rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY' gpurun_out/sanitize_$1_$2.log | tail -1)"
 }
 for tool in memcheck racecheck synccheck; do
   run $tool cfg1 1
