@@ -46,7 +46,9 @@ mcl_status_t mcl_probe_int_rate(int device, int op, double* lane_ops_per_s,
    (default), 1 = register-blocked (u32 loads, falls back to 64-bit when a bound needs it),
    2 = register-blocked with 64-bit loads, 3 = generic, 4 = small batched, 5 = register-
    blocked u32 over a flattened (epoch, block) space (batched calls), 6 = always run the
-   branch-and-bound kernel in mcl_map_queues_pruned (no small-space cutover). A path that does
+   branch-and-bound kernel in mcl_map_queues_pruned (no small-space cutover), 7 = warp-per-
+   epoch batched kernel (unconstrained single-GPU batches of the shapes it is instantiated
+   for; chosen automatically from one full wave of epochs). A path that does
    not support (Q, D) or the handle's sharding makes the call fail with MCL_E_INVAL. */
 mcl_status_t mcl_force_path(mcl_mapper_t* h, int path);
 

@@ -210,6 +210,22 @@ cudaError_t launch_score(uint32_t Q, uint32_t D, uint64_t E, const uint64_t* K, 
 cudaError_t launch_generic(const GenericArgs& a, dim3 grid, int threads, size_t smem,
                            cudaStream_t st);
 
+// Batched search, one warp per epoch, compile-time (Q, D) (search_batch.cu): u32 loads,
+// unconstrained, single GPU, shapes with >= ~32 chunks of D^2 blocks per epoch.
+struct BatchArgs {
+  uint32_t Q, D;
+  uint64_t E;
+  const uint64_t* K;
+  const uint64_t* X;
+  uint64_t* index;
+  uint64_t* makespan;
+  uint8_t* mapping;
+  volatile uint32_t* flags;
+  uint32_t one;
+};
+bool batch_supported(uint32_t Q, uint32_t D);
+cudaError_t launch_batch(const BatchArgs& a, int num_sms, cudaStream_t st, int* grid_out);
+
 // Small batched search (search_small.cu): one thread per epoch, tiles staged in shared
 // memory by cp.async.bulk (TMA bulk copy). Instantiated for a few (Q, D) shapes.
 struct SmallArgs {

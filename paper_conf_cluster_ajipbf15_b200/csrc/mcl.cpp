@@ -360,7 +360,7 @@ mcl_status_t mcl_set_timing(mcl_mapper_t* h, int enable) {
 }
 
 mcl_status_t mcl_force_path(mcl_mapper_t* h, int path) {
-  if (!h || path < 0 || path > 6) return MCL_E_INVAL;
+  if (!h || path < 0 || path > 7) return MCL_E_INVAL;
   h->force_path = path;
   return MCL_OK;
 }
@@ -582,12 +582,16 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
   const bool shard_mode = h->world > 1;  // NCCL collective or single-GPU shard test
   // the small and flattened kernels take no constraints; the blocked and generic ones do
   int path;
+  // warp-per-epoch kernel: batches of at least one full wave of warps (16 per SM)
+  const bool batch_ok = !shard_mode && !multi && !constrained && mcl::batch_supported(Q, D);
   if (!shard_mode && !multi && !constrained && mcl::small_supported(Q, D)) path = 4;
+  else if (batch_ok && epochs >= (uint64_t)h->num_sms * 16) path = 7;
   else if (mcl::blocked_supported(Q, D)) path = 1;
   else path = 3;
   if (h->force_path && h->force_path != 6) {  // 6 only affects mcl_map_queues_pruned
     const int f = h->force_path;
     const bool ok = (f == 3) || ((f == 1 || f == 2) && mcl::blocked_supported(Q, D)) ||
+                    (f == 7 && batch_ok) ||
                     (f == 5 && epochs > 1 && !shard_mode && !multi && !constrained &&
                      mcl::flat_supported(Q, D, mcl::index_bits_host(N))) ||
                     (f == 4 && !shard_mode && !multi && !constrained && mcl::small_supported(Q, D));
@@ -605,7 +609,13 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
     dim3 grid(1, 1, 1);
     int threads = 0;
     if (h->timing) MCL_CUDA(h, record_start(h, s), "cudaEventRecord(start)");
-    if (path == 4) {
+    if (path == 7) {
+      mcl::BatchArgs a{Q, D, epochs, K, X, o_idx, o_ms, o_map, h->flags_dev, 1u};
+      int gx = 0;
+      MCL_CUDA(h, mcl::launch_batch(a, h->num_sms, s, &gx), "search_batch launch");
+      grid.x = gx;
+      threads = 128;
+    } else if (path == 4) {
       mcl::SmallArgs a{Q, D, epochs, K, X, o_idx, o_ms, o_map, h->flags_dev};
       int gx = 0;
       MCL_CUDA(h, mcl::launch_small(a, h->num_sms, s, &gx, &threads), "search_small launch");
@@ -727,7 +737,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
       h->info[6] = (flags & mcl::kFlagTwoStep) ? 1 : 0;
     }
     if (flags & mcl::kFlagNeedU64) {  // some epoch's bound needs 64-bit loads: rerun the wide kernel
-      if (path != 1 && path != 5) {
+      if (path != 1 && path != 5 && path != 7) {
         h->last_err = "internal: 64-bit request from a 64-bit kernel";
         return MCL_E_CUDA;
       }

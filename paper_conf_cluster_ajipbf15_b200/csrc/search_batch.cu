@@ -1,0 +1,235 @@
+// search_batch.cu -- batched exhaustive search, one WARP per epoch with compile-time
+// (Q, D) (cfg2: 8 queues x 4 devices x 10^4 epochs).
+//
+// Same scoring core as search_blocked.cu (blocked_core.cuh: the D^4 leaves of a
+// super-block folded into one running minimum, one integer max per mapping; PAPER.md
+// L1048-1052 loads / makespan, L2106-2118 C = K + X), but the per-epoch work around it is
+// cut to what a warp-sized epoch needs, because with 4^8 = 65,536 mappings per epoch that
+// setup is a fifth of the instructions in the CTA-per-epoch kernel:
+//   * persistent warps stride over the epochs; the next epoch's K and X are loaded into
+//     registers while the current one is searched (no load latency in the prologue);
+//   * no __syncthreads, no shared atomics: everything is warp-synchronous;
+//   * the chunk digits (queues 0..Q-6) come from compile-time divisions of the chunk
+//     index, the one-hot prefix vectors from selects on the cost table -- no outer tables;
+//   * lane l walks chunks l, l + 32, ... (D^2 blocks each, the super-block path), keeping
+//     the first strict minimum of its own increasing sequence; the warp takes the
+//     lexicographic minimum of (makespan, super-block index), and re-scans only that
+//     super-block (block by block, 32 leaves per ballot) for the lowest leaf index.
+// Mapping index m = ((chunk * D + y) * D + x) * D^3 + leaf, queue 0 most significant
+// (R6): chunk = digits of queues 0..Q-6, y = queue Q-5, x = queue Q-4, leaf =
+// queues Q-3..Q-1.
+#include "blocked_core.cuh"
+
+namespace mcl {
+
+namespace {
+
+template <int B, int E>
+struct IPow {
+  static constexpr uint64_t v = (uint64_t)B * IPow<B, E - 1>::v;
+};
+template <int B>
+struct IPow<B, 0> {
+  static constexpr uint64_t v = 1;
+};
+
+constexpr int kBatchWarps = 4;  // warps per CTA (each its own epochs)
+
+}  // namespace
+
+template <int Q, int D>
+__global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(BatchArgs a) {
+  using T = uint32_t;
+  constexpr int QD = Q * D;
+  constexpr uint32_t kChunks = (uint32_t)IPow<D, Q - 5>::v;  // chunks of D^2 blocks per epoch
+  static_assert(QD <= 64, "two cost entries per lane");
+  static_assert(Q >= 6, "chunks need queues 0..Q-6");
+  __shared__ __align__(16) uint64_t sC64[kBatchWarps][QD];
+  __shared__ __align__(16) T sC[kBatchWarps][QD];
+  __shared__ __align__(16) T sIn[kBatchWarps][8 * D];
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  uint64_t* C64 = sC64[wib];
+  T* Cs = sC[wib];
+  T* in = sIn[wib];
+  const uint32_t one = a.one;
+  const uint64_t nwarps = (uint64_t)gridDim.x * kBatchWarps;
+  uint64_t e = (uint64_t)blockIdx.x * kBatchWarps + wib;
+
+  // prefetch of epoch e's costs: entries lane and lane + 32
+  uint64_t k0 = 0, x0 = 0, k1 = 0, x1 = 0;
+  auto prefetch = [&](uint64_t ep) {
+    const uint64_t* Ke = a.K + ep * QD;
+    const uint64_t* Xe = a.X + ep * QD;
+    if (lane < QD) { k0 = Ke[lane]; x0 = Xe[lane]; }
+    if (lane + 32 < QD) { k1 = Ke[lane + 32]; x1 = Xe[lane + 32]; }
+  };
+  if (e < a.E) prefetch(e);
+
+  for (; e < a.E; e += nwarps) {
+    // ---- a1: C = K + X, range check, bound UB = sum_q max_d C (decides 32-bit loads) ----
+    bool bad = false;
+    if (lane < QD) {
+      bad |= (k0 >= kEntryLimit) | (x0 >= kEntryLimit);
+      C64[lane] = k0 + x0;
+    }
+    if (lane + 32 < QD) {
+      bad |= (k1 >= kEntryLimit) | (x1 >= kEntryLimit);
+      C64[lane + 32] = k1 + x1;
+    }
+    if (e + nwarps < a.E) prefetch(e + nwarps);  // travels while this epoch is searched
+    __syncwarp();
+    uint64_t row = 0;
+    if (lane < Q) {
+#pragma unroll
+      for (int d = 0; d < D; ++d) row = max(row, C64[lane * D + d]);
+    }
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) row += __shfl_xor_sync(0xffffffffu, row, off);
+    if (__any_sync(0xffffffffu, bad)) {
+      if (lane == 0) raise_flag(a.flags, kFlagRange);
+      continue;
+    }
+    if (row >= (1ull << 32)) {
+      if (lane == 0) raise_flag(a.flags, kFlagNeedU64);
+      continue;
+    }
+    // ---- tables: composed costs (u32) and the inner queues' sums ----
+    if (lane < QD) Cs[lane] = (T)C64[lane];
+    if (lane + 32 < QD) Cs[lane + 32] = (T)C64[lane + 32];
+    if (lane < D) {
+      const T A = (T)C64[(Q - 3) * D + lane], B = (T)C64[(Q - 2) * D + lane], Cc = (T)C64[(Q - 1) * D + lane];
+      in[0 * D + lane] = A;
+      in[1 * D + lane] = B;
+      in[2 * D + lane] = Cc;
+      in[3 * D + lane] = A + B;
+      in[4 * D + lane] = A + Cc;
+      in[5 * D + lane] = B + Cc;
+      in[6 * D + lane] = A + B + Cc;
+      in[7 * D + lane] = (T)C64[(Q - 4) * D + lane];
+    }
+    __syncwarp();
+    const T* c4 = in + 7 * D;
+    const T* Cy = Cs + (Q - 5) * D;
+
+    // prefix loads of chunk c: one-hot costs of queues 0..Q-6 on their digits' devices
+    auto chunk_base = [&](uint32_t c, T (&b)[D]) {
+#pragma unroll
+      for (int d = 0; d < D; ++d) b[d] = 0;
+#pragma unroll
+      for (int q = Q - 6; q >= 0; --q) {
+        const uint32_t dq = c % D;
+        c /= D;
+#pragma unroll
+        for (int d = 0; d < D; ++d) b[d] = add_f(b[d], (dq == (uint32_t)d) ? Cs[q * D + d] : T(0), one);
+      }
+    };
+
+    // ---- a2-a5: lane l walks chunks l, l + 32, ... (increasing) ----
+    T best = ~T(0);
+    uint32_t best_sb = 0xffffffffu;  // super-block index within the epoch: chunk * D + y
+    for (uint32_t c = lane; c < kChunks; c += 32) {
+      T base2[D];
+      chunk_base(c, base2);
+      for (int y = 0; y < D; ++y) {
+        const T cy = Cy[y];
+        T base[D];
+#pragma unroll
+        for (int d = 0; d < D; ++d) base[d] = add_f(base2[d], (y == d) ? cy : T(0), one);
+        const T gs = superblock_eval<T, D>(base, in, c4, one);
+        if (gs < best) {
+          best = gs;
+          best_sb = c * D + (uint32_t)y;
+        }
+      }
+    }
+    // ---- warp argmin on (makespan, super-block), then the lowest leaf inside it ----
+    uint64_t key = ((uint64_t)best << 32) | best_sb;
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) key = min(key, __shfl_xor_sync(0xffffffffu, key, off));
+    const T target = (T)(key >> 32);
+    const uint32_t sb = (uint32_t)key;
+    T base[D];
+    {
+      T base2[D];
+      chunk_base(sb / D, base2);
+      const uint32_t y = sb % D;
+#pragma unroll
+      for (int d = 0; d < D; ++d) base[d] = add_f(base2[d], (y == (uint32_t)d) ? Cy[y] : T(0), one);
+    }
+    uint64_t idx = kNone;
+    for (int x = 0; x < D; ++x) {
+      T P[D];
+#pragma unroll
+      for (int d = 0; d < D; ++d) P[d] = (x == d) ? base[d] + c4[d] : base[d];
+      const uint32_t leaf = block_first_warp<T, D>(P, in, target);
+      if (leaf != 0xffffffffu) {
+        idx = ((uint64_t)sb * D + (uint64_t)x) * (uint64_t)(D * D * D) + leaf;
+        break;
+      }
+    }
+    // ---- a7: outputs (digits of the index, queue 0 most significant) ----
+    if (lane == 0) {
+      a.index[e] = idx;
+      a.makespan[e] = (uint64_t)target;
+    }
+    if (a.mapping && lane < Q) {
+      uint64_t rest = idx;
+      for (int q = Q - 1; q > lane; --q) rest /= D;
+      a.mapping[e * Q + lane] = (uint8_t)(rest % D);
+    }
+  }
+}
+
+namespace {
+template <int Q, int D>
+cudaError_t launch_batch_t(const BatchArgs& a, int num_sms, cudaStream_t st, int* grid_out) {
+  auto k = search_batch_kernel<Q, D>;
+  static std::atomic<int> occ[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int per_sm = occ[dev & 63].load(std::memory_order_relaxed);
+  if (per_sm == 0) {
+    cudaError_t err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, 32 * kBatchWarps, 0);
+    if (err != cudaSuccess) return err;
+    if (per_sm < 1) per_sm = 1;
+    occ[dev & 63].store(per_sm, std::memory_order_relaxed);
+  }
+  const uint64_t ctas_needed = (a.E + kBatchWarps - 1) / kBatchWarps;
+  uint64_t grid = (uint64_t)num_sms * per_sm;
+  if (grid > ctas_needed) grid = ctas_needed;
+  k<<<(unsigned)grid, 32 * kBatchWarps, 0, st>>>(a);
+  *grid_out = (int)grid;
+  return cudaGetLastError();
+}
+}  // namespace
+
+// Shapes with a warp-per-epoch instantiation: >= 32 chunks per epoch (every lane busy),
+// at most 2^26 mappings per epoch (a warp-sized epoch), QD <= 64.
+bool batch_supported(uint32_t Q, uint32_t D) {
+  switch (Q * 100 + D) {
+    case 803: case 903: case 1003: case 1103:  // D = 3: 3^(Q-5) >= 27 ... lanes mostly busy
+    case 804: case 904: case 1004: case 1104:
+    case 805: case 905:
+      return true;
+    default:
+      return false;
+  }
+}
+
+cudaError_t launch_batch(const BatchArgs& a, int num_sms, cudaStream_t st, int* grid_out) {
+  switch (a.Q * 100 + a.D) {
+    case 803: return launch_batch_t<8, 3>(a, num_sms, st, grid_out);
+    case 903: return launch_batch_t<9, 3>(a, num_sms, st, grid_out);
+    case 1003: return launch_batch_t<10, 3>(a, num_sms, st, grid_out);
+    case 1103: return launch_batch_t<11, 3>(a, num_sms, st, grid_out);
+    case 804: return launch_batch_t<8, 4>(a, num_sms, st, grid_out);
+    case 904: return launch_batch_t<9, 4>(a, num_sms, st, grid_out);
+    case 1004: return launch_batch_t<10, 4>(a, num_sms, st, grid_out);
+    case 1104: return launch_batch_t<11, 4>(a, num_sms, st, grid_out);
+    case 805: return launch_batch_t<8, 5>(a, num_sms, st, grid_out);
+    case 905: return launch_batch_t<9, 5>(a, num_sms, st, grid_out);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+}  // namespace mcl

@@ -1,0 +1,130 @@
+"""GPU parity of the warp-per-epoch batched kernel (search_batch.cu, force_path 7) against
+the CPU oracle, bit-exact, on every (Q, D) it is instantiated for; plus its automatic
+selection, the 64-bit rerun, range errors and ragged batches. Run with ``pytest -m gpu``.
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import oracle
+from conftest import cuda_available
+from paper_conf_cluster_ajipbf15_b200 import workloads
+from paper_conf_cluster_ajipbf15_b200.mcl import MCL_E_RANGE, Mapper, MclError
+
+pytestmark = pytest.mark.gpu
+
+BATCH_SHAPES = [(8, 3), (9, 3), (10, 3), (11, 3), (8, 4), (9, 4), (10, 4), (11, 4), (8, 5), (9, 5)]
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    if not cuda_available():
+        pytest.fail("no CUDA device: the -m gpu tests must run on a GPU box")
+    import torch
+
+    return torch
+
+
+@pytest.fixture(scope="module")
+def mapper(torch_cuda):
+    m = Mapper(0)
+    yield m
+    m.close()
+
+
+def run(torch, mp, K, X, path):
+    mp.force_path(path)
+    try:
+        idx, mapping, ms = mp.map_queues(torch.from_numpy(np.ascontiguousarray(K)).cuda(),
+                                         torch.from_numpy(np.ascontiguousarray(X)).cuda())
+        info = mp.launch_info()
+    finally:
+        mp.force_path(0)
+    return (idx.cpu().numpy(), mapping.cpu().numpy(), ms.cpu().numpy()), info
+
+
+def check(got, want, ctx):
+    gi, gmp, gms = got
+    wi, wms, wmp = want
+    bad = np.nonzero((gi != wi) | (gms != wms))[0]
+    assert bad.size == 0, f"{ctx}: {bad.size} epochs differ, first {bad[:5]}: gpu {gi[bad[:5]]}/{gms[bad[:5]]} oracle {wi[bad[:5]]}/{wms[bad[:5]]}"
+    assert (gmp == wmp).all(), ctx
+
+
+@pytest.mark.parametrize("Q,D", BATCH_SHAPES)
+def test_batch_kernel_shapes(torch_cuda, mapper, Q, D):
+    # E not a multiple of the 4 warps per CTA; fewer epochs for the large index spaces
+    E = 37 if D**Q <= 300_000 else 5
+    for seed, maker in ((50 * Q + D, workloads.random_tables), (900 + 50 * Q + D, workloads.small_int_tables)):
+        K, X = maker(seed, E, Q, D)
+        got, info = run(torch_cuda, mapper, K, X, 7)
+        assert info["path"] == "batch_u32"
+        check(got, oracle.oracle_map(K, X), f"Q={Q} D={D} {maker.__name__}")
+
+
+def test_batch_degenerate_ties(torch_cuda, mapper):
+    """All-zero, all-equal and one-hot-cheap epochs side by side in one batch."""
+    for Q, D in ((8, 4), (9, 3), (8, 5)):
+        zeros = np.zeros((1, Q, D), np.uint64)
+        eq = np.full((1, Q, D), 7, np.uint64)
+        hot = np.full((1, Q, D), 1000, np.uint64)
+        hot[0, :, D - 1] = 1
+        K = np.concatenate([zeros, eq, hot, eq, zeros])
+        X = np.zeros_like(K)
+        got, _ = run(torch_cuda, mapper, K, X, 7)
+        check(got, oracle.oracle_map(K, X), f"{Q}x{D} ties")
+
+
+def test_batch_auto_selection_cfg2(torch_cuda, mapper):
+    """cfg2 (10^4 epochs >= one wave of warps) runs the batched kernel automatically and
+    agrees with the CTA-per-epoch kernel and the oracle on every epoch."""
+    K, X = workloads.cfg2()
+    want = oracle.oracle_map(K, X)
+    got, info = run(torch_cuda, mapper, K, X, 0)
+    assert info["path"] == "batch_u32", info
+    check(got, want, "cfg2 auto")
+    got, info = run(torch_cuda, mapper, K, X, 1)
+    assert info["path"] == "blocked_u32"
+    check(got, want, "cfg2 CTA per epoch")
+    # a batch below one wave keeps the CTA-per-epoch kernel (it splits epochs over CTAs)
+    got, info = run(torch_cuda, mapper, K[:100], X[:100], 0)
+    assert info["path"] == "blocked_u32", info
+    check(got, tuple(w[:100] for w in want), "cfg2[:100]")
+
+
+def test_batch_u64_rerun(torch_cuda, mapper):
+    """A batch whose bound needs 64-bit loads is detected on the device and rerun with the
+    64-bit blocked kernel (mixed with ordinary epochs)."""
+    K, X = workloads.random_tables(71, 9, 8, 4)
+    K[4] = np.random.default_rng(1).integers(1 << 46, 1 << 47, size=(8, 4), dtype=np.uint64)
+    got, info = run(torch_cuda, mapper, K, X, 7)
+    assert info["path"] == "blocked_u64"
+    check(got, oracle.oracle_map(K, X), "u64 rerun")
+
+
+def test_batch_range_error(torch_cuda, mapper):
+    K, X = workloads.random_tables(72, 6, 8, 4)
+    X[3, 2, 1] = 1 << 48
+    with pytest.raises(MclError) as ei:
+        run(torch_cuda, mapper, K, X, 7)
+    assert ei.value.status == MCL_E_RANGE
+
+
+def test_batch_single_epoch_and_no_mapping_output(torch_cuda, mapper):
+    torch = torch_cuda
+    K, X = workloads.random_tables(73, 1, 9, 4)
+    got, _ = run(torch, mapper, K, X, 7)
+    check(got, oracle.oracle_map(K, X), "E=1")
+    # mapping output optional (NULL): index and makespan only
+    K, X = workloads.random_tables(74, 11, 8, 4)
+    Kd, Xd = torch.from_numpy(K).cuda(), torch.from_numpy(X).cuda()
+    idx = torch.empty(11, dtype=torch.uint64, device="cuda")
+    ms = torch.empty(11, dtype=torch.uint64, device="cuda")
+    mapper.force_path(7)
+    try:
+        mapper.map_queues_into(Kd, Xd, idx, None, ms)
+    finally:
+        mapper.force_path(0)
+    wi, wms, _ = oracle.oracle_map(K, X)
+    assert (idx.cpu().numpy() == wi).all() and (ms.cpu().numpy() == wms).all()
