@@ -90,8 +90,16 @@ struct DevBuf {
     cudaError_t e = cudaMalloc(&p, want);
     if (e != cudaSuccess) return e;
     cap = want;
-    if (zero) return cudaMemset(p, 0, want);
+    if (zero) return fill(0);
     return cudaSuccess;
+  }
+  // Fill the whole buffer before any later launch can read it: the memset runs on the
+  // legacy stream, which a non-blocking stream (the handle's, or torch's) does not wait
+  // for, so the device is synchronised here (buffers grow rarely; not on the hot path).
+  cudaError_t fill(int byte) {
+    cudaError_t e = cudaMemset(p, byte, cap);
+    if (e != cudaSuccess) return e;
+    return cudaDeviceSynchronize();
   }
   void release() {
     if (p) cudaFree(p);
@@ -126,6 +134,7 @@ struct mcl_mapper {
   DevBuf done;             // uint32 per epoch, zero between calls
   DevBuf key, pair, gms, cand;
   DevBuf flat_keys, flat_done;  // flattened batched kernel: per-epoch key / block count
+  DevBuf batch_keys, batch_done;  // warp-per-epoch kernel: split epochs' key / piece count
   DevBuf bnb_next, bnb_inc, bnb_nodes;  // pruned search: subtree counters, incumbents, nodes
   DevBuf model_buf[9], cost_k, cost_x;  // cost-table construction: staged model, built K / X
   DevBuf in_k, in_x, in_base, in_elig, out_idx, out_ms, out_map;  // staging for host pointers
@@ -326,7 +335,7 @@ void mcl_mapper_destroy(mcl_mapper_t* h) {
     for (void* p : h->peer_opened) cudaIpcCloseMemHandle(p);
     for (DevBuf* b : {&h->peer_slab, &h->peer_kdone, &h->peer_gms, &h->peer_ptrs}) b->release();
     for (DevBuf* b : {&h->scratch, &h->done, &h->key, &h->pair, &h->gms, &h->cand, &h->flat_keys,
-                      &h->flat_done, &h->bnb_next, &h->bnb_inc, &h->bnb_nodes, &h->in_k,
+                      &h->flat_done, &h->batch_keys, &h->batch_done, &h->bnb_next, &h->bnb_inc, &h->bnb_nodes, &h->in_k,
                       &h->in_base, &h->in_elig,
                       &h->in_x, &h->out_idx, &h->out_ms, &h->out_map, &h->cost_k, &h->cost_x})
       b->release();
@@ -611,6 +620,13 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
     if (h->timing) MCL_CUDA(h, record_start(h, s), "cudaEventRecord(start)");
     if (path == 7) {
       mcl::BatchArgs a{Q, D, epochs, K, X, o_idx, o_ms, o_map, h->flags_dev, 1u};
+      if (h->batch_keys.cap < epochs * 8) {
+        MCL_CUDA(h, h->batch_keys.ensure(epochs * 8), "cudaMalloc(batch keys)");
+        MCL_CUDA(h, h->batch_keys.fill(0xff), "cudaMemset(batch keys)");
+      }
+      MCL_CUDA(h, h->batch_done.ensure(epochs * 4, true), "cudaMalloc(batch done)");
+      a.keys = (uint64_t*)h->batch_keys.p;
+      a.done = (uint32_t*)h->batch_done.p;
       int gx = 0;
       MCL_CUDA(h, mcl::launch_batch(a, h->num_sms, s, &gx), "search_batch launch");
       grid.x = gx;
@@ -630,7 +646,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
       a.ibits = ibits; a.out = out; a.flags = h->flags_dev; a.one = 1;
       if (h->flat_keys.cap < epochs * 8) {
         MCL_CUDA(h, h->flat_keys.ensure(epochs * 8), "cudaMalloc(keys)");
-        MCL_CUDA(h, cudaMemset(h->flat_keys.p, 0xff, h->flat_keys.cap), "cudaMemset(keys)");
+        MCL_CUDA(h, h->flat_keys.fill(0xff), "cudaMemset(keys)");
       }
       MCL_CUDA(h, h->flat_done.ensure(epochs * 8, true), "cudaMalloc(done_blocks)");
       a.keys = (uint64_t*)h->flat_keys.p;
@@ -903,7 +919,7 @@ mcl_status_t mcl_map_queues_pruned(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint
   if (h->bnb_next.cap < epochs * 8) {
     MCL_CUDA(h, h->bnb_next.ensure(epochs * 8, true), "cudaMalloc(bnb)");
     MCL_CUDA(h, h->bnb_inc.ensure(epochs * 8), "cudaMalloc(bnb)");
-    MCL_CUDA(h, cudaMemset(h->bnb_inc.p, 0xff, h->bnb_inc.cap), "cudaMemset(bnb)");
+    MCL_CUDA(h, h->bnb_inc.fill(0xff), "cudaMemset(bnb)");
   }
   MCL_CUDA(h, h->bnb_nodes.ensure(8, true), "cudaMalloc(bnb)");
   MCL_CUDA(h, cudaMemsetAsync(h->bnb_nodes.p, 0, 8, s), "cudaMemset(bnb)");

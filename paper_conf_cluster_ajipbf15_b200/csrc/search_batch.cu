@@ -18,6 +18,8 @@
 // Mapping index m = ((chunk * D + y) * D + x) * D^3 + leaf, queue 0 most significant
 // (R6): chunk = digits of queues 0..Q-6, y = queue Q-5, x = queue Q-4, leaf =
 // queues Q-3..Q-1.
+#include <algorithm>
+
 #include "blocked_core.cuh"
 
 namespace mcl {
@@ -53,19 +55,52 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
   T* in = sIn[wib];
   const uint32_t one = a.one;
   const uint64_t nwarps = (uint64_t)gridDim.x * kBatchWarps;
-  uint64_t e = (uint64_t)blockIdx.x * kBatchWarps + wib;
+  // Work units: epochs 0..e_full-1 whole (one warp each); each remaining epoch in `pieces`
+  // contiguous super-block ranges (the last, partial wave spread over all warps).
+  const uint64_t nunits = a.e_full + (a.E - a.e_full) * a.pieces;
+  auto epoch_of = [&](uint64_t u) -> uint64_t {
+    return u < a.e_full ? u : a.e_full + (u - a.e_full) / a.pieces;
+  };
 
-  // prefetch of epoch e's costs: entries lane and lane + 32
+  // prefetch of a unit's epoch costs: entries lane and lane + 32
   uint64_t k0 = 0, x0 = 0, k1 = 0, x1 = 0;
-  auto prefetch = [&](uint64_t ep) {
+  auto prefetch = [&](uint64_t u) {
+    const uint64_t ep = epoch_of(u);
     const uint64_t* Ke = a.K + ep * QD;
     const uint64_t* Xe = a.X + ep * QD;
     if (lane < QD) { k0 = Ke[lane]; x0 = Xe[lane]; }
     if (lane + 32 < QD) { k1 = Ke[lane + 32]; x1 = Xe[lane + 32]; }
   };
-  if (e < a.E) prefetch(e);
+  uint64_t u = (uint64_t)blockIdx.x * kBatchWarps + wib;
+  if (u < nunits) prefetch(u);
 
-  for (; e < a.E; e += nwarps) {
+  const T* c4 = in + 7 * D;
+  const T* Cy = Cs + (Q - 5) * D;
+  // prefix loads of chunk c: one-hot costs of queues 0..Q-6 on their digits' devices
+  auto chunk_base = [&](uint32_t c, T (&b)[D]) {
+#pragma unroll
+    for (int d = 0; d < D; ++d) b[d] = 0;
+#pragma unroll
+    for (int q = Q - 6; q >= 0; --q) {
+      const uint32_t dq = c % D;
+      c /= D;
+#pragma unroll
+      for (int d = 0; d < D; ++d) b[d] = add_f(b[d], (dq == (uint32_t)d) ? Cs[q * D + d] : T(0), one);
+    }
+  };
+  // prefix loads of super-block sb = chunk * D + y
+  auto sb_base = [&](uint32_t sb, T (&b)[D]) {
+    T b2[D];
+    chunk_base(sb / D, b2);
+    const uint32_t y = sb % D;
+    const T cy = Cy[y];
+#pragma unroll
+    for (int d = 0; d < D; ++d) b[d] = add_f(b2[d], (y == (uint32_t)d) ? cy : T(0), one);
+  };
+
+  for (; u < nunits; u += nwarps) {
+    const uint64_t e = epoch_of(u);
+    const bool whole = u < a.e_full;
     // ---- a1: C = K + X, range check, bound UB = sum_q max_d C (decides 32-bit loads) ----
     bool bad = false;
     if (lane < QD) {
@@ -76,7 +111,7 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
       bad |= (k1 >= kEntryLimit) | (x1 >= kEntryLimit);
       C64[lane + 32] = k1 + x1;
     }
-    if (e + nwarps < a.E) prefetch(e + nwarps);  // travels while this epoch is searched
+    if (u + nwarps < nunits) prefetch(u + nwarps);  // travels while this unit is searched
     __syncwarp();
     uint64_t row = 0;
     if (lane < Q) {
@@ -85,77 +120,96 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
     }
 #pragma unroll
     for (int off = 16; off > 0; off >>= 1) row += __shfl_xor_sync(0xffffffffu, row, off);
-    if (__any_sync(0xffffffffu, bad)) {
-      if (lane == 0) raise_flag(a.flags, kFlagRange);
-      continue;
-    }
-    if (row >= (1ull << 32)) {
-      if (lane == 0) raise_flag(a.flags, kFlagNeedU64);
-      continue;
-    }
-    // ---- tables: composed costs (u32) and the inner queues' sums ----
-    if (lane < QD) Cs[lane] = (T)C64[lane];
-    if (lane + 32 < QD) Cs[lane + 32] = (T)C64[lane + 32];
-    if (lane < D) {
-      const T A = (T)C64[(Q - 3) * D + lane], B = (T)C64[(Q - 2) * D + lane], Cc = (T)C64[(Q - 1) * D + lane];
-      in[0 * D + lane] = A;
-      in[1 * D + lane] = B;
-      in[2 * D + lane] = Cc;
-      in[3 * D + lane] = A + B;
-      in[4 * D + lane] = A + Cc;
-      in[5 * D + lane] = B + Cc;
-      in[6 * D + lane] = A + B + Cc;
-      in[7 * D + lane] = (T)C64[(Q - 4) * D + lane];
-    }
-    __syncwarp();
-    const T* c4 = in + 7 * D;
-    const T* Cy = Cs + (Q - 5) * D;
+    // 32-bit loads need UB < 2^32 - 1: every makespan then stays below the all-ones
+    // "no candidate" value the lanes start from (UB = 2^32 - 1 takes the 64-bit rerun)
+    const bool anybad = __any_sync(0xffffffffu, bad);
+    const bool skip = anybad || row >= 0xffffffffull;
+    if (skip && lane == 0) raise_flag(a.flags, anybad ? kFlagRange : kFlagNeedU64);
 
-    // prefix loads of chunk c: one-hot costs of queues 0..Q-6 on their digits' devices
-    auto chunk_base = [&](uint32_t c, T (&b)[D]) {
-#pragma unroll
-      for (int d = 0; d < D; ++d) b[d] = 0;
-#pragma unroll
-      for (int q = Q - 6; q >= 0; --q) {
-        const uint32_t dq = c % D;
-        c /= D;
-#pragma unroll
-        for (int d = 0; d < D; ++d) b[d] = add_f(b[d], (dq == (uint32_t)d) ? Cs[q * D + d] : T(0), one);
+    uint64_t key = ~0ull;  // (makespan << 32) | super-block index
+    if (!skip) {
+      // ---- tables: composed costs (u32) and the inner queues' sums ----
+      if (lane < QD) Cs[lane] = (T)C64[lane];
+      if (lane + 32 < QD) Cs[lane + 32] = (T)C64[lane + 32];
+      if (lane < D) {
+        const T A = (T)C64[(Q - 3) * D + lane], B = (T)C64[(Q - 2) * D + lane], Cc = (T)C64[(Q - 1) * D + lane];
+        in[0 * D + lane] = A;
+        in[1 * D + lane] = B;
+        in[2 * D + lane] = Cc;
+        in[3 * D + lane] = A + B;
+        in[4 * D + lane] = A + Cc;
+        in[5 * D + lane] = B + Cc;
+        in[6 * D + lane] = A + B + Cc;
+        in[7 * D + lane] = (T)C64[(Q - 4) * D + lane];
       }
-    };
+      __syncwarp();
 
-    // ---- a2-a5: lane l walks chunks l, l + 32, ... (increasing) ----
-    T best = ~T(0);
-    uint32_t best_sb = 0xffffffffu;  // super-block index within the epoch: chunk * D + y
-    for (uint32_t c = lane; c < kChunks; c += 32) {
-      T base2[D];
-      chunk_base(c, base2);
-      for (int y = 0; y < D; ++y) {
-        const T cy = Cy[y];
-        T base[D];
+      // ---- a2-a5: each lane walks its units in increasing order, first strict minimum ----
+      T best = ~T(0);
+      uint32_t best_sb = 0xffffffffu;
+      if (whole) {  // lane l: chunks l, l + 32, ... (D super-blocks each)
+        for (uint32_t c = lane; c < kChunks; c += 32) {
+          T base2[D];
+          chunk_base(c, base2);
+          for (int y = 0; y < D; ++y) {
+            const T cy = Cy[y];
+            T base[D];
 #pragma unroll
-        for (int d = 0; d < D; ++d) base[d] = add_f(base2[d], (y == d) ? cy : T(0), one);
-        const T gs = superblock_eval<T, D>(base, in, c4, one);
-        if (gs < best) {
-          best = gs;
-          best_sb = c * D + (uint32_t)y;
+            for (int d = 0; d < D; ++d) base[d] = add_f(base2[d], (y == d) ? cy : T(0), one);
+            const T gs = superblock_eval<T, D>(base, in, c4, one);
+            if (gs < best) {
+              best = gs;
+              best_sb = c * D + (uint32_t)y;
+            }
+          }
+        }
+      } else {  // piece p of the epoch: super-blocks [s0, s1), lane l: s0 + l, s0 + l + 32, ...
+        const uint32_t p = (uint32_t)((u - a.e_full) % a.pieces);
+        const uint32_t nsb = kChunks * D;
+        const uint32_t s0 = (uint32_t)((uint64_t)nsb * p / a.pieces);
+        const uint32_t s1 = (uint32_t)((uint64_t)nsb * (p + 1) / a.pieces);
+        for (uint32_t sb = s0 + lane; sb < s1; sb += 32) {
+          T base[D];
+          sb_base(sb, base);
+          const T gs = superblock_eval<T, D>(base, in, c4, one);
+          if (gs < best) {
+            best = gs;
+            best_sb = sb;
+          }
         }
       }
-    }
-    // ---- warp argmin on (makespan, super-block), then the lowest leaf inside it ----
-    uint64_t key = ((uint64_t)best << 32) | best_sb;
+      key = ((uint64_t)best << 32) | best_sb;
 #pragma unroll
-    for (int off = 16; off > 0; off >>= 1) key = min(key, __shfl_xor_sync(0xffffffffu, key, off));
+      for (int off = 16; off > 0; off >>= 1) key = min(key, __shfl_xor_sync(0xffffffffu, key, off));
+    }
+    if (!whole) {
+      // a split epoch: fold this piece's key into the epoch's; the last piece finishes it
+      const uint64_t t = e - a.e_full;
+      uint32_t last = 0;
+      if (lane == 0) {
+        if (key != ~0ull) atomicMin(reinterpret_cast<unsigned long long*>(&a.keys[t]), key);
+        __threadfence();
+        last = (atomicAdd(&a.done[t], 1u) == a.pieces - 1);
+      }
+      last = __shfl_sync(0xffffffffu, last, 0);
+      if (!last) continue;
+      __threadfence();
+      key = *reinterpret_cast<volatile uint64_t*>(&a.keys[t]);
+      __syncwarp();
+      if (lane == 0) {  // self-reset for the next call
+        a.keys[t] = ~0ull;
+        a.done[t] = 0;
+      }
+      if (skip || key == ~0ull) continue;  // outputs of a failed call are not read
+      // this warp's tables hold epoch e (it searched one of its pieces)
+    } else if (skip) {
+      continue;
+    }
+    // ---- the lowest leaf inside the winning super-block ----
     const T target = (T)(key >> 32);
     const uint32_t sb = (uint32_t)key;
     T base[D];
-    {
-      T base2[D];
-      chunk_base(sb / D, base2);
-      const uint32_t y = sb % D;
-#pragma unroll
-      for (int d = 0; d < D; ++d) base[d] = add_f(base2[d], (y == (uint32_t)d) ? Cy[y] : T(0), one);
-    }
+    sb_base(sb, base);
     uint64_t idx = kNone;
     for (int x = 0; x < D; ++x) {
       T P[D];
@@ -194,10 +248,20 @@ cudaError_t launch_batch_t(const BatchArgs& a, int num_sms, cudaStream_t st, int
     if (per_sm < 1) per_sm = 1;
     occ[dev & 63].store(per_sm, std::memory_order_relaxed);
   }
-  const uint64_t ctas_needed = (a.E + kBatchWarps - 1) / kBatchWarps;
-  uint64_t grid = (uint64_t)num_sms * per_sm;
-  if (grid > ctas_needed) grid = ctas_needed;
-  k<<<(unsigned)grid, 32 * kBatchWarps, 0, st>>>(a);
+  // one resident wave of warps; whole waves of epochs take one warp each, the epochs of
+  // the last partial wave are split into pieces of >= 32 super-blocks over the idle warps
+  const uint64_t slots = (uint64_t)num_sms * per_sm * kBatchWarps;
+  BatchArgs b = a;
+  b.e_full = a.E / slots * slots;
+  const uint64_t rem = a.E - b.e_full;
+  static const int kPiecesCap = env_int("MCL_BATCH_PIECES", 64, 1, 1 << 20);  // tuning knob
+  const uint64_t max_pieces =
+      std::max<uint64_t>(1, std::min<uint64_t>(IPow<D, Q - 5>::v * D / 32, (uint64_t)kPiecesCap));
+  b.pieces = rem ? (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(slots / rem, max_pieces)) : 1;
+  if (b.pieces == 1) b.e_full = a.E;  // nothing to split
+  const uint64_t units = b.e_full + (a.E - b.e_full) * b.pieces;
+  uint64_t grid = std::min<uint64_t>((uint64_t)num_sms * per_sm, (units + kBatchWarps - 1) / kBatchWarps);
+  k<<<(unsigned)grid, 32 * kBatchWarps, 0, st>>>(b);
   *grid_out = (int)grid;
   return cudaGetLastError();
 }

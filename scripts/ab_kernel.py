@@ -3,6 +3,7 @@
     python scripts/ab_kernel.py --libs ab/libmcl_head.so paper_conf_cluster_ajipbf15_b200/libmcl.so \
         --workloads cfg5 cfg4 cfg2 --rounds 3
 
+A library may carry environment settings for its subprocess: `lib.so@MCL_BATCH_PIECES=1`.
 Each (round, library) pair runs in its own subprocess (the binding loads one library per
 process); libraries alternate within a round so clock drift hits them alike. Prints the
 median kernel time (CUDA events around the search launch) per library and workload, and
@@ -52,8 +53,13 @@ def main():
     results = {}
     for r in range(args.rounds):
         for lib in (args.libs if r % 2 == 0 else args.libs[::-1]):
-            code = CHILD.format(root=ROOT, lib=os.path.abspath(lib), wls=args.workloads)
-            p = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True)
+            path, _, envs = lib.partition("@")
+            env = dict(os.environ)
+            for kv in filter(None, envs.split(",")):
+                k, _, v = kv.partition("=")
+                env[k] = v
+            code = CHILD.format(root=ROOT, lib=os.path.abspath(path), wls=args.workloads)
+            p = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, env=env)
             if p.returncode:
                 print(lib, "failed:", p.stderr[-2000:])
                 continue

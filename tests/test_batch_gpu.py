@@ -104,11 +104,29 @@ def test_batch_u64_rerun(torch_cuda, mapper):
 
 
 def test_batch_range_error(torch_cuda, mapper):
+    """An entry >= 2^48 in a split epoch fails the call; the split epochs' scratch (keys,
+    piece counters) is left reset, so the next call on the same shapes is exact."""
     K, X = workloads.random_tables(72, 6, 8, 4)
     X[3, 2, 1] = 1 << 48
     with pytest.raises(MclError) as ei:
         run(torch_cuda, mapper, K, X, 7)
     assert ei.value.status == MCL_E_RANGE
+    X[3, 2, 1] = 5
+    got, _ = run(torch_cuda, mapper, K, X, 7)
+    check(got, oracle.oracle_map(K, X), "after range error")
+
+
+@pytest.mark.parametrize("Q,D", [(9, 3), (8, 4), (8, 5)])
+def test_batch_whole_and_split_epochs(torch_cuda, mapper, Q, D):
+    """More epochs than resident warps: whole epochs (one warp each) plus a last partial
+    wave split into super-block pieces, merged by the last piece to finish."""
+    E = 148 * 16 + 123
+    K, X = workloads.small_int_tables(77 * Q + D, E, Q, D, hi=64)
+    want = oracle.oracle_map(K, X)
+    for rep in range(2):  # the second call reuses the self-reset per-epoch scratch
+        got, info = run(torch_cuda, mapper, K, X, 7)
+        assert info["path"] == "batch_u32"
+        check(got, want, f"{Q}x{D} E={E} rep {rep}")
 
 
 def test_batch_single_epoch_and_no_mapping_output(torch_cuda, mapper):
