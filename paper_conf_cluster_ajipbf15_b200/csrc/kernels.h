@@ -222,10 +222,7 @@ struct BatchArgs {
   uint8_t* mapping;
   volatile uint32_t* flags;
   uint32_t one;
-  uint64_t* keys;     // [E] packed (makespan, super-block) of split epochs, all-ones on entry
-  uint32_t* done;     // [E] pieces finished, zero on entry; both self-resetting
-  uint64_t e_full;    // set by launch_batch: epochs searched whole
-  uint32_t pieces;    // set by launch_batch: pieces of each remaining epoch
+  uint64_t e_full;    // set by launch_batch: epochs searched by one warp (whole waves)
 };
 bool batch_supported(uint32_t Q, uint32_t D);
 cudaError_t launch_batch(const BatchArgs& a, int num_sms, cudaStream_t st, int* grid_out);

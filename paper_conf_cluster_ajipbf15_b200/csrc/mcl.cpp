@@ -134,7 +134,6 @@ struct mcl_mapper {
   DevBuf done;             // uint32 per epoch, zero between calls
   DevBuf key, pair, gms, cand;
   DevBuf flat_keys, flat_done;  // flattened batched kernel: per-epoch key / block count
-  DevBuf batch_keys, batch_done;  // warp-per-epoch kernel: split epochs' key / piece count
   DevBuf bnb_next, bnb_inc, bnb_nodes;  // pruned search: subtree counters, incumbents, nodes
   DevBuf model_buf[9], cost_k, cost_x;  // cost-table construction: staged model, built K / X
   DevBuf in_k, in_x, in_base, in_elig, out_idx, out_ms, out_map;  // staging for host pointers
@@ -335,7 +334,7 @@ void mcl_mapper_destroy(mcl_mapper_t* h) {
     for (void* p : h->peer_opened) cudaIpcCloseMemHandle(p);
     for (DevBuf* b : {&h->peer_slab, &h->peer_kdone, &h->peer_gms, &h->peer_ptrs}) b->release();
     for (DevBuf* b : {&h->scratch, &h->done, &h->key, &h->pair, &h->gms, &h->cand, &h->flat_keys,
-                      &h->flat_done, &h->batch_keys, &h->batch_done, &h->bnb_next, &h->bnb_inc, &h->bnb_nodes, &h->in_k,
+                      &h->flat_done, &h->bnb_next, &h->bnb_inc, &h->bnb_nodes, &h->in_k,
                       &h->in_base, &h->in_elig,
                       &h->in_x, &h->out_idx, &h->out_ms, &h->out_map, &h->cost_k, &h->cost_x})
       b->release();
@@ -591,10 +590,10 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
   const bool shard_mode = h->world > 1;  // NCCL collective or single-GPU shard test
   // the small and flattened kernels take no constraints; the blocked and generic ones do
   int path;
-  // warp-per-epoch kernel: batches of at least one full wave of warps (16 per SM)
+  // warp-per-epoch kernel: batches of at least one epoch per resident CTA (4 per SM)
   const bool batch_ok = !shard_mode && !multi && !constrained && mcl::batch_supported(Q, D);
   if (!shard_mode && !multi && !constrained && mcl::small_supported(Q, D)) path = 4;
-  else if (batch_ok && epochs >= (uint64_t)h->num_sms * 16) path = 7;
+  else if (batch_ok && epochs >= (uint64_t)h->num_sms * 4) path = 7;
   else if (mcl::blocked_supported(Q, D)) path = 1;
   else path = 3;
   if (h->force_path && h->force_path != 6) {  // 6 only affects mcl_map_queues_pruned
@@ -620,13 +619,6 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
     if (h->timing) MCL_CUDA(h, record_start(h, s), "cudaEventRecord(start)");
     if (path == 7) {
       mcl::BatchArgs a{Q, D, epochs, K, X, o_idx, o_ms, o_map, h->flags_dev, 1u};
-      if (h->batch_keys.cap < epochs * 8) {
-        MCL_CUDA(h, h->batch_keys.ensure(epochs * 8), "cudaMalloc(batch keys)");
-        MCL_CUDA(h, h->batch_keys.fill(0xff), "cudaMemset(batch keys)");
-      }
-      MCL_CUDA(h, h->batch_done.ensure(epochs * 4, true), "cudaMalloc(batch done)");
-      a.keys = (uint64_t*)h->batch_keys.p;
-      a.done = (uint32_t*)h->batch_done.p;
       int gx = 0;
       MCL_CUDA(h, mcl::launch_batch(a, h->num_sms, s, &gx), "search_batch launch");
       grid.x = gx;

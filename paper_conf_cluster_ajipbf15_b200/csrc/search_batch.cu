@@ -8,13 +8,17 @@
 // setup is a fifth of the instructions in the CTA-per-epoch kernel:
 //   * persistent warps stride over the epochs; the next epoch's K and X are loaded into
 //     registers while the current one is searched (no load latency in the prologue);
-//   * no __syncthreads, no shared atomics: everything is warp-synchronous;
-//   * the chunk digits (queues 0..Q-6) come from compile-time divisions of the chunk
-//     index, the one-hot prefix vectors from selects on the cost table -- no outer tables;
+//   * warp-synchronous setup, no outer tables: the chunk digits (queues 0..Q-6) come from
+//     compile-time divisions of the chunk index, the one-hot prefix vectors from selects
+//     on the cost table;
 //   * lane l walks chunks l, l + 32, ... (D^2 blocks each, the super-block path), keeping
 //     the first strict minimum of its own increasing sequence; the warp takes the
 //     lexicographic minimum of (makespan, super-block index), and re-scans only that
 //     super-block (block by block, 32 leaves per ballot) for the lowest leaf index.
+// Wave quantisation: whole waves of epochs (one per warp) run first; the epochs of the last,
+// partial wave go one per CTA, its warps splitting the epoch's super-blocks and merging
+// their keys through shared memory (no global atomics or fences). A batch below one wave
+// runs one warp per epoch.
 // Mapping index m = ((chunk * D + y) * D + x) * D^3 + leaf, queue 0 most significant
 // (R6): chunk = digits of queues 0..Q-6, y = queue Q-5, x = queue Q-4, leaf =
 // queues Q-3..Q-1.
@@ -44,35 +48,38 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
   using T = uint32_t;
   constexpr int QD = Q * D;
   constexpr uint32_t kChunks = (uint32_t)IPow<D, Q - 5>::v;  // chunks of D^2 blocks per epoch
+  constexpr uint32_t kSb = kChunks * D;                      // super-blocks per epoch
   static_assert(QD <= 64, "two cost entries per lane");
   static_assert(Q >= 6, "chunks need queues 0..Q-6");
   __shared__ __align__(16) uint64_t sC64[kBatchWarps][QD];
   __shared__ __align__(16) T sC[kBatchWarps][QD];
   __shared__ __align__(16) T sIn[kBatchWarps][8 * D];
+  __shared__ uint64_t s_key[2][kBatchWarps];  // split epochs: each warp's key (double-buffered)
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   uint64_t* C64 = sC64[wib];
   T* Cs = sC[wib];
   T* in = sIn[wib];
   const uint32_t one = a.one;
   const uint64_t nwarps = (uint64_t)gridDim.x * kBatchWarps;
-  // Work units: epochs 0..e_full-1 whole (one warp each); each remaining epoch in `pieces`
-  // contiguous super-block ranges (the last, partial wave spread over all warps).
-  const uint64_t nunits = a.e_full + (a.E - a.e_full) * a.pieces;
-  auto epoch_of = [&](uint64_t u) -> uint64_t {
-    return u < a.e_full ? u : a.e_full + (u - a.e_full) / a.pieces;
+  const uint64_t gw = (uint64_t)blockIdx.x * kBatchWarps + wib;
+  // This warp's units: whole epochs gw, gw + nwarps, ... below e_full, then the CTA's
+  // split epochs e_full + blockIdx.x, + gridDim.x, ... There are split epochs only when
+  // e_full is a multiple of nwarps, so the CTA's warps then share one unit sequence (the
+  // barrier of a split epoch is reached by all of them).
+  const uint64_t n_whole = a.e_full > gw ? (a.e_full - gw + nwarps - 1) / nwarps : 0;
+  auto unit_epoch = [&](uint64_t i) -> uint64_t {
+    return i < n_whole ? gw + i * nwarps : a.e_full + blockIdx.x + (i - n_whole) * gridDim.x;
   };
 
-  // prefetch of a unit's epoch costs: entries lane and lane + 32
+  // prefetch of an epoch's costs: entries lane and lane + 32
   uint64_t k0 = 0, x0 = 0, k1 = 0, x1 = 0;
-  auto prefetch = [&](uint64_t u) {
-    const uint64_t ep = epoch_of(u);
+  auto prefetch = [&](uint64_t ep) {
     const uint64_t* Ke = a.K + ep * QD;
     const uint64_t* Xe = a.X + ep * QD;
     if (lane < QD) { k0 = Ke[lane]; x0 = Xe[lane]; }
     if (lane + 32 < QD) { k1 = Ke[lane + 32]; x1 = Xe[lane + 32]; }
   };
-  uint64_t u = (uint64_t)blockIdx.x * kBatchWarps + wib;
-  if (u < nunits) prefetch(u);
+  if (unit_epoch(0) < a.E) prefetch(unit_epoch(0));
 
   const T* c4 = in + 7 * D;
   const T* Cy = Cs + (Q - 5) * D;
@@ -97,10 +104,46 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
 #pragma unroll
     for (int d = 0; d < D; ++d) b[d] = add_f(b2[d], (y == (uint32_t)d) ? cy : T(0), one);
   };
+  // a warp's lexicographic minimum of (makespan << 32 | super-block)
+  auto warp_key = [&](T best, uint32_t best_sb) {
+    uint64_t key = ((uint64_t)best << 32) | best_sb;
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) key = min(key, __shfl_xor_sync(0xffffffffu, key, off));
+    return key;
+  };
+  // the lowest leaf inside the winning super-block, then the outputs (a5, a7)
+  auto finish = [&](uint64_t e, uint64_t key) {
+    const T target = (T)(key >> 32);
+    const uint32_t sb = (uint32_t)key;
+    T base[D];
+    sb_base(sb, base);
+    uint64_t idx = kNone;
+    for (int x = 0; x < D; ++x) {
+      T P[D];
+#pragma unroll
+      for (int d = 0; d < D; ++d) P[d] = (x == d) ? base[d] + c4[d] : base[d];
+      const uint32_t leaf = block_first_warp<T, D>(P, in, target);
+      if (leaf != 0xffffffffu) {
+        idx = ((uint64_t)sb * D + (uint64_t)x) * (uint64_t)(D * D * D) + leaf;
+        break;
+      }
+    }
+    if (lane == 0) {
+      a.index[e] = idx;
+      a.makespan[e] = (uint64_t)target;
+    }
+    if (a.mapping && lane < Q) {  // digits of the index, queue 0 most significant
+      uint64_t rest = idx;
+      for (int q = Q - 1; q > lane; --q) rest /= D;
+      a.mapping[e * Q + lane] = (uint8_t)(rest % D);
+    }
+  };
 
-  for (; u < nunits; u += nwarps) {
-    const uint64_t e = epoch_of(u);
-    const bool whole = u < a.e_full;
+  int par = 0;
+  for (uint64_t i = 0;; ++i) {
+    const uint64_t e = unit_epoch(i);
+    if (e >= a.E) break;
+    const bool whole = i < n_whole;
     // ---- a1: C = K + X, range check, bound UB = sum_q max_d C (decides 32-bit loads) ----
     bool bad = false;
     if (lane < QD) {
@@ -111,7 +154,8 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
       bad |= (k1 >= kEntryLimit) | (x1 >= kEntryLimit);
       C64[lane + 32] = k1 + x1;
     }
-    if (u + nwarps < nunits) prefetch(u + nwarps);  // travels while this unit is searched
+    const uint64_t en = unit_epoch(i + 1);
+    if (en < a.E) prefetch(en);  // travels while this epoch is searched
     __syncwarp();
     uint64_t row = 0;
     if (lane < Q) {
@@ -124,9 +168,9 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
     // "no candidate" value the lanes start from (UB = 2^32 - 1 takes the 64-bit rerun)
     const bool anybad = __any_sync(0xffffffffu, bad);
     const bool skip = anybad || row >= 0xffffffffull;
-    if (skip && lane == 0) raise_flag(a.flags, anybad ? kFlagRange : kFlagNeedU64);
+    if (skip && lane == 0 && (whole || wib == 0)) raise_flag(a.flags, anybad ? kFlagRange : kFlagNeedU64);
 
-    uint64_t key = ~0ull;  // (makespan << 32) | super-block index
+    uint64_t key = ~0ull;
     if (!skip) {
       // ---- tables: composed costs (u32) and the inner queues' sums ----
       if (lane < QD) Cs[lane] = (T)C64[lane];
@@ -143,8 +187,7 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
         in[7 * D + lane] = (T)C64[(Q - 4) * D + lane];
       }
       __syncwarp();
-
-      // ---- a2-a5: each lane walks its units in increasing order, first strict minimum ----
+      // ---- a2-a5: each lane walks its share in increasing order, first strict minimum ----
       T best = ~T(0);
       uint32_t best_sb = 0xffffffffu;
       if (whole) {  // lane l: chunks l, l + 32, ... (D super-blocks each)
@@ -163,11 +206,8 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
             }
           }
         }
-      } else {  // piece p of the epoch: super-blocks [s0, s1), lane l: s0 + l, s0 + l + 32, ...
-        const uint32_t p = (uint32_t)((u - a.e_full) % a.pieces);
-        const uint32_t nsb = kChunks * D;
-        const uint32_t s0 = (uint32_t)((uint64_t)nsb * p / a.pieces);
-        const uint32_t s1 = (uint32_t)((uint64_t)nsb * (p + 1) / a.pieces);
+      } else {  // warp wib of the CTA: super-blocks [s0, s1), lane l: s0 + l, s0 + l + 32, ...
+        const uint32_t s0 = kSb * (uint32_t)wib / kBatchWarps, s1 = kSb * (uint32_t)(wib + 1) / kBatchWarps;
         for (uint32_t sb = s0 + lane; sb < s1; sb += 32) {
           T base[D];
           sb_base(sb, base);
@@ -178,59 +218,22 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
           }
         }
       }
-      key = ((uint64_t)best << 32) | best_sb;
-#pragma unroll
-      for (int off = 16; off > 0; off >>= 1) key = min(key, __shfl_xor_sync(0xffffffffu, key, off));
+      key = warp_key(best, best_sb);
     }
-    if (!whole) {
-      // a split epoch: fold this piece's key into the epoch's; the last piece finishes it
-      const uint64_t t = e - a.e_full;
-      uint32_t last = 0;
-      if (lane == 0) {
-        if (key != ~0ull) atomicMin(reinterpret_cast<unsigned long long*>(&a.keys[t]), key);
-        __threadfence();
-        last = (atomicAdd(&a.done[t], 1u) == a.pieces - 1);
-      }
-      last = __shfl_sync(0xffffffffu, last, 0);
-      if (!last) continue;
-      __threadfence();
-      key = *reinterpret_cast<volatile uint64_t*>(&a.keys[t]);
-      __syncwarp();
-      if (lane == 0) {  // self-reset for the next call
-        a.keys[t] = ~0ull;
-        a.done[t] = 0;
-      }
-      if (skip || key == ~0ull) continue;  // outputs of a failed call are not read
-      // this warp's tables hold epoch e (it searched one of its pieces)
-    } else if (skip) {
+    if (whole) {
+      if (!skip) finish(e, key);
       continue;
     }
-    // ---- the lowest leaf inside the winning super-block ----
-    const T target = (T)(key >> 32);
-    const uint32_t sb = (uint32_t)key;
-    T base[D];
-    sb_base(sb, base);
-    uint64_t idx = kNone;
-    for (int x = 0; x < D; ++x) {
-      T P[D];
+    // a split epoch: the CTA's warps merge their keys in shared memory; warp 0 finishes
+    if (lane == 0) s_key[par][wib] = key;
+    __syncthreads();
+    if (wib == 0 && !skip) {
+      uint64_t k = s_key[par][0];
 #pragma unroll
-      for (int d = 0; d < D; ++d) P[d] = (x == d) ? base[d] + c4[d] : base[d];
-      const uint32_t leaf = block_first_warp<T, D>(P, in, target);
-      if (leaf != 0xffffffffu) {
-        idx = ((uint64_t)sb * D + (uint64_t)x) * (uint64_t)(D * D * D) + leaf;
-        break;
-      }
+      for (int w = 1; w < kBatchWarps; ++w) k = min(k, s_key[par][w]);
+      finish(e, k);
     }
-    // ---- a7: outputs (digits of the index, queue 0 most significant) ----
-    if (lane == 0) {
-      a.index[e] = idx;
-      a.makespan[e] = (uint64_t)target;
-    }
-    if (a.mapping && lane < Q) {
-      uint64_t rest = idx;
-      for (int q = Q - 1; q > lane; --q) rest /= D;
-      a.mapping[e * Q + lane] = (uint8_t)(rest % D);
-    }
+    par ^= 1;  // the next split epoch writes the other buffer (one barrier in between)
   }
 }
 
@@ -249,18 +252,17 @@ cudaError_t launch_batch_t(const BatchArgs& a, int num_sms, cudaStream_t st, int
     occ[dev & 63].store(per_sm, std::memory_order_relaxed);
   }
   // one resident wave of warps; whole waves of epochs take one warp each, the epochs of
-  // the last partial wave are split into pieces of >= 32 super-blocks over the idle warps
-  const uint64_t slots = (uint64_t)num_sms * per_sm * kBatchWarps;
+  // the last partial wave one CTA each (its warps split the super-blocks)
+  // (measured, scripts/batch_waves.py: splitting pays after at least one whole wave; a
+  // batch below one wave runs one warp per epoch)
+  const uint64_t ctas = (uint64_t)num_sms * per_sm;
   BatchArgs b = a;
-  b.e_full = a.E / slots * slots;
-  const uint64_t rem = a.E - b.e_full;
-  static const int kPiecesCap = env_int("MCL_BATCH_PIECES", 64, 1, 1 << 20);  // tuning knob
-  const uint64_t max_pieces =
-      std::max<uint64_t>(1, std::min<uint64_t>(IPow<D, Q - 5>::v * D / 32, (uint64_t)kPiecesCap));
-  b.pieces = rem ? (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(slots / rem, max_pieces)) : 1;
-  if (b.pieces == 1) b.e_full = a.E;  // nothing to split
-  const uint64_t units = b.e_full + (a.E - b.e_full) * b.pieces;
-  uint64_t grid = std::min<uint64_t>((uint64_t)num_sms * per_sm, (units + kBatchWarps - 1) / kBatchWarps);
+  b.e_full = a.E / (ctas * kBatchWarps) * (ctas * kBatchWarps);
+  uint64_t grid = ctas;
+  if (b.e_full == 0) {
+    b.e_full = a.E;
+    grid = std::min<uint64_t>(ctas, (a.E + kBatchWarps - 1) / kBatchWarps);
+  }
   k<<<(unsigned)grid, 32 * kBatchWarps, 0, st>>>(b);
   *grid_out = (int)grid;
   return cudaGetLastError();

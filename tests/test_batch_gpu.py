@@ -77,7 +77,7 @@ def test_batch_degenerate_ties(torch_cuda, mapper):
 
 
 def test_batch_auto_selection_cfg2(torch_cuda, mapper):
-    """cfg2 (10^4 epochs >= one wave of warps) runs the batched kernel automatically and
+    """cfg2 (10^4 epochs >= one per resident CTA) runs the batched kernel automatically and
     agrees with the CTA-per-epoch kernel and the oracle on every epoch."""
     K, X = workloads.cfg2()
     want = oracle.oracle_map(K, X)
@@ -87,7 +87,7 @@ def test_batch_auto_selection_cfg2(torch_cuda, mapper):
     got, info = run(torch_cuda, mapper, K, X, 1)
     assert info["path"] == "blocked_u32"
     check(got, want, "cfg2 CTA per epoch")
-    # a batch below one wave keeps the CTA-per-epoch kernel (it splits epochs over CTAs)
+    # a batch below one epoch per resident CTA keeps the CTA-per-epoch kernel
     got, info = run(torch_cuda, mapper, K[:100], X[:100], 0)
     assert info["path"] == "blocked_u32", info
     check(got, tuple(w[:100] for w in want), "cfg2[:100]")
@@ -104,8 +104,8 @@ def test_batch_u64_rerun(torch_cuda, mapper):
 
 
 def test_batch_range_error(torch_cuda, mapper):
-    """An entry >= 2^48 in a split epoch fails the call; the split epochs' scratch (keys,
-    piece counters) is left reset, so the next call on the same shapes is exact."""
+    """An entry >= 2^48 in a split epoch fails the call; the next call on the same shapes
+    is exact."""
     K, X = workloads.random_tables(72, 6, 8, 4)
     X[3, 2, 1] = 1 << 48
     with pytest.raises(MclError) as ei:
@@ -119,11 +119,11 @@ def test_batch_range_error(torch_cuda, mapper):
 @pytest.mark.parametrize("Q,D", [(9, 3), (8, 4), (8, 5)])
 def test_batch_whole_and_split_epochs(torch_cuda, mapper, Q, D):
     """More epochs than resident warps: whole epochs (one warp each) plus a last partial
-    wave split into super-block pieces, merged by the last piece to finish."""
+    wave of epochs split over the warps of a CTA, merged in shared memory."""
     E = 148 * 16 + 123
     K, X = workloads.small_int_tables(77 * Q + D, E, Q, D, hi=64)
     want = oracle.oracle_map(K, X)
-    for rep in range(2):  # the second call reuses the self-reset per-epoch scratch
+    for rep in range(2):
         got, info = run(torch_cuda, mapper, K, X, 7)
         assert info["path"] == "batch_u32"
         check(got, want, f"{Q}x{D} E={E} rep {rep}")
