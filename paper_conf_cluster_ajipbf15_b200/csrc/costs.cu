@@ -14,12 +14,10 @@
 //  interpolation techniques", L905-907). fp64 with explicitly rounded operations (no FMA
 //  contraction), so the result is bit-identical to a plain IEEE evaluation.
 //
-// Tiles of 256 (epoch, queue) pairs per CTA: the tile's CSR offsets and its contiguous
-// slice of kernel ids are staged in shared memory with coalesced loads (the profile table
-// too, when it fits), then one thread per pair sums its invocations' profile rows and
-// interpolates the curves (sizes and bandwidths in shared memory; one segment search serves
-// every device because the sample sizes are shared). Memory-bound: reads ids / offsets /
-// bytes / source / cached once, writes 2 x D x 8 bytes per pair.
+// Tiles of 256 (epoch, queue) pairs per CTA, one thread per pair: it sums its invocations'
+// profile rows and interpolates the curves (sizes and bandwidths in shared memory; one
+// segment search serves every device because the sample sizes are shared). Memory-bound:
+// reads ids / offsets / bytes / source / cached once, writes 2 x D x 8 bytes per pair.
 #include "common.cuh"
 #include "kernels.h"
 
@@ -41,24 +39,30 @@ __device__ __forceinline__ uint64_t transfer_ns(uint64_t bytes, double bw) {
 
 }  // namespace
 
-constexpr int kCostTile = 256;      // (epoch, queue) pairs per CTA tile (= blockDim.x)
-constexpr int kIdsCap = 8192;       // kernel ids of a tile staged in shared memory
+constexpr int kCostTile = 256;        // (epoch, queue) pairs per CTA tile (= blockDim.x)
 constexpr int kProfCapBytes = 32768;  // profile table staged when it fits
 
+// Memory pipeline: a persistent CTA walks its tiles with each thread's next pair (CSR
+// offsets, bytes, source, cached mask) loaded into registers while the current pair is
+// computed, so the loads of tile t + 1 are in flight during tile t -- no block barriers in
+// the tile loop. Invocation ids are read straight from global memory through L1 (the lists
+// of a warp's pairs are adjacent, so a warp's reads of one list position share lines);
+// profile rows and bandwidth curves come from shared memory. Outputs go through a per-warp
+// shared buffer so every store instruction writes 32 consecutive words.
 template <int D>
 __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const uint32_t M = a.M;
-  const int tid = threadIdx.x;
-  // layout: sizes[M] u64 | h2d[D][M] f64 | d2h[D][M] f64 | off[kCostTile+1] u64 |
-  //         prof[num_kernels][D] u64 (if it fits) | ids[kIdsCap] u32
-  uint64_t* s_sizes = reinterpret_cast<uint64_t*>(smem_raw);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  // layout: outK[kCostTile*D] u64 | outX[kCostTile*D] u64 | sizes[M] u64 | h2d[D][M] f64 |
+  //         d2h[D][M] f64 | prof[num_kernels][D] u64 (if it fits)
+  uint64_t* s_outK = reinterpret_cast<uint64_t*>(smem_raw);
+  uint64_t* s_outX = s_outK + (size_t)kCostTile * D;
+  uint64_t* s_sizes = s_outX + (size_t)kCostTile * D;
   double* s_h2d = reinterpret_cast<double*>(s_sizes + M);
   double* s_d2h = s_h2d + (size_t)D * M;
-  uint64_t* s_off = reinterpret_cast<uint64_t*>(s_d2h + (size_t)D * M);
-  uint64_t* s_prof = s_off + (kCostTile + 1);
+  uint64_t* s_prof = reinterpret_cast<uint64_t*>(s_d2h + (size_t)D * M);
   const bool prof_in_smem = (size_t)a.num_kernels * D * 8 <= (size_t)kProfCapBytes;
-  uint32_t* s_ids = reinterpret_cast<uint32_t*>(s_prof + (prof_in_smem ? (size_t)a.num_kernels * D : 0));
   for (uint32_t t = tid; t < M; t += blockDim.x) s_sizes[t] = a.sizes[t];
   for (uint32_t t = tid; t < D * M; t += blockDim.x) {
     s_h2d[t] = a.h2d[t];
@@ -76,41 +80,49 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
       if (!(s_h2d[i] > 0.0) || !(s_d2h[i] > 0.0)) status |= kFlagBadModel;
     if (a.offsets[a.EQ] != a.nnz) status |= kFlagBadModel;
   }
+
+  // this thread's pair of a tile, loaded one tile ahead
+  uint64_t n_j0 = 0, n_j1 = 0, n_bytes = 0;
+  int32_t n_src = 0;
+  uint32_t n_cached = 0;
+  auto fetch = [&](uint64_t tile) {
+    const uint64_t eq = tile * kCostTile + tid;
+    if (eq < a.EQ) {
+      n_j0 = a.offsets[eq];
+      n_j1 = a.offsets[eq + 1];
+      n_bytes = a.bytes[eq];
+      n_src = a.source[eq];
+      n_cached = a.cached ? (uint32_t)a.cached[eq] : 0u;
+    }
+  };
   const uint64_t ntiles = (a.EQ + kCostTile - 1) / kCostTile;
+  if (blockIdx.x < ntiles) fetch(blockIdx.x);
   for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-    const uint64_t t0 = tile * kCostTile;
-    const uint32_t n = (uint32_t)((a.EQ - t0 < (uint64_t)kCostTile) ? a.EQ - t0 : kCostTile);
-    __syncthreads();  // the previous tile's staging is no longer read
-    for (uint32_t i = tid; i <= n; i += blockDim.x) s_off[i] = a.offsets[t0 + i];
-    __syncthreads();
-    // the tile's invocation lists are one contiguous slice of kernel_ids: stage it coalesced
-    const uint64_t lo = s_off[0], hi = s_off[n];
-    const bool ids_in_smem = hi >= lo && hi <= a.nnz && hi - lo <= (uint64_t)kIdsCap;
-    if (ids_in_smem)
-      for (uint64_t j = lo + tid; j < hi; j += blockDim.x) s_ids[j - lo] = a.ids[j];
-    __syncthreads();
-    if ((uint32_t)tid < n) {
-      const uint64_t eq = t0 + tid;
+    const uint64_t j0 = n_j0, j1 = n_j1, bytes = n_bytes;
+    const int32_t src = n_src;
+    const uint32_t cached = n_cached;
+    if (tile + gridDim.x < ntiles) fetch(tile + gridDim.x);
+    const uint64_t eq = tile * kCostTile + tid;
+    if (eq < a.EQ) {
       // ---- kernel part: sum of the invoked kernels' profile rows ----
       uint64_t k[D];
 #pragma unroll
       for (int d = 0; d < D; ++d) k[d] = 0;
-      const uint64_t j0 = s_off[tid], j1 = s_off[tid + 1];
       bool ok = j0 <= j1 && j1 <= a.nnz;
-      for (uint64_t j = j0; ok && j < j1; ++j) {
-        const uint32_t kid = ids_in_smem ? s_ids[j - lo] : a.ids[j];
-        if (kid >= a.num_kernels) {
-          ok = false;
-          break;
-        }
-        const uint64_t* row = prof + (uint64_t)kid * D;
+      if (ok) {
+#pragma unroll 4
+        for (uint64_t j = j0; j < j1; ++j) {
+          const uint32_t kid = __ldg(a.ids + j);
+          if (kid >= a.num_kernels) {
+            ok = false;
+            break;
+          }
+          const uint64_t* row = prof + (uint64_t)kid * D;
 #pragma unroll
-        for (int d = 0; d < D; ++d) k[d] += row[d];
+          for (int d = 0; d < D; ++d) k[d] += row[d];
+        }
       }
       // ---- transfer part ----
-      const uint64_t bytes = a.bytes[eq];
-      const int32_t src = a.source[eq];
-      const uint32_t cached = a.cached ? (uint32_t)a.cached[eq] : 0u;
       ok = ok && src >= -1 && src < (int32_t)D;
       if (!ok) status |= kFlagBadModel;
       const bool clo = bytes <= s_sizes[0], chi = bytes >= s_sizes[M - 1];
@@ -140,10 +152,23 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
           x = down + up;
         }
         if (k[d] >= kEntryLimit || x >= kEntryLimit) status |= kFlagRange;
-        a.K[eq * D + d] = k[d];
-        a.X[eq * D + d] = x;
+        s_outK[(size_t)tid * D + d] = k[d];
+        s_outX[(size_t)tid * D + d] = x;
       }
     }
+    // ---- coalesced stores: the warp's 32 pairs are 32 * D consecutive words ----
+    __syncwarp();
+    const uint64_t base = tile * kCostTile + (uint64_t)warp * 32;
+    if (base < a.EQ) {
+      const uint32_t np = (uint32_t)((a.EQ - base < 32) ? a.EQ - base : 32);
+      const uint64_t* sk = s_outK + (size_t)warp * 32 * D;
+      const uint64_t* sx = s_outX + (size_t)warp * 32 * D;
+      for (uint32_t w = lane; w < np * D; w += 32) {
+        a.K[base * D + w] = sk[w];
+        a.X[base * D + w] = sx[w];
+      }
+    }
+    __syncwarp();  // the buffer is rewritten by the next tile
   }
   if (__any_sync(0xffffffffu, status != 0)) {
     const uint32_t all = __reduce_or_sync(0xffffffffu, status);
@@ -154,15 +179,24 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
 namespace {
 template <int D>
 cudaError_t launch_build_costs_t(const CostArgs& a, int num_sms, cudaStream_t st) {
-  size_t smem = (size_t)a.M * 8 + 2 * (size_t)D * a.M * 8 + (kCostTile + 1) * 8;
+  size_t smem = 2 * (size_t)kCostTile * D * 8 + (size_t)a.M * 8 + 2 * (size_t)D * a.M * 8;
   if ((size_t)a.num_kernels * D * 8 <= (size_t)kProfCapBytes) smem += (size_t)a.num_kernels * D * 8;
-  smem += (size_t)kIdsCap * 4;
   auto k = build_costs_kernel<D>;
   static SmemAttrCache cache;
   cudaError_t err = ensure_smem(k, smem, cache);
   if (err != cudaSuccess) return err;
+  static std::atomic<int> occ[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int per_sm = occ[dev & 63].load(std::memory_order_relaxed);
+  if (per_sm == 0) {  // resident CTAs per SM at this shared-memory size (persistent grid)
+    err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kCostTile, smem);
+    if (err != cudaSuccess) return err;
+    per_sm = per_sm < 1 ? 1 : per_sm;
+    occ[dev & 63].store(per_sm, std::memory_order_relaxed);
+  }
   uint64_t grid = (a.EQ + kCostTile - 1) / kCostTile;
-  const uint64_t cap = (uint64_t)num_sms * 4;
+  const uint64_t cap = (uint64_t)num_sms * per_sm;
   if (grid > cap) grid = cap;
   if (grid == 0) grid = 1;
   k<<<(unsigned)grid, kCostTile, smem, st>>>(a);
