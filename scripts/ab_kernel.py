@@ -3,6 +3,7 @@
     python scripts/ab_kernel.py --libs ab/libmcl_head.so paper_conf_cluster_ajipbf15_b200/libmcl.so \
         --workloads cfg5 cfg4 cfg2 --rounds 3
 
+A workload may carry generator / path options: `cfg2:E=600:path=7`.
 A library may carry environment settings for its subprocess: `lib.so@MCL_BATCH_PIECES=1`.
 Each (round, library) pair runs in its own subprocess (the binding loads one library per
 process); libraries alternate within a round so clock drift hits them alike. Prints the
@@ -27,8 +28,11 @@ mcl.load_library({lib!r})
 out = {{}}
 with Mapper(0) as m:
     m.set_timing(1)
-    for name in {wls!r}:
-        K, X = workloads.make(name)
+    for spec in {wls!r}:
+        name, *opts = spec.split(":")
+        kw = {{k: int(v) for k, v in (o.split("=") for o in opts)}}
+        m.force_path(kw.pop("path", 0))
+        K, X = workloads.make(name, **kw)
         Kd, Xd = torch.from_numpy(K).cuda(), torch.from_numpy(X).cuda()
         reps = 5 if name == "cfg5" else 20
         for _ in range(3):
@@ -37,7 +41,7 @@ with Mapper(0) as m:
         for _ in range(reps):
             idx, mp, ms = m.map_queues(Kd, Xd)
             ts.append(m.last_kernel_time_ms()[0])
-        out[name] = {{"ms": statistics.median(ts), "min": min(ts),
+        out[spec] = {{"ms": statistics.median(ts), "min": min(ts),
                       "res": [int(idx[:64].sum()), int(ms[:64].sum())]}}
 print(json.dumps(out))
 """

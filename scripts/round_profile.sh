@@ -15,7 +15,7 @@ for wl in cfg5 cfg4 cfg2 cfg3; do
   timeout 900 $NCU --set full --clock-control none --import-source on -k regex:search_ -s 2 -c 1 \
       -o gpurun_out/prof_$wl -f python scripts/profile_run.py $wl 3 > /dev/null 2>&1
 done
-timeout 600 $NCU --set full --clock-control none -k regex:build_costs -s 2 -c 1 -o gpurun_out/prof_costs -f \
+timeout 600 $NCU --set full --clock-control none --import-source on -k regex:build_costs -s 2 -c 1 -o gpurun_out/prof_costs -f \
     python scripts/profile_costs.py > /dev/null 2>&1
 python scripts/bench_variants.py --reps 7 > gpurun_out/variants.jsonl 2>&1
 ./scripts/sanitize.sh > gpurun_out/sanitize_summary.txt 2>&1

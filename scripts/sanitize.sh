@@ -4,8 +4,8 @@ cd "${GRAFT_REPO_ROOT:-$(dirname "$0")/..}"
 mkdir -p gpurun_out
 CS=/usr/local/cuda/bin/compute-sanitizer
 run() {  # tool, workload, reps, [epochs]
-  timeout 900 $CS --tool $1 --error-exitcode 9 python scripts/profile_run.py $2 $3 $4 > gpurun_out/sanitize_$1_$2.log 2>&1
-  echo "$1 $2 rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY' gpurun_out/sanitize_$1_$2.log | tail -1)"
+  timeout 900 $CS --tool $1 --error-exitcode 9 python scripts/profile_run.py $2 $3 $4 > gpurun_out/sanitize_$1_$2_$4.log 2>&1
+  echo "$1 $2 rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY' gpurun_out/sanitize_$1_$2_$4.log | tail -1)"
 }
 for tool in memcheck racecheck synccheck; do
   run $tool cfg1 1
@@ -13,3 +13,7 @@ for tool in memcheck racecheck synccheck; do
   run $tool cfg3 1 5000
 done
 run memcheck cfg4 1
+# warp-per-epoch batched kernel: one whole wave (2368 warps) plus split tail epochs
+run memcheck cfg2 1 2400
+run racecheck cfg2 1 2400
+run synccheck cfg2 1 2400

@@ -119,7 +119,8 @@ def test_batch_range_error(torch_cuda, mapper):
 @pytest.mark.parametrize("Q,D", [(9, 3), (8, 4), (8, 5)])
 def test_batch_whole_and_split_epochs(torch_cuda, mapper, Q, D):
     """More epochs than resident warps: whole epochs (one warp each) plus a last partial
-    wave of epochs split over the warps of a CTA, merged in shared memory."""
+    wave of epochs split over the warps of a CTA, merged in shared memory; repeated and
+    interleaved with other batch sizes (below one wave: one warp per epoch)."""
     E = 148 * 16 + 123
     K, X = workloads.small_int_tables(77 * Q + D, E, Q, D, hi=64)
     want = oracle.oracle_map(K, X)
@@ -127,6 +128,9 @@ def test_batch_whole_and_split_epochs(torch_cuda, mapper, Q, D):
         got, info = run(torch_cuda, mapper, K, X, 7)
         assert info["path"] == "batch_u32"
         check(got, want, f"{Q}x{D} E={E} rep {rep}")
+        sub = 3 + 40 * rep  # every epoch split, then whole + split again
+        got, _ = run(torch_cuda, mapper, K[:sub], X[:sub], 7)
+        check(got, tuple(w[:sub] for w in want), f"{Q}x{D} E={sub} after E={E}")
 
 
 def test_batch_single_epoch_and_no_mapping_output(torch_cuda, mapper):
