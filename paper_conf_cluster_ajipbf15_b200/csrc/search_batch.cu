@@ -14,7 +14,8 @@
 //   * lane l walks chunks l, l + 32, ... (D^2 blocks each, the super-block path), keeping
 //     the first strict minimum of its own increasing sequence; the warp takes the
 //     lexicographic minimum of (makespan, super-block index), and re-scans only that
-//     super-block (block by block, 32 leaves per ballot) for the lowest leaf index.
+//     super-block (lane x * D + i takes the leaves (x, i, *, *); one ballot) for the
+//     lowest leaf index.
 // Wave quantisation: whole waves of epochs (one per warp) run first; the epochs of the last,
 // partial wave go one per CTA, its warps splitting the epoch's super-blocks and merging
 // their keys through shared memory (no global atomics or fences). A batch below one wave
@@ -51,6 +52,7 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
   constexpr uint32_t kSb = kChunks * D;                      // super-blocks per epoch
   static_assert(QD <= 64, "two cost entries per lane");
   static_assert(Q >= 6, "chunks need queues 0..Q-6");
+  static_assert(D * D <= 32, "finish: one lane per (x, i) pair of a super-block");
   __shared__ __align__(16) uint64_t sC64[kBatchWarps][QD];
   __shared__ __align__(16) T sC[kBatchWarps][QD];
   __shared__ __align__(16) T sIn[kBatchWarps][8 * D];
@@ -111,22 +113,43 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
     for (int off = 16; off > 0; off >>= 1) key = min(key, __shfl_xor_sync(0xffffffffu, key, off));
     return key;
   };
-  // the lowest leaf inside the winning super-block, then the outputs (a5, a7)
+  // The lowest leaf inside the winning super-block, then the outputs (a5, a7). Leaf
+  // (x, i, j, k) of the super-block has offset ((x * D + i) * D + j) * D + k: lane
+  // x * D + i takes the D^2 leaves (j, k) in order with loads P' = base + C[Q-4][x] on x +
+  // A[i] on i and forms max(M', P'_j + B_j, P'_k + C_k) (j, k static; one sum when j == k;
+  // M' = max P' covers the untouched devices); one ballot finds the lowest lane holding the
+  // target, so the rescan is one pass instead of up to D rounds of block re-scans.
   auto finish = [&](uint64_t e, uint64_t key) {
     const T target = (T)(key >> 32);
     const uint32_t sb = (uint32_t)key;
     T base[D];
     sb_base(sb, base);
-    uint64_t idx = kNone;
-    for (int x = 0; x < D; ++x) {
-      T P[D];
+    const uint32_t x = (uint32_t)lane / D, i = (uint32_t)lane % D;
+    T PB[D], PC[D];
+    T Mp = 0;
 #pragma unroll
-      for (int d = 0; d < D; ++d) P[d] = (x == d) ? base[d] + c4[d] : base[d];
-      const uint32_t leaf = block_first_warp<T, D>(P, in, target);
-      if (leaf != 0xffffffffu) {
-        idx = ((uint64_t)sb * D + (uint64_t)x) * (uint64_t)(D * D * D) + leaf;
-        break;
+    for (int d = 0; d < D; ++d) {
+      T v = base[d];
+      if (x == (uint32_t)d) v += c4[d];
+      if (i == (uint32_t)d) v += in[0 * D + d];
+      Mp = max2(Mp, v);
+      PB[d] = v + in[1 * D + d];
+      PC[d] = v + in[2 * D + d];
+    }
+    uint32_t hit = 0xffffffffu;
+#pragma unroll
+    for (int j = D - 1; j >= 0; --j)
+#pragma unroll
+      for (int k = D - 1; k >= 0; --k) {
+        const T v = (j == k) ? max2(Mp, PB[j] + in[2 * D + j]) : max3(Mp, PB[j], PC[k]);
+        if (v == target) hit = (uint32_t)(j * D + k);
       }
+    const uint32_t m = __ballot_sync(0xffffffffu, lane < D * D && hit != 0xffffffffu);
+    uint64_t idx = kNone;
+    if (m) {
+      const int src = __ffs(m) - 1;
+      const uint32_t t = __shfl_sync(0xffffffffu, hit, src);
+      idx = (uint64_t)sb * (uint64_t)(D * D * D * D) + (uint64_t)src * (D * D) + t;
     }
     if (lane == 0) {
       a.index[e] = idx;
