@@ -16,7 +16,8 @@ ncclAllReduce(MIN) + a decode kernel instead).
 
 Rank 0 prints one JSON line. `value` is whole-job mappings/s from CUDA events over exactly
 K timed steps (L2 flushed between steps, outside the events), max over ranks; `e2e` is the
-same metric through the C ABI with pinned host buffers (H2D + D2H inside the timed region);
+same metric through the C ABI with pinned host buffers (H2D + D2H inside the timed region;
+batched workloads stage in pipelined chunks, `e2e.pipelined_chunks`);
 `roofline` is the dominant kernel's algorithmic ALU-instruction rate against the B200
 ALU-pipe peak; `cpu_baseline` is the CPU oracle timed on a bounded sample of the workload.
 `--impl reference` times the oracle instead (this tier's reference arm).
@@ -347,6 +348,7 @@ def main():
     if world > 1:
         dist.all_reduce(e2e_s, op=dist.ReduceOp.MAX)
     e2e_value = mappings_per_step / float(e2e_s[0])
+    e2e_chunks = mapper.launch_info()["chunks"]  # pipelined staging (mcl_set_pipeline_chunks)
     h2d = 2 * K.nbytes
     d2h = E * (8 + 8 + Q)
 
@@ -400,7 +402,7 @@ def main():
             "clocks": clocks,
             "gpu_launches": launches,
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-                    "ms_per_step": float(e2e_s[0]) * 1e3},
+                    "ms_per_step": float(e2e_s[0]) * 1e3, "pipelined_chunks": e2e_chunks},
             "roofline": roof,
         }
     mapper.close()

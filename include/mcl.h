@@ -254,7 +254,8 @@ const char* mcl_last_error_string(const mcl_mapper_t* h);
  *   info[1] = number of kernels launched by the call, info[2] = CTAs of the main kernel,
  *   info[3] = threads per CTA, info[4] = 1 if an NCCL all-reduce ran, 2 if the fused peer
  *   exchange ran, info[5] = index bits of the packed key, info[6] = 1 if the two-step
- *   reduce ran.
+ *   reduce ran, info[7] = nodes visited (mcl_map_queues_pruned) or the number of chunks of
+ *   a pipelined host-resident call (mcl_set_pipeline_chunks in mcl_ext.h), else 0.
  */
 mcl_status_t mcl_last_launch_info(const mcl_mapper_t* h, int64_t info[8]);
 

@@ -52,6 +52,18 @@ mcl_status_t mcl_probe_int_rate(int device, int op, double* lane_ops_per_s,
    not support (Q, D) or the handle's sharding makes the call fail with MCL_E_INVAL. */
 mcl_status_t mcl_force_path(mcl_mapper_t* h, int path);
 
+/* Pipelined staging of host-resident batches. When every cost table and output of an
+   unconstrained single-GPU mcl_map_queues call is host memory, the epochs are cut into
+   chunks whose host->device copies, search and device->host copies are issued on three
+   rotating streams, so the PCIe copies of one chunk overlap the search of another (the copy
+   engines run both directions at once). Results are identical to the unpipelined call
+   (epochs are independent). chunks: 0 = automatic (default: at least 1.5 MB of K + X per
+   chunk, at most 4 chunks, each at least one wave of the warp-per-epoch kernel: 16 epochs
+   per SM),
+   1 = off, n > 1 = exactly min(n, epochs) chunks. mcl_last_launch_info's info[7] is the
+   number of chunks of a pipelined call (0 otherwise). Errors: MCL_E_INVAL (NULL h, n < 0). */
+mcl_status_t mcl_set_pipeline_chunks(mcl_mapper_t* h, int chunks);
+
 /* Number of SMs of `device` (for roofline bookkeeping). */
 mcl_status_t mcl_device_sms(int device, int* sms);
 

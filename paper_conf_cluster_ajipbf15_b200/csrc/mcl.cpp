@@ -150,6 +150,10 @@ struct mcl_mapper {
   uint32_t hold_us = 0;         // timing aid: spin kernel ahead of the start event
   bool timing_pending = false;  // events recorded, elapsed times not read yet
   int force_path = 0;
+  int pipeline_chunks = 0;      // 0 auto, 1 off, n forced (mcl_set_pipeline_chunks)
+  bool async_call = false;      // pipelined chunk: enqueue only (the wrapper syncs, reads flags)
+  cudaStream_t pipe[3] = {nullptr, nullptr, nullptr};  // pipelined staging streams
+  cudaEvent_t pipe_ev[4] = {nullptr, nullptr, nullptr, nullptr};  // start + per-stream join
   cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
   int64_t info[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   std::string last_err;
@@ -342,6 +346,10 @@ void mcl_mapper_destroy(mcl_mapper_t* h) {
     if (h->flags_host) cudaFreeHost(h->flags_host);
     for (auto& ev : h->ev)
       if (ev) cudaEventDestroy(ev);
+    for (cudaStream_t& ps : h->pipe)
+      if (ps) cudaStreamSynchronize(ps), cudaStreamDestroy(ps);
+    for (cudaEvent_t& pe : h->pipe_ev)
+      if (pe) cudaEventDestroy(pe);
     if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
   }
   delete h;
@@ -364,6 +372,12 @@ mcl_status_t mcl_set_timing(mcl_mapper_t* h, int enable) {
   if (enable < 0 || enable > 2) return MCL_E_INVAL;
   h->timing = enable;
   h->timing_pending = false;
+  return MCL_OK;
+}
+
+mcl_status_t mcl_set_pipeline_chunks(mcl_mapper_t* h, int chunks) {
+  if (!h || chunks < 0) return MCL_E_INVAL;
+  h->pipeline_chunks = chunks;
   return MCL_OK;
 }
 
@@ -527,6 +541,106 @@ cudaError_t record_start(mcl_mapper* h, cudaStream_t s) {
 mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
                       const uint64_t* cost_kernel, const uint64_t* cost_xfer,
                       const uint64_t* base_load, const uint16_t* eligible,
+                      uint64_t* mapping_index, uint8_t* mapping, uint64_t* makespan);
+
+// Chunks of a pipelined host-resident call: at least 1.5 MB of K + X per chunk, at most 4
+// (each chunk costs ~15-20 us of host enqueue and a kernel ramp; measured,
+// scripts/pipeline_study.py: 8 x 4 x 10^4 epochs 0.214 -> 0.186 ms with 2-4 chunks, 2 x 3 x
+// 10^6 epochs 2.10 -> 1.90 ms with 4, worse again at 16), each at least one wave of the
+// warp-per-epoch kernel (16 epochs per SM) so no chunk runs a partly empty GPU; 1 = no
+// pipelining. A forced count (mcl_set_pipeline_chunks) is taken as is.
+uint64_t pipeline_chunk_count(const mcl_mapper* h, uint32_t Q, uint32_t D, uint64_t epochs) {
+  if (h->pipeline_chunks > 1) return std::min<uint64_t>((uint64_t)h->pipeline_chunks, epochs);
+  const uint64_t bytes = 2 * epochs * Q * D * sizeof(uint64_t);
+  uint64_t nc = std::min<uint64_t>(4, bytes / (3u << 19));
+  nc = std::min<uint64_t>(nc, epochs / ((uint64_t)h->num_sms * 16));
+  return std::max<uint64_t>(nc, 1);
+}
+
+// Pipelined staging: chunk c's H2D copies, search and D2H copies go to stream pipe[c % 3]
+// (after the handle's stream, which joins them at the end), so the copies of one chunk
+// overlap the search of another. Each chunk is an ordinary call on device pointers into the
+// staging buffers, enqueued without a sync (async_call); the flags of all chunks are read
+// once at the end. *plain = true: some epoch's bound needs 64-bit loads (every chunk ran
+// the 32-bit kernels), so the caller reruns the whole call unpipelined.
+mcl_status_t map_pipelined(mcl_mapper* h, uint32_t Q, uint32_t D, uint64_t epochs, uint64_t nc,
+                           const uint64_t* Kh, const uint64_t* Xh, uint64_t* idx_h, uint8_t* map_h,
+                           uint64_t* ms_h, bool* plain) {
+  *plain = false;
+  const size_t row = (size_t)Q * D;
+  MCL_CUDA(h, h->in_k.ensure(epochs * row * 8), "cudaMalloc(staging)");
+  MCL_CUDA(h, h->in_x.ensure(epochs * row * 8), "cudaMalloc(staging)");
+  MCL_CUDA(h, h->out_idx.ensure(epochs * 8), "cudaMalloc(staging)");
+  MCL_CUDA(h, h->out_ms.ensure(epochs * 8), "cudaMalloc(staging)");
+  if (map_h) MCL_CUDA(h, h->out_map.ensure(epochs * Q), "cudaMalloc(staging)");
+  for (cudaStream_t& ps : h->pipe)
+    if (!ps) MCL_CUDA(h, cudaStreamCreateWithFlags(&ps, cudaStreamNonBlocking), "cudaStreamCreate(pipe)");
+  for (cudaEvent_t& pe : h->pipe_ev)
+    if (!pe) MCL_CUDA(h, cudaEventCreateWithFlags(&pe, cudaEventDisableTiming), "cudaEventCreate(pipe)");
+  uint64_t* Kd = (uint64_t*)h->in_k.p;
+  uint64_t* Xd = (uint64_t*)h->in_x.p;
+  uint64_t* Id = (uint64_t*)h->out_idx.p;
+  uint64_t* Md = (uint64_t*)h->out_ms.p;
+  uint8_t* Pd = map_h ? (uint8_t*)h->out_map.p : nullptr;
+  const cudaStream_t s0 = h->stream;
+  const int timing = h->timing;
+  const int nstreams = (int)std::min<uint64_t>(nc, 3);
+  clear_flags(h);
+  if (timing >= 2) MCL_CUDA(h, cudaEventRecord(h->ev[2], s0), "cudaEventRecord");
+  MCL_CUDA(h, cudaEventRecord(h->pipe_ev[0], s0), "cudaEventRecord(pipe)");
+  for (int i = 0; i < nstreams; ++i)
+    MCL_CUDA(h, cudaStreamWaitEvent(h->pipe[i], h->pipe_ev[0], 0), "cudaStreamWaitEvent(pipe)");
+  mcl_status_t st = MCL_OK;
+  int64_t launches = 0;
+  h->timing = 0;  // the chunks' own events are not recorded; the span is (below)
+  for (uint64_t c = 0; c < nc && st == MCL_OK; ++c) {
+    const uint64_t lo = epochs * c / nc, hi = epochs * (c + 1) / nc, ec = hi - lo;
+    const cudaStream_t ps = h->pipe[c % 3];
+    cudaError_t e = cudaMemcpyAsync(Kd + lo * row, Kh + lo * row, ec * row * 8, cudaMemcpyHostToDevice, ps);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(Xd + lo * row, Xh + lo * row, ec * row * 8, cudaMemcpyHostToDevice, ps);
+    if (e == cudaSuccess && timing && c == 0) e = cudaEventRecord(h->ev[0], ps);
+    if (e != cudaSuccess) {
+      st = cuda_fail(h, e, "pipelined H2D");
+      break;
+    }
+    h->stream = ps;
+    h->async_call = true;
+    st = map_impl(h, Q, D, ec, Kd + lo * row, Xd + lo * row, nullptr, nullptr, Id + lo,
+                  Pd ? Pd + lo * Q : nullptr, Md + lo);
+    h->async_call = false;
+    h->stream = s0;
+    if (st != MCL_OK) break;
+    launches += h->info[1];
+    if (timing && c == nc - 1) e = cudaEventRecord(h->ev[1], ps);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(idx_h + lo, Id + lo, ec * 8, cudaMemcpyDeviceToHost, ps);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(ms_h + lo, Md + lo, ec * 8, cudaMemcpyDeviceToHost, ps);
+    if (e == cudaSuccess && map_h) e = cudaMemcpyAsync(map_h + lo * Q, Pd + lo * Q, ec * Q, cudaMemcpyDeviceToHost, ps);
+    if (e != cudaSuccess) st = cuda_fail(h, e, "pipelined D2H");
+  }
+  h->timing = timing;
+  // join the pipe streams into the handle's stream, then wait for everything
+  for (int i = 0; i < nstreams; ++i) {
+    cudaEventRecord(h->pipe_ev[1 + i], h->pipe[i]);
+    cudaStreamWaitEvent(s0, h->pipe_ev[1 + i], 0);
+  }
+  if (timing >= 2) cudaEventRecord(h->ev[3], s0);
+  const cudaError_t se = cudaStreamSynchronize(s0);
+  if (st != MCL_OK) return st;
+  MCL_CUDA(h, se, "pipelined call");
+  if ((st = status_from_flags(h)) != MCL_OK) return st;
+  if (*(volatile uint32_t*)h->flags_host & mcl::kFlagNeedU64) {
+    *plain = true;
+    return MCL_OK;
+  }
+  h->info[1] = launches;
+  h->info[7] = (int64_t)nc;
+  h->timing_pending = timing > 0;
+  return MCL_OK;
+}
+
+mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                      const uint64_t* cost_kernel, const uint64_t* cost_xfer,
+                      const uint64_t* base_load, const uint16_t* eligible,
                       uint64_t* mapping_index, uint8_t* mapping, uint64_t* makespan) {
   if (!h) return MCL_E_INVAL;
   h->last_err.clear();
@@ -544,6 +658,26 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
   const bool fused = h->peer_ready && epochs <= h->peer_cap;
   const bool use_nccl = !fused && h->comm != nullptr;
   const bool multi = fused || use_nccl;
+
+  // ---- host-resident batch: pipelined staging (chunks of H2D / search / D2H) ----
+  if (!multi && !base_load && !eligible && h->pipeline_chunks != 1 && !h->async_call && epochs > 1) {
+    bool dk = true, dx = true, di = true, dm = true, dmap = false;
+    if ((st = classify(h, cost_kernel, &dk)) != MCL_OK) return st;
+    if ((st = classify(h, cost_xfer, &dx)) != MCL_OK) return st;
+    if ((st = classify(h, mapping_index, &di)) != MCL_OK) return st;
+    if ((st = classify(h, makespan, &dm)) != MCL_OK) return st;
+    if (mapping && (st = classify(h, mapping, &dmap)) != MCL_OK) return st;
+    if (!dk && !dx && !di && !dm && !dmap) {
+      const uint64_t nc = pipeline_chunk_count(h, Q, D, epochs);
+      if (nc > 1) {
+        bool plain = false;
+        st = map_pipelined(h, Q, D, epochs, nc, cost_kernel, cost_xfer, mapping_index, mapping,
+                           makespan, &plain);
+        if (!plain) return st;  // else a bound needs 64-bit loads: the unpipelined call below
+      }
+    }
+  }
+  h->info[7] = 0;
 
   // ---- where do the buffers live? host buffers are staged through device memory ----
   cudaStream_t s = h->stream;
@@ -612,7 +746,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
 
   int nlaunch = 0;
   for (int attempt = 0; attempt < 2; ++attempt) {
-    clear_flags(h);
+    if (!h->async_call) clear_flags(h);
     nlaunch = 0;
     dim3 grid(1, 1, 1);
     int threads = 0;
@@ -735,6 +869,10 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
       MCL_CUDA(h, mcl::launch_decode_key(out.key, epochs, Q, D, ibits, o_idx, o_ms, o_map, h->flags_dev, s), "decode launch");
       nlaunch += 1;
       h->info[4] = 1;
+    }
+    if (h->async_call) {  // a pipelined chunk: the wrapper syncs and reads the flags
+      h->info[1] = nlaunch;
+      return MCL_OK;
     }
     MCL_CUDA(h, cudaStreamSynchronize(s), "search kernel");
     const uint32_t flags = *(volatile uint32_t*)h->flags_host;

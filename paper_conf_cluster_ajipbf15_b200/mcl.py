@@ -24,7 +24,7 @@ PATH_NAMES = {1: "blocked_u32", 2: "blocked_u64", 3: "generic", 4: "small_batche
 EXPORTED = [
     "mcl_mapper_create", "mcl_map_queues", "mcl_mapper_destroy", "mcl_status_string",
     "mcl_last_error_string", "mcl_last_launch_info", "mcl_version",
-    "mcl_set_timing", "mcl_set_timing_hold", "mcl_last_kernel_time", "mcl_force_path", "mcl_probe_int_rate",
+    "mcl_set_timing", "mcl_set_timing_hold", "mcl_last_kernel_time", "mcl_force_path", "mcl_set_pipeline_chunks", "mcl_probe_int_rate",
     "mcl_device_sms",
     "mcl_comm_unique_id", "mcl_comm_init", "mcl_comm_destroy",
     "mcl_map_queues_constrained", "mcl_score_mappings", "mcl_map_queues_pruned",
@@ -94,6 +94,7 @@ def load_library(path: str | None = None) -> ctypes.CDLL:
         "mcl_set_timing": (i32, [vp, i32]),
         "mcl_set_timing_hold": (i32, [vp, u32]),
         "mcl_force_path": (i32, [vp, i32]),
+        "mcl_set_pipeline_chunks": (i32, [vp, i32]),
         "mcl_last_kernel_time": (i32, [vp, ctypes.POINTER(ctypes.c_float), ctypes.POINTER(ctypes.c_float)]),
         "mcl_probe_int_rate": (i32, [i32, i32, ctypes.POINTER(ctypes.c_double),
                                      ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]),
@@ -422,7 +423,8 @@ class Mapper:
         i = mcl_last_launch_info(self.handle)
         return {"path": PATH_NAMES.get(i[0], str(i[0])), "launches": i[1], "ctas": i[2],
                 "threads": i[3], "allreduce": bool(i[4]), "fused_exchange": i[4] == 2,
-                "index_bits": i[5], "two_step": bool(i[6]), "nodes": i[7]}
+                "index_bits": i[5], "two_step": bool(i[6]),
+                "nodes": i[7] if i[0] == 6 else 0, "chunks": i[7] if i[0] != 6 else 0}
 
     def peer_export(self, max_epochs: int = 1) -> bytes:
         """Allocate this rank's exchange slab for the fused cross-GPU exchange and return
@@ -452,6 +454,13 @@ class Mapper:
         got: list = [None] * world
         dist.all_gather_object(got, mine, group=group)
         self.peer_import(got, timeout_ms)
+
+    def set_pipeline_chunks(self, chunks: int) -> None:
+        """Pipelined staging of host-resident batches (include/mcl_ext.h
+        mcl_set_pipeline_chunks): 0 automatic, 1 off, n > 1 exactly n chunks."""
+        st = load_library().mcl_set_pipeline_chunks(self.handle, chunks)
+        if st != MCL_OK:
+            raise MclError(st, "mcl_set_pipeline_chunks")
 
     def force_path(self, path: int) -> None:
         """Testing aid: 0 auto, 1 blocked u32 (CTA per epoch), 2 blocked u64, 3 generic,

@@ -1,0 +1,137 @@
+"""GPU parity of the pipelined staging of host-resident batches (include/mcl_ext.h
+mcl_set_pipeline_chunks): every chunk's H2D copy, search and D2H copy on rotating streams.
+The results must equal the oracle's (and the unpipelined call's) bit for bit, for any chunk
+count, ragged chunk sizes, every batched kernel path, with and without the mapping output,
+and through the 64-bit rerun and range errors. Run with ``pytest -m gpu``.
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import oracle
+from conftest import cuda_available
+from paper_conf_cluster_ajipbf15_b200 import workloads
+from paper_conf_cluster_ajipbf15_b200.mcl import MCL_E_RANGE, Mapper, MclError
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    if not cuda_available():
+        pytest.fail("no CUDA device: the -m gpu tests must run on a GPU box")
+    import torch
+
+    return torch
+
+
+@pytest.fixture(scope="module")
+def mapper(torch_cuda):
+    m = Mapper(0)
+    yield m
+    m.close()
+
+
+def host_call(torch, m, K, X, with_mapping=True, pinned=True):
+    E, Q, _ = K.shape
+    Kh, Xh = torch.from_numpy(np.ascontiguousarray(K)), torch.from_numpy(np.ascontiguousarray(X))
+    idx = torch.empty(E, dtype=torch.uint64)
+    ms = torch.empty(E, dtype=torch.uint64)
+    mp = torch.empty((E, Q), dtype=torch.uint8) if with_mapping else None
+    if pinned:
+        Kh, Xh, idx, ms = Kh.pin_memory(), Xh.pin_memory(), idx.pin_memory(), ms.pin_memory()
+        mp = mp.pin_memory() if mp is not None else None
+    m.map_queues_into(Kh, Xh, idx, mp, ms)
+    return idx.numpy(), (mp.numpy() if mp is not None else None), ms.numpy()
+
+
+def check(got, want, ctx, with_mapping=True):
+    gi, gmp, gms = got
+    wi, wms, wmp = want
+    bad = np.nonzero((gi != wi) | (gms != wms))[0]
+    assert bad.size == 0, f"{ctx}: {bad.size} epochs differ, first {bad[:5]}"
+    if with_mapping:
+        assert (gmp == wmp).all(), ctx
+
+
+@pytest.mark.parametrize("chunks", [2, 3, 5, 7])
+def test_pipelined_chunks_cfg2_shape(torch_cuda, mapper, chunks):
+    """8 x 4 batches (warp-per-epoch / CTA-per-epoch kernels per chunk), ragged chunk sizes."""
+    K, X = workloads.cfg2(E=3001, seed=31)
+    want = oracle.oracle_map(K, X)
+    mapper.set_pipeline_chunks(chunks)
+    try:
+        got = host_call(torch_cuda, mapper, K, X)
+        assert mapper.launch_info()["chunks"] == chunks
+    finally:
+        mapper.set_pipeline_chunks(0)
+    check(got, want, f"chunks={chunks}")
+
+
+def test_pipelined_small_kernel_and_pageable(torch_cuda, mapper):
+    """2 x 3 batches (thread-per-epoch kernel per chunk); pageable host buffers too."""
+    K, X = workloads.cfg3(E=200_003, seed=32)
+    want = oracle.oracle_map(K, X)
+    mapper.set_pipeline_chunks(6)
+    try:
+        for pinned in (True, False):
+            got = host_call(torch_cuda, mapper, K, X, pinned=pinned)
+            assert mapper.launch_info()["chunks"] == 6
+            check(got, want, f"cfg3 pinned={pinned}")
+    finally:
+        mapper.set_pipeline_chunks(0)
+
+
+def test_pipelined_auto_matches_unpipelined(torch_cuda, mapper):
+    """The automatic chunking of a full cfg2 batch (4 chunks of one wave or more) and the
+    unpipelined staged call return identical outputs; no mapping output (NULL) works."""
+    K, X = workloads.cfg2()
+    got_auto = host_call(torch_cuda, mapper, K, X)
+    assert mapper.launch_info()["chunks"] > 1
+    mapper.set_pipeline_chunks(1)
+    try:
+        got_off = host_call(torch_cuda, mapper, K, X)
+        assert mapper.launch_info()["chunks"] == 0
+    finally:
+        mapper.set_pipeline_chunks(0)
+    for a, b in zip(got_auto, got_off):
+        assert (a == b).all()
+    check(got_auto, oracle.oracle_map(K, X), "cfg2 auto")
+    gi, _, gms = host_call(torch_cuda, mapper, K, X, with_mapping=False)
+    assert (gi == got_auto[0]).all() and (gms == got_auto[2]).all()
+
+
+def test_pipelined_u64_rerun_and_range_error(torch_cuda, mapper):
+    """A chunk whose bound needs 64-bit loads makes the whole call rerun unpipelined (same
+    outputs as the oracle); an entry >= 2^48 in any chunk fails the call, and the next call
+    is exact."""
+    K, X = workloads.random_tables(33, 64, 8, 4)
+    K[50] = np.random.default_rng(2).integers(1 << 46, 1 << 47, size=(8, 4), dtype=np.uint64)
+    mapper.set_pipeline_chunks(4)
+    try:
+        got = host_call(torch_cuda, mapper, K, X)
+        assert mapper.launch_info()["path"] == "blocked_u64"
+        assert mapper.launch_info()["chunks"] == 0
+        check(got, oracle.oracle_map(K, X), "u64 rerun")
+        K2, X2 = workloads.random_tables(34, 64, 8, 4)
+        X2[40, 1, 2] = 1 << 48
+        with pytest.raises(MclError) as ei:
+            host_call(torch_cuda, mapper, K2, X2)
+        assert ei.value.status == MCL_E_RANGE
+        X2[40, 1, 2] = 9
+        got = host_call(torch_cuda, mapper, K2, X2)
+        check(got, oracle.oracle_map(K2, X2), "after range error")
+    finally:
+        mapper.set_pipeline_chunks(0)
+
+
+def test_pipelined_more_chunks_than_epochs(torch_cuda, mapper):
+    K, X = workloads.random_tables(35, 3, 9, 3)
+    mapper.set_pipeline_chunks(16)
+    try:
+        got = host_call(torch_cuda, mapper, K, X)
+        assert mapper.launch_info()["chunks"] == 3
+    finally:
+        mapper.set_pipeline_chunks(0)
+    check(got, oracle.oracle_map(K, X), "E=3, 16 chunks requested")
