@@ -18,5 +18,6 @@ done
 timeout 600 $NCU --set full --clock-control none --import-source on -k regex:build_costs -s 2 -c 1 -o gpurun_out/prof_costs -f \
     python scripts/profile_costs.py > /dev/null 2>&1
 python scripts/bench_variants.py --reps 7 > gpurun_out/variants.jsonl 2>&1
+python scripts/pipeline_study.py > gpurun_out/pipeline_study.jsonl 2>&1
 ./scripts/sanitize.sh > gpurun_out/sanitize_summary.txt 2>&1
 ls gpurun_out
