@@ -60,6 +60,8 @@ def parse():
     p.add_argument("--workload", default="cfg5", choices=["cfg1", "cfg2", "cfg3", "cfg4", "cfg5"])
     p.add_argument("--impl", default="mcl", choices=["mcl", "reference"])
     p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--pipeline-chunks", type=int, default=0,
+                   help="e2e staging of the host-resident batch: 0 auto, 1 off, n chunks")
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="CPU-oracle sample budget")
     p.add_argument("--collective", default="auto", choices=["auto", "fused", "nccl"],
                    help="cross-GPU combine of a sharded single-epoch search: fused = in-kernel "
@@ -78,6 +80,27 @@ def workload(name):
 
 def is_batched(w):
     return w["E"] > 1
+
+
+def gpu_local_cpus(device_index):
+    """CPUs of the NUMA node the GPU hangs off (sysfs local_cpulist of its PCI device), or
+    None when unknown."""
+    try:
+        import pynvml
+
+        pynvml.nvmlInit()
+        bus = pynvml.nvmlDeviceGetPciInfo(pynvml.nvmlDeviceGetHandleByIndex(device_index)).busId
+        bus = bus.decode() if isinstance(bus, bytes) else bus
+        bus = bus.lower()[-12:]  # domain:bus:device.function as sysfs names it
+        text = open(f"/sys/bus/pci/devices/{bus}/local_cpulist").read().strip()
+        cpus = set()
+        for part in text.split(","):
+            a, _, b = part.partition("-")
+            cpus.update(range(int(a), int(b or a) + 1))
+        cpus &= os.sched_getaffinity(0)
+        return cpus or None
+    except Exception:
+        return None
 
 
 # ------------------------------------------------------------------ clocks -----------
@@ -227,6 +250,27 @@ def main():
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    # Pinned host arena for the e2e leg, allocated first, in one piece, from the CPUs of the
+    # GPU's NUMA node: on the pool's VMs later / separate pinned allocations copied at 14-47
+    # instead of 53 GB/s (scripts/e2e_dbg.py), which made the e2e time bimodal by process.
+    E0, Q0 = w["E"], w["Q"]
+    sizes = [K.nbytes, X.nbytes, E0 * 8, E0 * 8, E0 * Q0]
+    offs = [0]
+    for n in sizes:
+        offs.append(offs[-1] + (n + 255) // 256 * 256)
+    prev_cpus = os.sched_getaffinity(0)
+    local_cpus = gpu_local_cpus(local)
+    if local_cpus:
+        os.sched_setaffinity(0, local_cpus)
+    arena = torch.empty(offs[-1], dtype=torch.uint8, pin_memory=True)
+    os.sched_setaffinity(0, prev_cpus)
+    Kh = arena[offs[0]:offs[0] + sizes[0]].view(torch.uint64).view(K.shape)
+    Xh = arena[offs[1]:offs[1] + sizes[1]].view(torch.uint64).view(X.shape)
+    ih = arena[offs[2]:offs[2] + sizes[2]].view(torch.uint64)
+    mh = arena[offs[3]:offs[3] + sizes[3]].view(torch.uint64)
+    ph = arena[offs[4]:offs[4] + sizes[4]].view(E0, Q0)
+    Kh.copy_(torch.from_numpy(K))
+    Xh.copy_(torch.from_numpy(X))
     explicit = args.collective != "auto"
     if world > 1 or explicit:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
@@ -331,13 +375,11 @@ def main():
         assert all((g == res).all() for g in gathered), "ranks disagree on the argmin"
 
     # ---- e2e through the C ABI with pinned host buffers (H2D + D2H inside the region) ----
-    Kh = torch.from_numpy(K).pin_memory()
-    Xh = torch.from_numpy(X).pin_memory()
-    ih = torch.empty(E, dtype=torch.uint64).pin_memory()
-    mh = torch.empty(E, dtype=torch.uint64).pin_memory()
-    ph = torch.empty((E, Q), dtype=torch.uint8).pin_memory()
-    e2e_steps = max(3, min(args.steps, 10))
-    mapper.map_queues_into(Kh, Xh, ih, ph, mh)
+    # (host buffers: the pinned arena allocated at start-up)
+    e2e_steps = max(10, args.steps)
+    mapper.set_pipeline_chunks(args.pipeline_chunks)
+    for _ in range(max(3, args.warmup)):
+        mapper.map_queues_into(Kh, Xh, ih, ph, mh)
     assert (ih[:1].numpy() == idx[:1].cpu().numpy()).all()
     if world > 1:
         dist.barrier()
@@ -402,7 +444,9 @@ def main():
             "clocks": clocks,
             "gpu_launches": launches,
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-                    "ms_per_step": float(e2e_s[0]) * 1e3, "pipelined_chunks": e2e_chunks},
+                    "ms_per_step": float(e2e_s[0]) * 1e3, "pipelined_chunks": e2e_chunks,
+                    "host_buffers": "one pinned arena allocated at start-up on the GPU's NUMA node"
+                    if local_cpus else "one pinned arena allocated at start-up"},
             "roofline": roof,
         }
     mapper.close()
