@@ -92,3 +92,36 @@ def test_map_from_profiles(torch_cuda, mapper, E, Q, D):
     want = oracle.oracle_map_constrained(K, X, base, elig)
     idx, mp, ms = mapper.map_from_profiles(on_device(torch_cuda, m), D, base, elig)
     assert (idx == want[0]).all() and (ms == want[1]).all() and (mp == want[2]).all()
+
+
+def test_build_costs_many_tiles_long_lists_misaligned(torch_cuda, mapper):
+    """Many tiles per persistent CTA (E x Q pairs well above 256 x the resident CTAs), tiles
+    whose invocation lists are long (~25k ids per 256-pair tile), a mix of long and short
+    lists in one call, and an ids array that starts 4 bytes past a 16-byte boundary."""
+    torch = torch_cuda
+    cases = [
+        workloads.cost_model(91, 40_000, 8, 4),                     # 1250 tiles, ~8.5 ids per pair
+        workloads.cost_model(92, 700, 4, 3, max_kernels=200),       # ~25k ids per tile
+    ]
+    mixed = workloads.cost_model(93, 3000, 4, 3)
+    counts = np.diff(mixed["offsets"].astype(np.int64))
+    counts[: 256 * 3] = 60                                          # the first tiles: long lists
+    mixed["offsets"] = np.concatenate([[0], np.cumsum(counts)]).astype(np.uint64)
+    mixed["kernel_ids"] = np.random.default_rng(4).integers(0, 64, int(counts.sum())).astype(np.uint32)
+    cases.append(mixed)
+    for m in cases:
+        Q, D = m["bytes"].shape[1], m["profile"].shape[1]
+        want_k, want_x = oracle.oracle_build_costs(Q, D, m)
+        Kd, Xd = mapper.build_costs(on_device(torch, m), D, device_out=True)
+        assert (Kd.cpu().numpy() == want_k).all() and (Xd.cpu().numpy() == want_x).all()
+    # misaligned ids: a device view starting one element into a 16-byte-aligned allocation
+    m = workloads.cost_model(94, 5000, 8, 4)
+    want_k, want_x = oracle.oracle_build_costs(8, 4, m)
+    dm = on_device(torch, m)
+    ids = m["kernel_ids"]
+    padded = torch.zeros(ids.size + 1, dtype=torch.int32, device="cuda")
+    padded[1:] = torch.from_numpy(ids.view(np.int32)).cuda()
+    dm["kernel_ids"] = padded[1:].view(torch.uint32)
+    assert dm["kernel_ids"].data_ptr() % 16 == 4
+    Kd, Xd = mapper.build_costs(dm, 4, device_out=True)
+    assert (Kd.cpu().numpy() == want_k).all() and (Xd.cpu().numpy() == want_x).all()
