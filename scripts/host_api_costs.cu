@@ -1,8 +1,9 @@
 // host_api_costs.cu -- host-side cost of the CUDA runtime calls one synchronous
 // mcl_map_queues makes (scripts/host_overhead.py measures the whole call).
-//   nvcc -gencode arch=compute_100a,code=sm_100a -O2 -o /tmp/hac scripts/host_api_costs.cu
+//   nvcc -gencode arch=compute_100a,code=sm_100a -O2 -o /tmp/hac scripts/host_api_costs.cu -lcuda
 #include <chrono>
 #include <cstdio>
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 __global__ void tiny(int* p) {
@@ -52,6 +53,29 @@ int main() {
            while (*(volatile int*)hp == 0) {
            }
          }));
+  printf("launch + cudaStreamQuery spin %.3f us\n", per_call_us([&] {
+           tiny<<<1, 32, 0, s>>>(d);
+           while (cudaStreamQuery(s) == cudaErrorNotReady) {
+           }
+         }));
+  unsigned int* hv;
+  cudaHostAlloc((void**)&hv, 64, cudaHostAllocMapped);
+  unsigned int* dv;
+  cudaHostGetDevicePointer((void**)&dv, hv, 0);
+  CUstream cs = (CUstream)s;
+  unsigned int seq = 0;
+  printf("launch + cuStreamWriteValue32 + poll %.3f us\n", per_call_us([&] {
+           tiny<<<1, 32, 0, s>>>(d);
+           ++seq;
+           cuStreamWriteValue32(cs, (CUdeviceptr)dv, seq, 0);
+           while (*(volatile unsigned int*)hv != seq) {
+           }
+         }));
+  cudaStreamSynchronize(s);
+  printf("cuStreamWriteValue32 enqueue alone %.3f us\n", per_call_us([&] {
+           cuStreamWriteValue32(cs, (CUdeviceptr)dv, ++seq, 0);
+         }));
+  cudaStreamSynchronize(s);
   printf("%s\n", cudaGetErrorString(cudaGetLastError()));
   return 0;
 }
