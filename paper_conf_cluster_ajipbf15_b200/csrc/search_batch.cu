@@ -56,6 +56,10 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
   __shared__ __align__(16) uint64_t sC64[kBatchWarps][QD];
   __shared__ __align__(16) T sC[kBatchWarps][QD];
   __shared__ __align__(16) T sIn[kBatchWarps][8 * D];
+  // one-hot rows of the outer queues 0..Q-5: sV[q][x][d] = C[q][x] if d == x else 0, so a
+  // digit's prefix contribution is one vector load instead of D compare-and-selects
+  constexpr int kVN = (Q - 4) * D * D;
+  __shared__ __align__(16) T sV[kBatchWarps][kVN];
   __shared__ uint64_t s_key[2][kBatchWarps];  // split epochs: each warp's key (double-buffered)
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   uint64_t* C64 = sC64[wib];
@@ -84,8 +88,8 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
   if (unit_epoch(0) < a.E) prefetch(unit_epoch(0));
 
   const T* c4 = in + 7 * D;
-  const T* Cy = Cs + (Q - 5) * D;
   // prefix loads of chunk c: one-hot costs of queues 0..Q-6 on their digits' devices
+  T* V = sV[wib];
   auto chunk_base = [&](uint32_t c, T (&b)[D]) {
 #pragma unroll
     for (int d = 0; d < D; ++d) b[d] = 0;
@@ -93,18 +97,18 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
     for (int q = Q - 6; q >= 0; --q) {
       const uint32_t dq = c % D;
       c /= D;
+      const T* row = V + (q * D + dq) * D;
 #pragma unroll
-      for (int d = 0; d < D; ++d) b[d] = add_f(b[d], (dq == (uint32_t)d) ? Cs[q * D + d] : T(0), one);
+      for (int d = 0; d < D; ++d) b[d] = add_f(b[d], row[d], one);
     }
   };
   // prefix loads of super-block sb = chunk * D + y
   auto sb_base = [&](uint32_t sb, T (&b)[D]) {
     T b2[D];
     chunk_base(sb / D, b2);
-    const uint32_t y = sb % D;
-    const T cy = Cy[y];
+    const T* row = V + ((Q - 5) * D + sb % D) * D;
 #pragma unroll
-    for (int d = 0; d < D; ++d) b[d] = add_f(b2[d], (y == (uint32_t)d) ? cy : T(0), one);
+    for (int d = 0; d < D; ++d) b[d] = add_f(b2[d], row[d], one);
   };
   // a warp's lexicographic minimum of (makespan << 32 | super-block)
   auto warp_key = [&](T best, uint32_t best_sb) {
@@ -209,6 +213,10 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
         in[6 * D + lane] = A + B + Cc;
         in[7 * D + lane] = (T)C64[(Q - 4) * D + lane];
       }
+      for (int t = lane; t < kVN; t += 32) {
+        const int q = t / (D * D), x = (t / D) % D, d = t % D;
+        V[t] = (d == x) ? (T)C64[q * D + x] : T(0);
+      }
       __syncwarp();
       // ---- a2-a5: each lane walks its share in increasing order, first strict minimum ----
       T best = ~T(0);
@@ -218,10 +226,10 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
           T base2[D];
           chunk_base(c, base2);
           for (int y = 0; y < D; ++y) {
-            const T cy = Cy[y];
+            const T* row = V + ((Q - 5) * D + y) * D;
             T base[D];
 #pragma unroll
-            for (int d = 0; d < D; ++d) base[d] = add_f(base2[d], (y == d) ? cy : T(0), one);
+            for (int d = 0; d < D; ++d) base[d] = add_f(base2[d], row[d], one);
             const T gs = superblock_eval<T, D>(base, in, c4, one);
             if (gs < best) {
               best = gs;
