@@ -557,6 +557,17 @@ uint64_t pipeline_chunk_count(const mcl_mapper* h, uint32_t Q, uint32_t D, uint6
   return std::max<uint64_t>(nc, 1);
 }
 
+// Chunk boundaries of a pipelined call: with three or more chunks the first and the last
+// are half as large as the others, so the search starts after a short first copy and only a
+// short search remains after the last copy (the middle chunks' searches overlap the copies).
+uint64_t chunk_edge(uint64_t epochs, uint64_t nc, uint64_t c) {
+  if (c >= nc) return epochs;
+  if (nc < 3) return epochs * c / nc;
+  // weights 1/2, 1, ..., 1, 1/2: cumulative weight of chunks [0, c) is c - 1/2 (c >= 1)
+  const uint64_t twice = c == 0 ? 0 : 2 * c - 1;  // in halves, of 2 * (nc - 1) halves
+  return (uint64_t)(((__uint128_t)epochs * twice) / (2 * (nc - 1)));
+}
+
 // Pipelined staging: chunk c's H2D copies, search and D2H copies go to stream pipe[c % 3]
 // (after the handle's stream, which joins them at the end), so the copies of one chunk
 // overlap the search of another. Each chunk is an ordinary call on device pointers into the
@@ -593,12 +604,15 @@ mcl_status_t map_pipelined(mcl_mapper* h, uint32_t Q, uint32_t D, uint64_t epoch
   mcl_status_t st = MCL_OK;
   int64_t launches = 0;
   h->timing = 0;  // the chunks' own events are not recorded; the span is (below)
+  bool started = false;  // ev[0] goes before the first non-empty chunk's search
   for (uint64_t c = 0; c < nc && st == MCL_OK; ++c) {
-    const uint64_t lo = epochs * c / nc, hi = epochs * (c + 1) / nc, ec = hi - lo;
+    const uint64_t lo = chunk_edge(epochs, nc, c), hi = chunk_edge(epochs, nc, c + 1), ec = hi - lo;
+    if (ec == 0) continue;
     const cudaStream_t ps = h->pipe[c % 3];
     cudaError_t e = cudaMemcpyAsync(Kd + lo * row, Kh + lo * row, ec * row * 8, cudaMemcpyHostToDevice, ps);
     if (e == cudaSuccess) e = cudaMemcpyAsync(Xd + lo * row, Xh + lo * row, ec * row * 8, cudaMemcpyHostToDevice, ps);
-    if (e == cudaSuccess && timing && c == 0) e = cudaEventRecord(h->ev[0], ps);
+    if (e == cudaSuccess && timing && !started) e = cudaEventRecord(h->ev[0], ps);
+    started = true;
     if (e != cudaSuccess) {
       st = cuda_fail(h, e, "pipelined H2D");
       break;
