@@ -135,3 +135,26 @@ def test_pipelined_more_chunks_than_epochs(torch_cuda, mapper):
     finally:
         mapper.set_pipeline_chunks(0)
     check(got, oracle.oracle_map(K, X), "E=3, 16 chunks requested")
+
+
+def test_pipelined_on_external_stream_with_timing(torch_cuda):
+    """A handle on a caller's stream: pipelined host calls interleaved with device calls on
+    the same handle, kernel timing on (the span from the first chunk's search to the last's
+    is reported), every result exact."""
+    torch = torch_cuda
+    stream = torch.cuda.Stream()
+    K, X = workloads.cfg2(E=2600, seed=36)
+    want = oracle.oracle_map(K, X)
+    Kd, Xd = torch.from_numpy(K).cuda(), torch.from_numpy(X).cuda()
+    with Mapper(0, stream=stream.cuda_stream) as m:
+        m.set_timing(True)
+        m.set_pipeline_chunks(3)
+        for rep in range(3):
+            got = host_call(torch, m, K, X)
+            assert m.launch_info()["chunks"] == 3
+            assert m.last_kernel_time_ms()[0] > 0
+            check(got, want, f"pipelined rep {rep}")
+            with torch.cuda.stream(stream):
+                idx, mp, ms = m.map_queues(Kd, Xd)
+                stream.synchronize()
+            assert (idx.cpu().numpy() == want[0]).all() and (ms.cpu().numpy() == want[1]).all()
