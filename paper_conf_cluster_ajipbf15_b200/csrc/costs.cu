@@ -41,6 +41,11 @@ __device__ __forceinline__ uint64_t transfer_ns(uint64_t bytes, double bw) {
 
 constexpr int kCostTile = 256;        // (epoch, queue) pairs per CTA tile (= blockDim.x)
 constexpr int kProfCapBytes = 32768;  // profile table staged when it fits
+// Row stride of the staged profile table in u64 words: odd, so the rows of a warp's random
+// kernel ids spread over 16 bank pairs instead of 32 / (2 D) (a stride of 4 words put every
+// row on one of 4 bank groups: 8-way conflicts on each 64-bit row load).
+template <int D>
+__host__ __device__ constexpr int prof_stride() { return D % 2 ? D : D + 1; }
 
 // Memory pipeline: a persistent CTA walks its tiles with each thread's next pair (CSR
 // offsets, bytes, source, cached mask) loaded into registers while the current pair is
@@ -62,14 +67,15 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
   double* s_h2d = reinterpret_cast<double*>(s_sizes + M);
   double* s_d2h = s_h2d + (size_t)D * M;
   uint64_t* s_prof = reinterpret_cast<uint64_t*>(s_d2h + (size_t)D * M);
-  const bool prof_in_smem = (size_t)a.num_kernels * D * 8 <= (size_t)kProfCapBytes;
+  constexpr int PS = prof_stride<D>();
+  const bool prof_in_smem = (size_t)a.num_kernels * PS * 8 <= (size_t)kProfCapBytes;
   for (uint32_t t = tid; t < M; t += blockDim.x) s_sizes[t] = a.sizes[t];
   for (uint32_t t = tid; t < D * M; t += blockDim.x) {
     s_h2d[t] = a.h2d[t];
     s_d2h[t] = a.d2h[t];
   }
   if (prof_in_smem)
-    for (uint32_t t = tid; t < a.num_kernels * D; t += blockDim.x) s_prof[t] = a.profile[t];
+    for (uint32_t t = tid; t < a.num_kernels * D; t += blockDim.x) s_prof[(t / D) * PS + t % D] = a.profile[t];
   __syncthreads();
   const uint64_t* prof = prof_in_smem ? s_prof : a.profile;
   uint32_t status = 0;
@@ -117,7 +123,7 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
             ok = false;
             break;
           }
-          const uint64_t* row = prof + (uint64_t)kid * D;
+          const uint64_t* row = prof + (uint64_t)kid * (prof_in_smem ? PS : D);
 #pragma unroll
           for (int d = 0; d < D; ++d) k[d] += row[d];
         }
@@ -180,7 +186,8 @@ namespace {
 template <int D>
 cudaError_t launch_build_costs_t(const CostArgs& a, int num_sms, cudaStream_t st) {
   size_t smem = 2 * (size_t)kCostTile * D * 8 + (size_t)a.M * 8 + 2 * (size_t)D * a.M * 8;
-  if ((size_t)a.num_kernels * D * 8 <= (size_t)kProfCapBytes) smem += (size_t)a.num_kernels * D * 8;
+  if ((size_t)a.num_kernels * prof_stride<D>() * 8 <= (size_t)kProfCapBytes)
+    smem += (size_t)a.num_kernels * prof_stride<D>() * 8;
   auto k = build_costs_kernel<D>;
   static SmemAttrCache cache;
   cudaError_t err = ensure_smem(k, smem, cache);
