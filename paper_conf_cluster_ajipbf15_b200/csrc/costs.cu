@@ -74,8 +74,22 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
     s_h2d[t] = a.h2d[t];
     s_d2h[t] = a.d2h[t];
   }
-  if (prof_in_smem)
-    for (uint32_t t = tid; t < a.num_kernels * D; t += blockDim.x) s_prof[(t / D) * PS + t % D] = a.profile[t];
+  // Profiles that all fit 32 bits (kernel times below 4.3 s) are staged as u32 rows of odd
+  // stride PS32: one 4-byte shared load per (id, device) instead of an 8-byte one, half the
+  // shared-memory wavefronts of the sum; the sums stay 64-bit.
+  constexpr int PS32 = D % 2 ? D : D + 1;
+  uint32_t* s_prof32 = reinterpret_cast<uint32_t*>(s_prof);
+  bool fits32 = false;
+  if (prof_in_smem) {
+    bool big = false;
+    for (uint32_t t = tid; t < a.num_kernels * D; t += blockDim.x) big |= (a.profile[t] >> 32) != 0;
+    fits32 = !__syncthreads_or(big);
+    if (fits32)
+      for (uint32_t t = tid; t < a.num_kernels * D; t += blockDim.x)
+        s_prof32[(t / D) * PS32 + t % D] = (uint32_t)a.profile[t];
+    else
+      for (uint32_t t = tid; t < a.num_kernels * D; t += blockDim.x) s_prof[(t / D) * PS + t % D] = a.profile[t];
+  }
   __syncthreads();
   const uint64_t* prof = prof_in_smem ? s_prof : a.profile;
   uint32_t status = 0;
@@ -115,7 +129,19 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
 #pragma unroll
       for (int d = 0; d < D; ++d) k[d] = 0;
       bool ok = j0 <= j1 && j1 <= a.nnz;
-      if (ok) {
+      if (ok && fits32) {
+#pragma unroll 4
+        for (uint64_t j = j0; j < j1; ++j) {
+          const uint32_t kid = __ldg(a.ids + j);
+          if (kid >= a.num_kernels) {
+            ok = false;
+            break;
+          }
+          const uint32_t* row = s_prof32 + (size_t)kid * PS32;
+#pragma unroll
+          for (int d = 0; d < D; ++d) k[d] += row[d];
+        }
+      } else if (ok) {
 #pragma unroll 4
         for (uint64_t j = j0; j < j1; ++j) {
           const uint32_t kid = __ldg(a.ids + j);

@@ -55,6 +55,7 @@ def test_build_costs_edge_models(torch_cuda, mapper):
         dict(m, bytes=m["sizes"][np.arange(E * Q) % len(m["sizes"])].reshape(E, Q)),  # exactly at samples
         dict(m, offsets=np.zeros(E * Q + 1, np.uint64), kernel_ids=np.zeros(0, np.uint32)),  # no kernels
         dict(m, sizes=m["sizes"][:1], h2d_bw=m["h2d_bw"][:, :1], d2h_bw=m["d2h_bw"][:, :1]),  # one sample
+        dict(m, profile=m["profile"] * np.uint64(1 << 20)),               # entries >= 2^32: 64-bit rows
     ]
     for v in variants:
         want = oracle.oracle_build_costs(Q, D, v)
