@@ -146,3 +146,19 @@ def test_score_mappings(torch_cuda, mapper):
     with pytest.raises(MclError) as e:
         mapper.score_mappings(K, X, bad)
     assert e.value.status == MCL_E_INVAL
+
+
+@pytest.mark.parametrize("Q,D", [(5, 1), (6, 3), (9, 7), (4, 16), (12, 5)])
+def test_score_mappings_every_device_count(torch_cuda, mapper, Q, D):
+    """The scoring kernel is compiled per device count: random mappings with and without
+    base loads equal the oracle's scores for several D up to 16."""
+    torch = torch_cuda
+    E = 300
+    K, X = workloads.random_tables(60 + D, E, Q, D)
+    base = np.random.default_rng(D).integers(0, 1 << 20, size=(E, D), dtype=np.uint64)
+    mps = np.random.default_rng(100 + D).integers(0, D, size=(E, Q)).astype(np.uint8)
+    got = mapper.score_mappings(dev(torch, K), dev(torch, X), dev(torch, mps), dev(torch, base)).cpu().numpy()
+    want = np.array([oracle.oracle_score_base(K[e], X[e], base[e], mps[e]) for e in range(E)], np.uint64)
+    assert (got == want).all()
+    got = mapper.score_mappings(K, X, mps)
+    assert (got == np.array([oracle.oracle_score(K[e], X[e], mps[e]) for e in range(E)], np.uint64)).all()
