@@ -59,8 +59,9 @@ mcl_status_t mcl_force_path(mcl_mapper_t* h, int path);
    engines run both directions at once). Results are identical to the unpipelined call
    (epochs are independent). chunks: 0 = automatic (default: at least 1.5 MB of K + X per
    chunk, at most 4 chunks, each at least one wave of the warp-per-epoch kernel: 16 epochs
-   per SM),
-   1 = off, n > 1 = exactly min(n, epochs) chunks. mcl_last_launch_info's info[7] is the
+   per SM), 1 = off, n > 1 = exactly min(n, epochs) chunks. With three or more chunks the
+   first and the last hold half as many epochs as the others (a short first copy before the
+   first search, a short search after the last copy). mcl_last_launch_info's info[7] is the
    number of chunks of a pipelined call (0 otherwise). Errors: MCL_E_INVAL (NULL h, n < 0). */
 mcl_status_t mcl_set_pipeline_chunks(mcl_mapper_t* h, int chunks);
 
