@@ -123,3 +123,11 @@ def test_fuzz_every_path(torch_cuda, mapper, seed):
         finally:
             mapper.force_path(0)
         assert (i.cpu().numpy() == want[0]).all() and (ms.cpu().numpy() == want[1]).all()
+        if E > 1:  # host buffers through the pipelined staging, a random chunk count
+            mapper.set_pipeline_chunks(int(rng.integers(2, 6)))
+            try:
+                i, mp, ms = mapper.map_queues(K, X)
+            finally:
+                mapper.set_pipeline_chunks(0)
+            ctx = f"Q={Q} D={D} E={E} hi={hi} pipelined"
+            assert (i == want[0]).all() and (ms == want[1]).all() and (mp == want[2]).all(), ctx
