@@ -190,9 +190,73 @@ __global__ void __launch_bounds__(256) search_small_kernel(SmallArgs a, int use_
 }
 
 namespace {
+// A few epochs (cfg1: one scheduling decision, 81 mappings): one WARP per epoch instead of
+// one thread, so the D^Q mappings are scored 32 at a time (lane l: l, l + 32, ...) and the
+// decision's latency is a few dependent steps plus five shuffles, not a serial loop of 81.
+// Lexicographic (makespan, index) through the packed key ms << 7 | m (D^Q <= 81 < 128;
+// ms < 2^51 for Q <= 4 entries below 2^48 each).
+template <int Q, int D>
+__global__ void __launch_bounds__(32) search_tiny_kernel(SmallArgs a) {
+  constexpr int QD = Q * D;
+  constexpr int N = Pow<Q, D>::N;
+  static_assert(N <= 128 && Q <= 4, "packed key: 7 index bits, ms < 2^51");
+  const uint64_t e = blockIdx.x;
+  const int lane = threadIdx.x;
+  __shared__ uint64_t C[QD];
+  bool bad = false;
+  if (lane < QD) {
+    const uint64_t k = a.K[e * QD + lane], x = a.X[e * QD + lane];
+    bad = (k >= kEntryLimit) | (x >= kEntryLimit);
+    C[lane] = k + x;  // a1: aggregate cost
+  }
+  __syncwarp();
+  if (__any_sync(0xffffffffu, bad)) {
+    if (lane == 0) raise_flag(a.flags, kFlagRange);
+    return;
+  }
+  uint64_t key = ~0ull;
+  for (int m = lane; m < N; m += 32) {  // increasing m: the first strict minimum is kept
+    uint64_t L[D];
+#pragma unroll
+    for (int d = 0; d < D; ++d) L[d] = 0;
+    int rest = m;
+#pragma unroll
+    for (int q = Q - 1; q >= 0; --q) {
+      const int dq = rest % D;
+      rest /= D;
+#pragma unroll
+      for (int d = 0; d < D; ++d) L[d] += (dq == d) ? C[q * D + d] : 0;
+    }
+    uint64_t ms = L[0];
+#pragma unroll
+    for (int d = 1; d < D; ++d) ms = max(ms, L[d]);
+    key = min(key, (ms << 7) | (uint64_t)m);
+  }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) key = min(key, __shfl_xor_sync(0xffffffffu, key, off));
+  const uint32_t idx = (uint32_t)(key & 127);
+  if (lane == 0) {
+    a.index[e] = idx;
+    a.makespan[e] = key >> 7;
+  }
+  if (a.mapping && lane < Q) {  // digits of the index, queue 0 most significant
+    uint32_t rest = idx;
+    for (int q = Q - 1; q > lane; --q) rest /= D;
+    a.mapping[e * Q + lane] = (uint8_t)(rest % D);
+  }
+}
+
+constexpr uint64_t kTinyMaxEpochs = 64;  // up to this many epochs: a warp per epoch
+
 template <int Q, int D>
 cudaError_t launch_small_t(const SmallArgs& a, int num_sms, cudaStream_t st, int* grid_out,
                            int* threads_out) {
+  if (a.E <= kTinyMaxEpochs) {
+    search_tiny_kernel<Q, D><<<(unsigned)a.E, 32, 0, st>>>(a);
+    *grid_out = (int)a.E;
+    *threads_out = 32;
+    return cudaGetLastError();
+  }
   // tile = one epoch per thread; tiny batches (cfg1: one epoch) get a single warp.
   // Defaults from the cfg3 sweep (scripts/sweep_small.sh, profiles/r01/sweep_small.txt):
   // 128-epoch tiles, 2 stages, 4 CTAs per SM (8 tiles in flight per SM) was fastest;

@@ -345,3 +345,24 @@ def test_probe(torch_cuda):
     for op in range(5):
         rate, per_clk, mhz = mcl.mcl_probe_int_rate(0, op)
         assert rate > 1e12 and 30 < per_clk < 140 and 500 < mhz < 2500
+
+
+@pytest.mark.parametrize("Q,D", [(2, 2), (2, 3), (2, 4), (3, 2), (3, 3), (3, 4), (4, 2), (4, 3)])
+def test_small_shapes_tiny_and_tiled(torch_cuda, mapper, Q, D):
+    """The small shapes at both sides of the warp-per-epoch cut-over (<= 64 epochs: one warp
+    per epoch; more: the thread-per-epoch TMA kernel), with random and tie-heavy tables and
+    entries near 2^48 (the packed key's makespan field)."""
+    for E in (1, 31, 64, 65):
+        for seed, maker in ((E + 10 * Q + D, workloads.random_tables), (E + 500 + 10 * Q + D, workloads.small_int_tables)):
+            K, X = maker(seed, E, Q, D)
+            got_i, got_mp, got_ms = mapper.map_queues(to_dev(torch_cuda, K), to_dev(torch_cuda, X))
+            assert mapper.launch_info()["path"] == "small_batched"
+            wi, wms, wmp = oracle.oracle_map(K, X)
+            ctx = f"Q={Q} D={D} E={E} {maker.__name__}"
+            assert (got_i.cpu().numpy() == wi).all() and (got_ms.cpu().numpy() == wms).all(), ctx
+            assert (got_mp.cpu().numpy() == wmp).all(), ctx
+    K = np.full((3, Q, D), (1 << 48) - 1, np.uint64)
+    X = np.zeros_like(K)
+    got_i, _, got_ms = mapper.map_queues(to_dev(torch_cuda, K), to_dev(torch_cuda, X))
+    wi, wms, _ = oracle.oracle_map(K, X)
+    assert (got_i.cpu().numpy() == wi).all() and (got_ms.cpu().numpy() == wms).all()
