@@ -152,8 +152,12 @@ struct mcl_mapper {
   int force_path = 0;
   int pipeline_chunks = 0;      // 0 auto, 1 off, n forced (mcl_set_pipeline_chunks)
   bool async_call = false;      // pipelined chunk: enqueue only (the wrapper syncs, reads flags)
-  cudaStream_t pipe[3] = {nullptr, nullptr, nullptr};  // pipelined staging streams
-  cudaEvent_t pipe_ev[4] = {nullptr, nullptr, nullptr, nullptr};  // start + per-stream join
+  // pipelined staging: pipe[0] host->device copies, pipe[1] the searches (one stream, so
+  // chunk kernels never run concurrently and share the handle's scratch safely), pipe[2]
+  // device->host copies; pipe_ev = start + per-stream join, chunk_ev = per-chunk hand-offs
+  cudaStream_t pipe[3] = {nullptr, nullptr, nullptr};
+  cudaEvent_t pipe_ev[4] = {nullptr, nullptr, nullptr, nullptr};
+  std::vector<cudaEvent_t> chunk_ev;
   cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
   int64_t info[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   std::string last_err;
@@ -350,6 +354,7 @@ void mcl_mapper_destroy(mcl_mapper_t* h) {
       if (ps) cudaStreamSynchronize(ps), cudaStreamDestroy(ps);
     for (cudaEvent_t& pe : h->pipe_ev)
       if (pe) cudaEventDestroy(pe);
+    for (cudaEvent_t& ce : h->chunk_ev) cudaEventDestroy(ce);
     if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
   }
   delete h;
@@ -568,12 +573,14 @@ uint64_t chunk_edge(uint64_t epochs, uint64_t nc, uint64_t c) {
   return (uint64_t)(((__uint128_t)epochs * twice) / (2 * (nc - 1)));
 }
 
-// Pipelined staging: chunk c's H2D copies, search and D2H copies go to stream pipe[c % 3]
-// (after the handle's stream, which joins them at the end), so the copies of one chunk
-// overlap the search of another. Each chunk is an ordinary call on device pointers into the
-// staging buffers, enqueued without a sync (async_call); the flags of all chunks are read
-// once at the end. *plain = true: some epoch's bound needs 64-bit loads (every chunk ran
-// the 32-bit kernels), so the caller reruns the whole call unpipelined.
+// Pipelined staging: chunk c's host->device copies go to pipe[0], its search to pipe[1]
+// (after the copy, through an event) and its device->host copies to pipe[2] (after the
+// search), so the copies of one chunk overlap the search of another while the searches run
+// one after another (they share the handle's scratch: split-epoch slots and done counters).
+// The handle's stream is joined at the end. Each search is an ordinary call on device
+// pointers into the staging buffers, enqueued without a sync (async_call); the flags of all
+// chunks are read once at the end. *plain = true: some epoch's bound needs 64-bit loads
+// (every chunk ran the 32-bit kernels), so the caller reruns the whole call unpipelined.
 mcl_status_t map_pipelined(mcl_mapper* h, uint32_t Q, uint32_t D, uint64_t epochs, uint64_t nc,
                            const uint64_t* Kh, const uint64_t* Xh, uint64_t* idx_h, uint8_t* map_h,
                            uint64_t* ms_h, bool* plain) {
@@ -588,18 +595,22 @@ mcl_status_t map_pipelined(mcl_mapper* h, uint32_t Q, uint32_t D, uint64_t epoch
     if (!ps) MCL_CUDA(h, cudaStreamCreateWithFlags(&ps, cudaStreamNonBlocking), "cudaStreamCreate(pipe)");
   for (cudaEvent_t& pe : h->pipe_ev)
     if (!pe) MCL_CUDA(h, cudaEventCreateWithFlags(&pe, cudaEventDisableTiming), "cudaEventCreate(pipe)");
+  while (h->chunk_ev.size() < 2 * nc) {
+    cudaEvent_t ce;
+    MCL_CUDA(h, cudaEventCreateWithFlags(&ce, cudaEventDisableTiming), "cudaEventCreate(chunk)");
+    h->chunk_ev.push_back(ce);
+  }
   uint64_t* Kd = (uint64_t*)h->in_k.p;
   uint64_t* Xd = (uint64_t*)h->in_x.p;
   uint64_t* Id = (uint64_t*)h->out_idx.p;
   uint64_t* Md = (uint64_t*)h->out_ms.p;
   uint8_t* Pd = map_h ? (uint8_t*)h->out_map.p : nullptr;
-  const cudaStream_t s0 = h->stream;
+  const cudaStream_t s0 = h->stream, sin = h->pipe[0], sk = h->pipe[1], sout = h->pipe[2];
   const int timing = h->timing;
-  const int nstreams = (int)std::min<uint64_t>(nc, 3);
   clear_flags(h);
   if (timing >= 2) MCL_CUDA(h, cudaEventRecord(h->ev[2], s0), "cudaEventRecord");
   MCL_CUDA(h, cudaEventRecord(h->pipe_ev[0], s0), "cudaEventRecord(pipe)");
-  for (int i = 0; i < nstreams; ++i)
+  for (int i = 0; i < 3; ++i)
     MCL_CUDA(h, cudaStreamWaitEvent(h->pipe[i], h->pipe_ev[0], 0), "cudaStreamWaitEvent(pipe)");
   mcl_status_t st = MCL_OK;
   int64_t launches = 0;
@@ -608,16 +619,18 @@ mcl_status_t map_pipelined(mcl_mapper* h, uint32_t Q, uint32_t D, uint64_t epoch
   for (uint64_t c = 0; c < nc && st == MCL_OK; ++c) {
     const uint64_t lo = chunk_edge(epochs, nc, c), hi = chunk_edge(epochs, nc, c + 1), ec = hi - lo;
     if (ec == 0) continue;
-    const cudaStream_t ps = h->pipe[c % 3];
-    cudaError_t e = cudaMemcpyAsync(Kd + lo * row, Kh + lo * row, ec * row * 8, cudaMemcpyHostToDevice, ps);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(Xd + lo * row, Xh + lo * row, ec * row * 8, cudaMemcpyHostToDevice, ps);
-    if (e == cudaSuccess && timing && !started) e = cudaEventRecord(h->ev[0], ps);
+    cudaEvent_t in_done = h->chunk_ev[2 * c], k_done = h->chunk_ev[2 * c + 1];
+    cudaError_t e = cudaMemcpyAsync(Kd + lo * row, Kh + lo * row, ec * row * 8, cudaMemcpyHostToDevice, sin);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(Xd + lo * row, Xh + lo * row, ec * row * 8, cudaMemcpyHostToDevice, sin);
+    if (e == cudaSuccess) e = cudaEventRecord(in_done, sin);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(sk, in_done, 0);
+    if (e == cudaSuccess && timing && !started) e = cudaEventRecord(h->ev[0], sk);
     started = true;
     if (e != cudaSuccess) {
       st = cuda_fail(h, e, "pipelined H2D");
       break;
     }
-    h->stream = ps;
+    h->stream = sk;
     h->async_call = true;
     st = map_impl(h, Q, D, ec, Kd + lo * row, Xd + lo * row, nullptr, nullptr, Id + lo,
                   Pd ? Pd + lo * Q : nullptr, Md + lo);
@@ -625,15 +638,17 @@ mcl_status_t map_pipelined(mcl_mapper* h, uint32_t Q, uint32_t D, uint64_t epoch
     h->stream = s0;
     if (st != MCL_OK) break;
     launches += h->info[1];
-    if (timing && c == nc - 1) e = cudaEventRecord(h->ev[1], ps);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(idx_h + lo, Id + lo, ec * 8, cudaMemcpyDeviceToHost, ps);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(ms_h + lo, Md + lo, ec * 8, cudaMemcpyDeviceToHost, ps);
-    if (e == cudaSuccess && map_h) e = cudaMemcpyAsync(map_h + lo * Q, Pd + lo * Q, ec * Q, cudaMemcpyDeviceToHost, ps);
+    if (timing && c == nc - 1) e = cudaEventRecord(h->ev[1], sk);
+    if (e == cudaSuccess) e = cudaEventRecord(k_done, sk);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(sout, k_done, 0);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(idx_h + lo, Id + lo, ec * 8, cudaMemcpyDeviceToHost, sout);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(ms_h + lo, Md + lo, ec * 8, cudaMemcpyDeviceToHost, sout);
+    if (e == cudaSuccess && map_h) e = cudaMemcpyAsync(map_h + lo * Q, Pd + lo * Q, ec * Q, cudaMemcpyDeviceToHost, sout);
     if (e != cudaSuccess) st = cuda_fail(h, e, "pipelined D2H");
   }
   h->timing = timing;
   // join the pipe streams into the handle's stream, then wait for everything
-  for (int i = 0; i < nstreams; ++i) {
+  for (int i = 0; i < 3; ++i) {
     cudaEventRecord(h->pipe_ev[1 + i], h->pipe[i]);
     cudaStreamWaitEvent(s0, h->pipe_ev[1 + i], 0);
   }

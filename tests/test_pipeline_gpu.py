@@ -158,3 +158,21 @@ def test_pipelined_on_external_stream_with_timing(torch_cuda):
                 idx, mp, ms = m.map_queues(Kd, Xd)
                 stream.synchronize()
             assert (idx.cpu().numpy() == want[0]).all() and (ms.cpu().numpy() == want[1]).all()
+
+
+@pytest.mark.parametrize("path", [1, 3])
+def test_pipelined_chunks_share_scratch(torch_cuda, mapper, path):
+    """Chunk searches that use the handle's scratch (split-epoch slots and done counters of
+    the CTA-per-epoch and generic kernels) must not overlap: many small chunks, forced
+    kernel path, every epoch exact."""
+    K, X = workloads.cfg2(E=1500, seed=37) if path == 1 else workloads.random_tables(38, 400, 6, 3)
+    want = oracle.oracle_map(K, X)
+    mapper.set_pipeline_chunks(9)
+    mapper.force_path(path)
+    try:
+        for rep in range(3):
+            got = host_call(torch_cuda, mapper, K, X)
+            check(got, want, f"path {path} rep {rep}")
+    finally:
+        mapper.force_path(0)
+        mapper.set_pipeline_chunks(0)
