@@ -17,3 +17,8 @@ run memcheck cfg4 1
 run memcheck cfg2 1 2400
 run racecheck cfg2 1 2400
 run synccheck cfg2 1 2400
+# pipelined staging of host-resident batches (copies / searches / copies on three streams)
+timeout 900 $CS --tool memcheck --error-exitcode 9 python -m pytest tests/test_pipeline_gpu.py -m gpu -q -p no:cacheprovider > gpurun_out/sanitize_memcheck_pipeline.log 2>&1
+echo "memcheck pipeline rc=$? $(grep -E 'ERROR SUMMARY' gpurun_out/sanitize_memcheck_pipeline.log | tail -1) $(grep -E 'passed|failed' gpurun_out/sanitize_memcheck_pipeline.log | tail -1)"
+timeout 900 $CS --tool racecheck --error-exitcode 9 python -m pytest tests/test_pipeline_gpu.py -m gpu -q -p no:cacheprovider -k "share_scratch or chunks_cfg2" > gpurun_out/sanitize_racecheck_pipeline.log 2>&1
+echo "racecheck pipeline rc=$? $(grep -E 'RACECHECK SUMMARY' gpurun_out/sanitize_racecheck_pipeline.log | tail -1) $(grep -E 'passed|failed' gpurun_out/sanitize_racecheck_pipeline.log | tail -1)"
