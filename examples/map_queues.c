@@ -1,0 +1,61 @@
+/* map_queues.c -- the C ABI used from plain C (no Python, no torch): one scheduling
+ * decision of 4 queues on {CPU, GPU0, GPU1} with host buffers, plus a batch of epochs.
+ *
+ * Epoch 0 is DESIGN.md Appendix A case E ("EP-like": every queue 2000 ns on the CPU and
+ * 100 ns on either GPU; EP goes to the GPUs): optimum (1, 1, 2, 2),
+ * index 44, makespan 200. Epoch 1 is case F ("BT-like", [100, 350, 350] per queue; mostly
+ * CPU, L1800-1807): (0, 0, 0, 1), index 1, makespan 350.
+ *
+ *   gcc -O2 -I include examples/map_queues.c -L paper_conf_cluster_ajipbf15_b200 -lmcl \
+ *       -Wl,-rpath,$PWD/paper_conf_cluster_ajipbf15_b200 -o /tmp/map_queues
+ */
+#include <stdint.h>
+#include <stdio.h>
+#include <string.h>
+
+#include "mcl.h"
+
+int main(void) {
+  enum { E = 2, Q = 4, D = 3 };
+  uint64_t K[E][Q][D], X[E][Q][D];
+  memset(X, 0, sizeof X);
+  for (int q = 0; q < Q; ++q) {
+    K[0][q][0] = 2000; K[0][q][1] = 100; K[0][q][2] = 100;
+    K[1][q][0] = 100;  K[1][q][1] = 350; K[1][q][2] = 350;
+  }
+  mcl_config_t cfg;
+  memset(&cfg, 0, sizeof cfg);
+  cfg.device = 0;
+  cfg.world = 1;
+  mcl_mapper_t* h = NULL;
+  mcl_status_t st = mcl_mapper_create(&cfg, &h);
+  if (st != MCL_OK) {
+    fprintf(stderr, "mcl_mapper_create: %s (%s)\n", mcl_status_string(st), mcl_last_error_string(NULL));
+    return 1;
+  }
+  uint64_t index[E], makespan[E];
+  uint8_t mapping[E][Q];
+  st = mcl_map_queues(h, Q, D, E, &K[0][0][0], &X[0][0][0], index, &mapping[0][0], makespan);
+  if (st != MCL_OK) {
+    fprintf(stderr, "mcl_map_queues: %s (%s)\n", mcl_status_string(st), mcl_last_error_string(h));
+    mcl_mapper_destroy(h);
+    return 1;
+  }
+  const uint64_t want_index[E] = {44, 1}, want_ms[E] = {200, 350};
+  int ok = 1;
+  for (int e = 0; e < E; ++e) {
+    printf("epoch %d: index %llu makespan %llu mapping", e, (unsigned long long)index[e],
+           (unsigned long long)makespan[e]);
+    for (int q = 0; q < Q; ++q) printf(" %u", mapping[e][q]);
+    printf("\n");
+    ok &= index[e] == want_index[e] && makespan[e] == want_ms[e];
+  }
+  /* an entry >= 2^48 is a range error, reported, not silently wrapped */
+  K[1][2][1] = (uint64_t)1 << 48;
+  st = mcl_map_queues(h, Q, D, E, &K[0][0][0], &X[0][0][0], index, NULL, makespan);
+  printf("entry 2^48: %s\n", mcl_status_string(st));
+  ok &= st == MCL_E_RANGE;
+  mcl_mapper_destroy(h);
+  printf("%s\n", ok ? "OK" : "MISMATCH");
+  return ok ? 0 : 2;
+}
