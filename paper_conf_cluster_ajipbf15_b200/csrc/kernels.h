@@ -113,13 +113,14 @@ inline int index_bits_host(uint64_t N) {
 }
 
 bool blocked_supported(uint32_t Q, uint32_t D);
-int blocked_ctas_per_sm(uint32_t D, bool wide, int threads, size_t smem);
+// lean: the one-CTA-per-SM register budget where one exists (u32, D = 5; single epochs)
+int blocked_ctas_per_sm(uint32_t D, bool wide, int threads, size_t smem, bool lean = false);
 size_t blocked_smem_bytes(uint32_t Q, uint32_t D, bool wide, int threads, size_t* off_red,
                           size_t* off_dig);
 // one-thread kernel spinning for `ns` nanoseconds of %globaltimer (timing aid, probe.cu)
 cudaError_t launch_hold(uint64_t ns, cudaStream_t st);
 cudaError_t launch_blocked(const BlockedArgs& a, bool wide, dim3 grid, int threads, size_t smem,
-                           cudaStream_t st);
+                           cudaStream_t st, bool lean = false);
 
 // Batched epochs over a flattened (epoch, block) space (search_flat.cu): u32 loads, whole
 // index space per epoch (no sharding), packed keys (index bits <= 32).

@@ -831,7 +831,8 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
       a.out = out; a.ibits = ibits; a.flags = h->flags_dev; a.one = 1;
       a.base = Bd; a.elig = Ed; a.peer = peer;
       const size_t smem = mcl::blocked_smem_bytes(Q, D, wide, threads, &a.off_red, &a.off_dig);
-      const int occ = mcl::blocked_ctas_per_sm(D, wide, threads, smem);
+      const bool lean = epochs == 1;  // single epochs: the spill-free one-CTA D = 5 build
+      const int occ = mcl::blocked_ctas_per_sm(D, wide, threads, smem, lean);
       // Work layout (1-D grid): whole waves of epochs get one CTA each; the epochs of the
       // last, partial wave are split over several CTAs so that wave is filled; a batch
       // smaller than one wave spreads every epoch over the resident CTAs.
@@ -860,7 +861,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
         a.scratch = (Cand*)h->scratch.p;
       }
       a.done = (uint32_t*)h->done.p;
-      MCL_CUDA(h, mcl::launch_blocked(a, wide, grid, threads, smem, s), "search_blocked launch");
+      MCL_CUDA(h, mcl::launch_blocked(a, wide, grid, threads, smem, s, lean), "search_blocked launch");
     } else {
       const uint64_t rows = N / D;
       uint64_t lo, hi;

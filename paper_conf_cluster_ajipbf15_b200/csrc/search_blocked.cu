@@ -33,8 +33,11 @@ namespace mcl {
 // remaining E - e_full epochs (the "tail") get tail_cpe CTAs each, so the last wave of a
 // batch runs split epochs instead of idling (wave quantisation), and a single large epoch
 // (e_full = 0) spreads over every CTA. The grid strides over this CTA index space.
-template <typename T, int D>
-__global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
+// kLean: the register budget of one CTA per SM for the u32 D = 5 kernel, whose two-CTA
+// build spills (56 bytes of stack); chosen for single-epoch searches (measured: 12 x 5 one
+// epoch 63 -> 50 us), while batched calls keep two CTAs per SM for their grid shapes.
+template <typename T, int D, bool kLean = false>
+__global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5 && !kLean) ? 2 : 1)
     search_blocked_kernel(BlockedArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const uint32_t Q = a.Q;
@@ -214,10 +217,10 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1)
   if (a.peer.world) peer_finish(a.peer, a.out, a.E, Q, D, a.ibits, a.flags, abandoned);
 }
 
-template <typename T, int D>
+template <typename T, int D, bool L = false>
 static cudaError_t launch_blocked_t(const BlockedArgs& a, dim3 grid, int threads, size_t smem,
                                    cudaStream_t st) {
-  auto k = search_blocked_kernel<T, D>;
+  auto k = search_blocked_kernel<T, D, L>;
   static SmemAttrCache cache;
   cudaError_t err = ensure_smem(k, smem, cache);
   if (err != cudaSuccess) return err;
@@ -239,7 +242,7 @@ size_t blocked_smem_bytes(uint32_t Q, uint32_t D, bool wide, int threads, size_t
 }
 
 namespace {
-template <typename T, int D>
+template <typename T, int D, bool L = false>
 int occ_t(int threads, size_t smem) {
   // cache the last (threads, smem) query: the launch path asks the same question every call
   static std::atomic<uint64_t> last{0};
@@ -247,7 +250,7 @@ int occ_t(int threads, size_t smem) {
   const uint64_t hit = last.load(std::memory_order_relaxed);
   if (hit && (hit & ~0xffull) == key) return (int)(hit & 0xff);
   int n = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, search_blocked_kernel<T, D>, threads, smem) !=
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, search_blocked_kernel<T, D, L>, threads, smem) !=
       cudaSuccess)
     return 1;
   n = n < 1 ? 1 : (n > 255 ? 255 : n);
@@ -256,7 +259,10 @@ int occ_t(int threads, size_t smem) {
 }
 }  // namespace
 
-int blocked_ctas_per_sm(uint32_t D, bool wide, int threads, size_t smem) {
+int blocked_ctas_per_sm(uint32_t D, bool wide, int threads, size_t smem, bool lean) {
+#ifndef MCL_ONLY_D
+  if (lean && !wide && D == 5) return occ_t<uint32_t, 5, true>(threads, smem);
+#endif
 #ifdef MCL_ONLY_D
   if (D != MCL_ONLY_D) return 1;
   return wide ? occ_t<uint64_t, MCL_ONLY_D>(threads, smem) : occ_t<uint32_t, MCL_ONLY_D>(threads, smem);
@@ -277,7 +283,10 @@ int blocked_ctas_per_sm(uint32_t D, bool wide, int threads, size_t smem) {
 bool blocked_supported(uint32_t Q, uint32_t D) { return Q >= 3 && D >= 2 && D <= kBlockedMaxD; }
 
 cudaError_t launch_blocked(const BlockedArgs& a, bool wide, dim3 grid, int threads, size_t smem,
-                           cudaStream_t st) {
+                           cudaStream_t st, bool lean) {
+#ifndef MCL_ONLY_D
+  if (lean && !wide && a.D == 5) return launch_blocked_t<uint32_t, 5, true>(a, grid, threads, smem, st);
+#endif
 #ifdef MCL_ONLY_D
 #define MCL_CASE(DD)                                                                  \
   case DD:                                                                            \

@@ -366,3 +366,22 @@ def test_small_shapes_tiny_and_tiled(torch_cuda, mapper, Q, D):
     got_i, _, got_ms = mapper.map_queues(to_dev(torch_cuda, K), to_dev(torch_cuda, X))
     wi, wms, _ = oracle.oracle_map(K, X)
     assert (got_i.cpu().numpy() == wi).all() and (got_ms.cpu().numpy() == wms).all()
+
+
+def test_d5_single_epoch_lean_build(torch_cuda, mapper):
+    """Single epochs with D = 5 run the one-CTA-per-SM (spill-free) build of the blocked
+    kernel: whole index spaces and sharded sub-ranges equal the oracle."""
+    for Q in (6, 8, 9):
+        K, X = workloads.random_tables(700 + Q, 1, Q, 5)
+        want = oracle.oracle_map(K, X)
+        i, mp, ms = mapper.map_queues(to_dev(torch_cuda, K), to_dev(torch_cuda, X))
+        assert mapper.launch_info()["path"] == "blocked_u32"
+        assert int(i[0]) == want[0][0] and int(ms[0]) == want[1][0] and (mp.cpu().numpy() == want[2]).all()
+        N, unit = 5**Q, 125
+        for r in range(3):
+            with Mapper(0, rank=r, world=3) as m:
+                si, _, sms = m.map_queues(to_dev(torch_cuda, K), to_dev(torch_cuda, X))
+            nb = N // unit
+            lo, hi = (nb * r // 3) * unit, (nb * (r + 1) // 3) * unit
+            oi, oms, _ = oracle.oracle_map(K, X, lo=lo, hi=hi)
+            assert (int(si[0]), int(sms[0])) == (int(oi[0]), int(oms[0])), f"Q={Q} shard {r}"
