@@ -48,7 +48,7 @@ KERNEL_TIMING = ("CUDA events on the mapper's stream around the search launch, i
                  "by a 200 us spin kernel so the events measure device execution; the timed steps record "
                  "no library events (one timing-event record costs ~2.7 us of host time, "
                  "scripts/host_api_costs.cu, which the step would be charged)")
-KERNEL_NAMES = {"blocked_u32": "search_blocked_kernel<u32, D>", "blocked_u64": "search_blocked_kernel<u64, D>",
+KERNEL_NAMES = {"blocked_u32": "search_blocked_kernel<u32, D>", "blocked_u32_lean": "search_blocked_kernel<u32, 5, lean>", "blocked_u64": "search_blocked_kernel<u64, D>",
                 "generic": "search_generic_kernel", "flat_u32": "search_flat_kernel<u32, D>",
                 "small_batched": "search_small_kernel<Q, D>", "batch_u32": "search_batch_kernel<Q, D>"}
 
@@ -400,7 +400,7 @@ def main():
         max_mhz = clocks.get("sm_max_mhz") or 1965
         # per GPU and launch: the full batch (batched replicas) or this rank's index shard
         mappings_per_launch = w["E"] * w["N"] if is_batched(w) else w["N"] / world
-        if info["path"] in ("blocked_u32", "blocked_u64", "generic", "flat_u32", "batch_u32"):
+        if info["path"] in ("blocked_u32", "blocked_u32_lean", "blocked_u64", "generic", "flat_u32", "batch_u32"):
             achieved = ALU_INSTR_PER_MAPPING * mappings_per_launch / (kern_mean / 1e3) / 1e12
             peak = ALU_LANES_PER_CLK_SM * sms * max_mhz * 1e6 / 1e12
             roof = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tops/s",

@@ -47,7 +47,9 @@ typedef enum {
 
 typedef struct {
   int device;      /* CUDA device ordinal this handle runs on                            */
-  void* stream;    /* cudaStream_t to run on; NULL = a non-blocking stream owned by the handle */
+  void* stream;    /* cudaStream_t to run on (cudaStreamLegacy = (void*)1 and cudaStreamPerThread
+                      = (void*)2 are accepted); NULL = a non-blocking stream owned by the handle,
+                      which is not ordered after work on any other stream                  */
   void* nccl_comm; /* ncclComm_t (e.g. torch ProcessGroupNCCL._comm_ptr()) or NULL        */
   int rank;        /* this process's shard, 0 <= rank < world                             */
   int world;       /* number of shards; 0 or 1 = the whole index space                    */
@@ -80,8 +82,14 @@ mcl_status_t mcl_mapper_create(const mcl_config_t* cfg, mcl_mapper_t** out);
  *   makespan      : [E] uint64 out: its makespan, in the same unit as the costs.
  * Every pointer may be device memory (the fast path: no copies) or host memory (pageable
  * or pinned; detected with cudaPointerGetAttributes and staged through handle-owned device
- * buffers inside the call). The caller owns all buffers; the library never frees them.
+ * buffers inside the call). A pointer the CUDA runtime cannot classify is MCL_E_INVAL;
+ * pageable host pointers cannot be validated and are trusted, as with any C library taking
+ * host buffers. The caller owns all buffers; the library never frees them.
  * Inputs are only read; outputs are fully written on MCL_OK and unspecified on error.
+ * Stream order: device inputs must be complete, and device outputs free to overwrite, in
+ * the order of the handle's stream (cfg->stream). Pass the stream that produced the inputs
+ * (cudaStreamLegacy = (void*)1 for the legacy default stream); with cfg->stream == NULL the
+ * handle's own non-blocking stream does NOT wait for work on other streams.
  *
  * Sharding: the index space [0, D^Q) of each epoch is cut into `world` contiguous ranges
  * [floor(r*N/G), floor((r+1)*N/G)) (in whole blocks of the innermost digits). With a
@@ -117,9 +125,11 @@ mcl_status_t mcl_map_queues(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t ep
  * Afterwards every mcl_map_queues / mcl_map_queues_constrained call on h with
  * epochs <= max_epochs is COLLECTIVE through the slabs: all ranks must make the same calls,
  * in the same order, with identical inputs. A communicator, if the handle has one, still
- * serves larger calls. If some rank does not signal within timeout_ms (0 = 30 s), the call
- * fails with MCL_E_NCCL ("peer exchange timed out") instead of hanging, and the handle's
- * exchange is disabled. Destroy the handles of all ranks together (a rank's slab stays
+ * serves larger calls; without one (world > 1), a larger call fails with MCL_E_INVAL
+ * instead of returning a shard-local result. If some rank does not signal within
+ * timeout_ms (0 = 30 s), the call fails with MCL_E_NCCL ("peer exchange timed out")
+ * instead of hanging, and the handle's exchange is disabled: later calls go to the
+ * communicator, or (without one) fail with MCL_E_NCCL until a new export / import. Destroy the handles of all ranks together (a rank's slab stays
  * mapped by its peers until they destroy theirs).
  * Errors: MCL_E_INVAL (bad arguments, world handles not matching, import before export),
  *         MCL_E_CUDA (IPC export/open failed, e.g. no peer access between the devices).
@@ -250,7 +260,9 @@ const char* mcl_last_error_string(const mcl_mapper_t* h);
  * mcl_last_launch_info fills, for the most recent successful mcl_map_queues call on h:
  *   info[0] = kernel path id (1 = register-blocked u32 search, 2 = register-blocked u64
  *             search, 3 = generic search, 4 = small batched (thread per epoch),
- *             5 = register-blocked u32 over a flattened (epoch, block) space)
+ *             5 = register-blocked u32 over a flattened (epoch, block) space,
+ *             6 = branch and bound (mcl_map_queues_pruned), 7 = warp-per-epoch batched u32,
+ *             8 = register-blocked u32, one-CTA-per-SM build (single epochs, D = 5))
  *   info[1] = number of kernels launched by the call, info[2] = CTAs of the main kernel,
  *   info[3] = threads per CTA, info[4] = 1 if an NCCL all-reduce ran, 2 if the fused peer
  *   exchange ran, info[5] = index bits of the packed key, info[6] = 1 if the two-step

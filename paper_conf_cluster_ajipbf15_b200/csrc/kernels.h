@@ -13,7 +13,7 @@ namespace mcl {
 // them into an mcl_status_t after the stream sync.
 enum : uint32_t {
   kFlagRange = 1u,       // some cost entry or base load >= 2^48
-  kFlagNeedU64 = 2u,     // some epoch's bound sum_q max_d C >= 2^32: rerun with 64-bit loads
+  kFlagNeedU64 = 2u,     // some epoch's bound sum_q max_d C >= 2^32 - 1: rerun with 64-bit loads
   kFlagNoPack = 4u,      // makespan does not fit beside the index in one u64 key (NCCL path)
   kFlagInfeasible = 8u,  // constrained call: some queue has no eligible device below D
   kFlagBadMapping = 16u, // scoring call: a mapping names a device >= D
@@ -113,6 +113,8 @@ inline int index_bits_host(uint64_t N) {
 }
 
 bool blocked_supported(uint32_t Q, uint32_t D);
+// whether launch_blocked(..., lean = true) runs a separate one-CTA-per-SM build for (D, wide)
+bool blocked_lean_built(uint32_t D, bool wide);
 // lean: the one-CTA-per-SM register budget where one exists (u32, D = 5; single epochs)
 int blocked_ctas_per_sm(uint32_t D, bool wide, int threads, size_t smem, bool lean = false);
 size_t blocked_smem_bytes(uint32_t Q, uint32_t D, bool wide, int threads, size_t* off_red,

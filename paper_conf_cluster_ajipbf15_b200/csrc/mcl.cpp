@@ -144,6 +144,7 @@ struct mcl_mapper {
   uint64_t peer_cap = 0;
   uint64_t peer_timeout_ns = 0;
   bool peer_ready = false;
+  bool peer_configured = false;  // slabs were imported (cleared only by a new export)
   uint32_t* flags_host = nullptr;               // host-mapped status word
   uint32_t* flags_dev = nullptr;
   int timing = 0;               // 0 off, 1 search kernel, 2 search kernel + whole call
@@ -186,10 +187,10 @@ mcl_status_t nccl_fail(mcl_mapper* h, ncclResult_t r, const char* what) {
 mcl_status_t classify(mcl_mapper* h, const void* p, bool* on_device) {
   cudaPointerAttributes at;
   cudaError_t e = cudaPointerGetAttributes(&at, p);
-  if (e != cudaSuccess) {  // unregistered host memory on older runtimes
+  if (e != cudaSuccess) {  // CUDA >= 11 reports unregistered host memory as success
     cudaGetLastError();
-    *on_device = false;
-    return MCL_OK;
+    h->last_err = std::string("cannot classify a buffer pointer: ") + cudaGetErrorString(e);
+    return MCL_E_INVAL;
   }
   if (at.type == cudaMemoryTypeDevice) {
     if (at.device != h->device) {
@@ -687,6 +688,18 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
   const bool fused = h->peer_ready && epochs <= h->peer_cap;
   const bool use_nccl = !fused && h->comm != nullptr;
   const bool multi = fused || use_nccl;
+  // A handle whose ranks exchange through peer slabs must never fall back to a sub-range
+  // search silently: without the exchange (a call above max_epochs, or the exchange
+  // disabled by a timeout) and without a communicator, this rank's shard-local argmin is
+  // not the global result.
+  if (h->peer_configured && h->world > 1 && !multi) {
+    if (!h->peer_ready) {
+      h->last_err = "peer exchange disabled by an earlier timeout and no NCCL communicator";
+      return MCL_E_NCCL;
+    }
+    h->last_err = "epochs exceed the peer exchange's max_epochs and the handle has no NCCL communicator";
+    return MCL_E_INVAL;
+  }
 
   // ---- host-resident batch: pipelined staging (chunks of H2D / search / D2H) ----
   if (!multi && !base_load && !eligible && h->pipeline_chunks != 1 && !h->async_call && epochs > 1) {
@@ -779,6 +792,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
     nlaunch = 0;
     dim3 grid(1, 1, 1);
     int threads = 0;
+    bool lean_ran = false;  // the one-CTA-per-SM build of the blocked kernel (reported as path 8)
     if (h->timing) MCL_CUDA(h, record_start(h, s), "cudaEventRecord(start)");
     if (path == 7) {
       mcl::BatchArgs a{Q, D, epochs, K, X, o_idx, o_ms, o_map, h->flags_dev, 1u};
@@ -862,6 +876,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
       }
       a.done = (uint32_t*)h->done.p;
       MCL_CUDA(h, mcl::launch_blocked(a, wide, grid, threads, smem, s, lean), "search_blocked launch");
+      lean_ran = lean && mcl::blocked_lean_built(D, wide);
     } else {
       const uint64_t rows = N / D;
       uint64_t lo, hi;
@@ -885,7 +900,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
     }
     ++nlaunch;
     if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[1], s), "cudaEventRecord");
-    h->info[0] = path;
+    h->info[0] = lean_ran ? 8 : path;
     h->info[2] = (int64_t)grid.x * grid.y;
     h->info[3] = threads;
     h->info[4] = 0;
@@ -986,6 +1001,7 @@ mcl_status_t mcl_peer_export(mcl_mapper_t* h, uint64_t max_epochs, uint8_t handl
   for (void* p : h->peer_opened) cudaIpcCloseMemHandle(p);  // a new slab voids any import
   h->peer_opened.clear();
   h->peer_ready = false;
+  h->peer_configured = false;
   h->peer_slab.release();  // a fresh allocation: the handle names exactly this slab
   const size_t words = mcl::kPeerHeaderWords + 2 * max_epochs;
   MCL_CUDA(h, h->peer_slab.ensure(words * 8), "cudaMalloc(peer slab)");
@@ -1042,6 +1058,7 @@ mcl_status_t mcl_peer_import(mcl_mapper_t* h, const uint8_t* handles, uint32_t t
            "H2D(peer)");
   h->peer_timeout_ns = (uint64_t)(timeout_ms ? timeout_ms : 30000) * 1000000ull;
   h->peer_ready = true;
+  h->peer_configured = true;
   return MCL_OK;
 }
 

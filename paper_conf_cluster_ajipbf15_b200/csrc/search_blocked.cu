@@ -99,7 +99,10 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5 && !kLean) ? 2 
       abandoned = true;
       continue;
     }
-    if (sizeof(T) == 4 && s_ub >= (1ull << 32)) {
+    // 32-bit loads need UB < 2^32 - 1: every makespan then stays below the all-ones
+    // "no candidate" value the running minima start from (UB = 2^32 - 1 takes the 64-bit
+    // rerun; with UB = 2^32 - 1 an optimum equal to it would never pass the strict <)
+    if (sizeof(T) == 4 && s_ub >= 0xffffffffull) {
       if (tid == 0 && part == 0) raise_flag(a.flags, kFlagNeedU64);
       abandoned = true;
       continue;
@@ -281,6 +284,16 @@ int blocked_ctas_per_sm(uint32_t D, bool wide, int threads, size_t smem, bool le
 }
 
 bool blocked_supported(uint32_t Q, uint32_t D) { return Q >= 3 && D >= 2 && D <= kBlockedMaxD; }
+
+bool blocked_lean_built(uint32_t D, bool wide) {
+#ifndef MCL_ONLY_D
+  return !wide && D == 5;
+#else
+  (void)D;
+  (void)wide;
+  return false;  // variant builds for one D compile no lean instantiation
+#endif
+}
 
 cudaError_t launch_blocked(const BlockedArgs& a, bool wide, dim3 grid, int threads, size_t smem,
                            cudaStream_t st, bool lean) {

@@ -76,7 +76,8 @@ __global__ void __launch_bounds__(32, (D <= 5) ? 16 : 8) search_flat_kernel(Flat
     }
 #pragma unroll
     for (int off = 16; off > 0; off >>= 1) part += __shfl_xor_sync(0xffffffffu, part, off);
-    if (sizeof(T) == 4 && part >= (1ull << 32)) {
+    // UB < 2^32 - 1 keeps every makespan below the all-ones start of the running minima
+    if (sizeof(T) == 4 && part >= 0xffffffffull) {
       if (lane == 0) raise_flag(a.flags, kFlagNeedU64);
       continue;
     }

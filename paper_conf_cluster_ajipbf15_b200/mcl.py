@@ -18,7 +18,7 @@ LIB_PATH = os.path.join(_HERE, "libmcl.so")
 
 MCL_OK, MCL_E_INVAL, MCL_E_RANGE, MCL_E_CUDA, MCL_E_NCCL, MCL_E_NOMEM = 0, -1, -2, -3, -4, -5
 PATH_NAMES = {1: "blocked_u32", 2: "blocked_u64", 3: "generic", 4: "small_batched", 5: "flat_u32",
-              6: "pruned", 7: "batch_u32"}
+              6: "pruned", 7: "batch_u32", 8: "blocked_u32_lean"}
 
 # Every symbol the headers declare (tests check the library exports all of them).
 EXPORTED = [
@@ -233,12 +233,46 @@ def _ptr_and_keepalive(x, dtype, convert: bool = False):
     return a.ctypes.data, a
 
 
+CUDA_STREAM_LEGACY = 1  # cudaStreamLegacy: the legacy default stream, as a stream handle
+
+
+def _shape(x) -> tuple:
+    return tuple(int(s) for s in x.shape)
+
+
+def _check(name: str, x, want: tuple) -> None:
+    """Raise ValueError unless ``x`` has exactly shape ``want`` (caught here, before any
+    pointer reaches the library, so a mismatch can never read or write out of bounds)."""
+    if x is not None and _shape(x) != want:
+        raise ValueError(f"{name}: expected shape {want}, got {_shape(x)}")
+
+
+def _default_stream(device: int):
+    """torch's current stream on ``device`` (the legacy default stream as cudaStreamLegacy),
+    so a handle created without an explicit stream is ordered after the torch work that
+    produced its CUDA inputs; None (the handle's own stream) without torch or CUDA."""
+    try:
+        import torch
+
+        if torch.cuda.is_available():
+            return torch.cuda.current_stream(device).cuda_stream or CUDA_STREAM_LEGACY
+    except Exception:  # pragma: no cover
+        pass
+    return None
+
+
 class Mapper:
-    """One mapper handle (see include/mcl.h). Use as a context manager or call close()."""
+    """One mapper handle (see include/mcl.h). Use as a context manager or call close().
+
+    ``stream``: None = torch's current stream on ``device`` at creation (so CUDA tensors
+    produced there are ready when the search runs, include/mcl.h "Stream order"); an
+    integer cudaStream_t otherwise; 0 = a private non-blocking stream of the handle."""
 
     def __init__(self, device: int = 0, stream: int | None = None, nccl_comm: int | None = None,
                  rank: int = 0, world: int = 1):
         self.device = device
+        if stream is None:
+            stream = _default_stream(device)
         self.handle = mcl_mapper_create(device, stream, nccl_comm, rank, world)
 
     def close(self):
@@ -262,7 +296,15 @@ class Mapper:
         """Run the search writing into caller-owned outputs. K, X: [E, Q, D] uint64;
         index, makespan: [E] uint64; mapping: [E, Q] uint8 or None. Tensors may live on the
         handle's CUDA device or on the host."""
+        if K.ndim != 3:
+            raise ValueError(f"K: expected [E, Q, D], got shape {_shape(K)}")
         E, Q, D = K.shape
+        if (X.shape != K.shape or index.shape != (E,) or makespan.shape != (E,)
+                or (mapping is not None and mapping.shape != (E, Q))):
+            _check("X", X, (E, Q, D))
+            _check("index", index, (E,))
+            _check("makespan", makespan, (E,))
+            _check("mapping", mapping, (E, Q))
         tensor_type, dtypes = _TORCH or _torch_types()
         if type(K) is tensor_type and type(X) is tensor_type and type(index) is tensor_type \
                 and type(makespan) is tensor_type and (mapping is None or type(mapping) is tensor_type):
@@ -295,6 +337,8 @@ class Mapper:
         (index[E], mapping[E, Q] or None, makespan[E])."""
         if K.ndim == 2:
             K, X = K[None], X[None]
+        if K.ndim != 3:
+            raise ValueError(f"K: expected [E, Q, D], got shape {_shape(K)}")
         E, Q, D = (int(s) for s in K.shape)
         try:
             import torch
@@ -328,7 +372,19 @@ class Mapper:
             return ptr
 
         nb = model["bytes"]
+        if nb.ndim != 2:
+            raise ValueError(f"bytes: expected [E, Q], got shape {_shape(nb)}")
         E, Q = int(nb.shape[0]), int(nb.shape[1])
+        nk, M = int(model["profile"].shape[0]), int(model["sizes"].shape[0])
+        _check("profile", model["profile"], (nk, D))
+        _check("offsets", model["offsets"], (E * Q + 1,))
+        if model["kernel_ids"].ndim != 1:
+            raise ValueError("kernel_ids: expected a 1-D array")
+        _check("source", model["source"], (E, Q))
+        _check("cached", model.get("cached"), (E, Q))
+        _check("sizes", model["sizes"], (M,))
+        for name in ("h2d_bw", "d2h_bw"):
+            _check(name, model[name], (D, M))
         c = mcl_cost_model_t(
             int(model["profile"].shape[0]), p("profile", np.uint64), p("offsets", np.uint64),
             p("kernel_ids", np.uint32) if int(model["kernel_ids"].shape[0]) else None,
@@ -387,7 +443,12 @@ class Mapper:
             K, X = K[None], X[None]
             base = None if base is None else base[None]
             eligible = None if eligible is None else eligible[None]
+        if K.ndim != 3:
+            raise ValueError(f"K: expected [E, Q, D], got shape {_shape(K)}")
         E, Q, D = (int(s) for s in K.shape)
+        _check("X", X, (E, Q, D))
+        _check("base", base, (E, D))
+        _check("eligible", eligible, (E, Q))
         idx, mp, ms = self._alloc_outputs(K, E, Q, with_mapping)
         pk, _k = _ptr_and_keepalive(K, np.uint64)
         px, _x = _ptr_and_keepalive(X, np.uint64)
@@ -407,7 +468,12 @@ class Mapper:
         if K.ndim == 2:
             K, X, mappings = K[None], X[None], mappings[None]
             base = None if base is None else base[None]
+        if K.ndim != 3:
+            raise ValueError(f"K: expected [E, Q, D], got shape {_shape(K)}")
         E, Q, D = (int(s) for s in K.shape)
+        _check("X", X, (E, Q, D))
+        _check("mappings", mappings, (E, Q))
+        _check("base", base, (E, D))
         ms = self._alloc_outputs(K, E, Q, False)[2]
         pk, _k = _ptr_and_keepalive(K, np.uint64)
         px, _x = _ptr_and_keepalive(X, np.uint64)

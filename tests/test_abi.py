@@ -99,3 +99,40 @@ def test_product_never_imports_oracle():
             text = open(path).read()
             assert not re.search(r"^\s*(from|import)\s+paper_conf", text, flags=re.M), path
             assert "#include" not in text or "mcl" not in "".join(re.findall(r"#include.*", text)), path
+
+
+def test_binding_rejects_mismatched_shapes_before_the_library():
+    """Mapper methods check every array against (E, Q, D) (and M for the cost model) and
+    raise ValueError before any pointer reaches libmcl.so (a mismatch would read
+    or write out of bounds). A handle-less Mapper shows no library call is made."""
+    import numpy as np
+
+    m = object.__new__(mcl.Mapper)
+    m.handle = None
+    m.device = 0
+    K = np.zeros((3, 5, 4), np.uint64)
+    ok_i, ok_ms, ok_mp = np.zeros(3, np.uint64), np.zeros(3, np.uint64), np.zeros((3, 5), np.uint8)
+    bad = [
+        (np.zeros((3, 5, 3), np.uint64), ok_i, ok_mp, ok_ms),  # X
+        (K, np.zeros(2, np.uint64), ok_mp, ok_ms),            # index
+        (K, ok_i, np.zeros((3, 4), np.uint8), ok_ms),         # mapping
+        (K, ok_i, ok_mp, np.zeros(4, np.uint64)),             # makespan
+    ]
+    for X, i, mp, ms in bad:
+        with pytest.raises(ValueError):
+            m.map_queues_into(K, X, i, mp, ms)
+    with pytest.raises(ValueError):
+        m.map_queues_into(K[0], K[0], ok_i, ok_mp, ok_ms)  # not [E, Q, D]
+    with pytest.raises(ValueError):
+        m.map_queues_constrained(K, K, base=np.zeros((3, 5), np.uint64))
+    with pytest.raises(ValueError):
+        m.map_queues_constrained(K, K, eligible=np.zeros((3, 4), np.uint16))
+    with pytest.raises(ValueError):
+        m.score_mappings(K, K, np.zeros((3, 4), np.uint8))
+    from paper_conf_cluster_ajipbf15_b200 import workloads
+
+    model = workloads.cost_model(1, 3, 5, 4)
+    for key, val in (("offsets", model["offsets"][:-1]), ("source", model["source"][:, :4]),
+                     ("h2d_bw", model["h2d_bw"][:, :-1]), ("profile", model["profile"][:, :3])):
+        with pytest.raises(ValueError):
+            m._cost_model(dict(model, **{key: val}), 4)

@@ -232,15 +232,95 @@ def test_u64_fallback_and_max_entries(torch_cuda, mapper):
     assert_same(run_gpu(torch_cuda, mapper, K, np.zeros_like(K)), oracle.oracle_map(K, np.zeros_like(K)), "max")
 
 
+U32_TOP = (1 << 32) - 1  # 0xFFFFFFFF: the all-ones "no candidate" start of the u32 minima
+
+
+def _one_big_queue(E, Q, D, totals, big_q=0):
+    """Epoch e: queue big_q costs totals[e] on every device, every other entry 0, so the
+    bound UB = sum_q max_d C = totals[e] and EVERY mapping's makespan is totals[e]: the
+    optimum equals UB (ms* = UB) and the lowest index 0 wins the all-way tie."""
+    K = np.zeros((E, Q, D), np.uint64)
+    for e, t in enumerate(totals):
+        K[e, big_q, :] = t
+    return K, np.zeros_like(K)
+
+
+def _balanced_at(total, Q=4, D=3):
+    """One epoch whose bound UB = sum_q max_d C equals `total` exactly: queue q costs r_q on
+    device 0 and r_q + 1 on the others, with sum_q (r_q + 1) = total."""
+    K = np.zeros((1, Q, D), np.uint64)
+    base = total // Q - 1
+    r = [base] * Q
+    r[0] += total - Q * (base + 1)
+    for q in range(Q):
+        K[0, q, 0] = r[q]
+        K[0, q, 1:] = r[q] + 1
+    assert sum(int(K[0, q].max()) for q in range(Q)) == total
+    return K, np.zeros_like(K)
+
+
+@pytest.mark.parametrize("Q,D", [(5, 2), (6, 3), (8, 4)])
+def test_u32_top_of_range_optimum_equals_bound(torch_cuda, mapper, Q, D):
+    """ms* = UB = 2^32 - 1: the u32 kernels' running minima start at
+    0xFFFFFFFF with a strict <, so this bound must take the 64-bit kernel (else the call
+    returned index = makespan = UINT64_MAX). UB = 2^32 - 2 is the largest bound the u32
+    kernels keep, and there the optimum equal to UB must still be found by them."""
+    for total, want_path in ((U32_TOP, "blocked_u64"), (U32_TOP - 1, "blocked_u32")):
+        K, X = _one_big_queue(1, Q, D, [total], big_q=1)
+        want = oracle.oracle_map(K, X)
+        assert int(want[1][0]) == total and int(want[0][0]) == 0
+        for p in (0, 1):
+            assert_same(run_gpu(torch_cuda, mapper, K, X, p), want, f"{Q}x{D} UB={total} path {p}")
+            assert mapper.launch_info()["path"] == want_path, (total, p, mapper.launch_info())
+
+
+@pytest.mark.parametrize("Q,D", [(6, 3), (8, 4)])
+def test_u32_top_of_range_batched(torch_cuda, mapper, Q, D):
+    """Three epochs in one call (UB = 2^32 - 1, an ordinary epoch, UB = 2^32 - 2): the whole
+    call reruns on 64-bit loads when any epoch needs it; the flattened and warp-per-epoch
+    batch kernels too."""
+    K, X = _one_big_queue(3, Q, D, [U32_TOP, 0, U32_TOP - 1], big_q=Q - 1)
+    rng = np.random.default_rng(Q * D)
+    K[1] = rng.integers(0, 1 << 20, size=(Q, D), dtype=np.uint64)
+    want = oracle.oracle_map(K, X)
+    assert int(want[1][0]) == U32_TOP and int(want[1][2]) == U32_TOP - 1
+    paths = [0, 1, 2, 3, 5] + ([7] if (Q, D) == (8, 4) else [])
+    for p in paths:
+        assert_same(run_gpu(torch_cuda, mapper, K, X, p), want, f"{Q}x{D} batched path {p}")
+    # without the top epoch, the u32 kernels keep the call (UB = 2^32 - 2 at most)
+    for p, name in ((1, "blocked_u32"), (5, "flat_u32")) + (((7, "batch_u32"),) if (Q, D) == (8, 4) else ()):
+        assert_same(run_gpu(torch_cuda, mapper, K[1:], X[1:], p), tuple(w[1:] for w in want), f"path {p}")
+        assert mapper.launch_info()["path"] == name
+
+
+def test_u32_top_of_range_shards(torch_cuda):
+    """Shard-mode handles (G = 3) at ms* = UB = 2^32 - 1 and 2^32 - 2: every shard's local
+    argmin equals the oracle's on the same index sub-range."""
+    torch = torch_cuda
+    Q, D, G = 6, 3, 3
+    nb = D ** (Q - 3)
+    for total in (U32_TOP, U32_TOP - 1):
+        K, X = _one_big_queue(1, Q, D, [total], big_q=2)
+        Kd, Xd = to_dev(torch, K), to_dev(torch, X)
+        for r in range(G):
+            with Mapper(0, rank=r, world=G) as m:
+                idx, _, ms = m.map_queues(Kd, Xd)
+                path = m.launch_info()["path"]
+            lo, hi = (nb * r // G) * D**3, (nb * (r + 1) // G) * D**3
+            oi, oms, _ = oracle.oracle_map(K, X, lo=lo, hi=hi)
+            assert (int(ms[0].item()), int(idx[0].item())) == (int(oms[0]), int(oi[0])), (total, r)
+            assert path == ("blocked_u64" if total == U32_TOP else "blocked_u32")
+
+
 def test_u32_boundary(torch_cuda, mapper):
-    """Bounds just below and just above 2^32."""
-    for total in ((1 << 32) - 1, 1 << 32):
-        K = np.zeros((1, 4, 3), dtype=np.uint64)
-        K[0, :, 0] = total // 4
-        K[0, 0, 0] += total - 4 * (total // 4)
-        K[0, :, 1:] = total // 4 + 1
-        X = np.zeros_like(K)
-        assert_same(run_gpu(torch_cuda, mapper, K, X, 1), oracle.oracle_map(K, X), str(total))
+    """Bounds UB = 2^32 - 2, 2^32 - 1 and 2^32 exactly (UB = sum_q max_d C, built to the
+    unit), with a non-trivial optimum below UB: the u32 kernel keeps the first, the other two
+    take the 64-bit rerun, and all three match the oracle."""
+    for total, want_path in ((U32_TOP - 1, "blocked_u32"), (U32_TOP, "blocked_u64"), (1 << 32, "blocked_u64")):
+        K, X = _balanced_at(total)
+        want = oracle.oracle_map(K, X)
+        assert_same(run_gpu(torch_cuda, mapper, K, X, 1), want, str(total))
+        assert mapper.launch_info()["path"] == want_path
 
 
 def test_degenerate_ties(torch_cuda, mapper):
@@ -375,7 +455,7 @@ def test_d5_single_epoch_lean_build(torch_cuda, mapper):
         K, X = workloads.random_tables(700 + Q, 1, Q, 5)
         want = oracle.oracle_map(K, X)
         i, mp, ms = mapper.map_queues(to_dev(torch_cuda, K), to_dev(torch_cuda, X))
-        assert mapper.launch_info()["path"] == "blocked_u32"
+        assert mapper.launch_info()["path"] == "blocked_u32_lean"
         assert int(i[0]) == want[0][0] and int(ms[0]) == want[1][0] and (mp.cpu().numpy() == want[2]).all()
         N, unit = 5**Q, 125
         for r in range(3):
@@ -385,3 +465,29 @@ def test_d5_single_epoch_lean_build(torch_cuda, mapper):
             lo, hi = (nb * r // 3) * unit, (nb * (r + 1) // 3) * unit
             oi, oms, _ = oracle.oracle_map(K, X, lo=lo, hi=hi)
             assert (int(si[0]), int(sms[0])) == (int(oi[0]), int(oms[0])), f"Q={Q} shard {r}"
+        # a batch of D = 5 epochs keeps the two-CTA build
+        KB, XB = workloads.random_tables(710 + Q, 3, Q, 5)
+        wb = oracle.oracle_map(KB, XB)
+        assert_same(run_gpu(torch_cuda, mapper, KB, XB, 1), wb, f"Q={Q} batch")
+        assert mapper.launch_info()["path"] == "blocked_u32"
+
+
+def test_default_stream_follows_torch_current_stream(torch_cuda):
+    """Mapper() without a stream runs on torch's current stream: inputs written
+    on that stream after a 20+ ms spin are complete when the search reads them. (On a
+    private non-blocking stream the search would read the zero tables.)"""
+    torch = torch_cuda
+    K, X = workloads.cfg2(E=300, seed=21)
+    want = oracle.oracle_map(K, X)
+    Ks, Xs = to_dev(torch, K), to_dev(torch, X)
+    torch.cuda.synchronize()
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        Kd, Xd = torch.zeros_like(Ks), torch.zeros_like(Xs)
+        torch.cuda._sleep(40_000_000)  # ~20 ms of device spin on s before the inputs land
+        Kd.copy_(Ks)
+        Xd.copy_(Xs)
+        with Mapper(0) as m:
+            i, mp, ms = m.map_queues(Kd, Xd)
+    torch.cuda.synchronize()
+    assert_same((i.cpu().numpy(), mp.cpu().numpy(), ms.cpu().numpy()), want, "torch stream order")

@@ -122,6 +122,15 @@ def _rank(rank, world, port, q):
                 i, mp, ms = m.map_queues(dev(torch, K), dev(torch, X))
                 out.append((name, i.cpu().numpy(), ms.cpu().numpy(), mp.cpu().numpy(),
                             m.launch_info()["fused_exchange"]))
+            # more epochs than the slabs hold and no communicator: an error, never this
+            # rank's shard-local argmin presented as the global result
+            K, X = workloads.small_int_tables(8, 64, 7, 3, hi=4)
+            try:
+                m.map_queues(dev(torch, K), dev(torch, X))
+                over = "returned"
+            except MclError as exc:
+                over = exc.status
+            out.append(("over max_epochs", over))
             dist.barrier()
         dist.destroy_process_group()
         q.put((rank, out, None))
@@ -146,7 +155,11 @@ def test_fused_exchange_two_ranks_one_gpu(torch_cuda):
         pytest.skip(f"CUDA IPC between two processes on one device unavailable: {errs[0]}")
     assert not errs, errs
     want = {name: oracle.oracle_map(K, X) for name, K, X in _cases() if K.shape[0] <= 8}
+    from paper_conf_cluster_ajipbf15_b200.mcl import MCL_E_INVAL
+
     for rank, out, _ in res:
+        assert out[-1] == ("over max_epochs", MCL_E_INVAL), (rank, out[-1])
+        out = out[:-1]
         assert len(out) == len(want)
         for name, i, ms, mp_, fused in out:
             assert fused, (rank, name)
