@@ -147,10 +147,18 @@ mcl_status_t mcl_peer_import(mcl_mapper_t* h, const uint8_t* handles, uint32_t t
  *               device. A queue pinned to one device has a single bit.
  * The result is the lowest index (in the full D^Q index space) among the mappings that
  * respect every mask and minimise max_d (base_load[d] + sum of C over the queues on d).
- * Either pointer may be NULL; both NULL is mcl_map_queues. Same buffer rules, sharding and
- * errors as mcl_map_queues, plus MCL_E_INVAL when some queue has no eligible device < D.
- * A shard-mode handle (world > 1, no communicator) whose index range holds no feasible
- * mapping reports index = makespan = UINT64_MAX and mapping bytes 0xFF for that epoch.
+ * Either pointer may be NULL; both NULL is mcl_map_queues. Same buffer rules and errors as
+ * mcl_map_queues, plus MCL_E_INVAL when some queue has no eligible device < D.
+ * With masks (2 <= D <= 8, Q >= 3) only the FEASIBLE mappings are enumerated (a true
+ * mixed-radix search): a pinned queue (one eligible device) leaves the enumeration -- its
+ * cost joins its device's base load, its digit is a constant of the index -- and the other
+ * queues run over their eligible devices only (the last three queues over all D devices with
+ * ineligible entries excluded), so the work is proportional to the product of the queues'
+ * eligible-device counts, not to D^Q. Sharding then cuts this feasible enumeration (in
+ * increasing full-index order) into `world` contiguous ranges, per epoch; without masks it
+ * cuts the full index space as in mcl_map_queues. A shard-mode handle (world > 1, no
+ * communicator) whose range holds no feasible mapping reports index = makespan = UINT64_MAX
+ * and mapping bytes 0xFF for that epoch.
  */
 typedef struct {
   const uint64_t* base_load; /* [E][D] or NULL */
@@ -262,7 +270,8 @@ const char* mcl_last_error_string(const mcl_mapper_t* h);
  *             search, 3 = generic search, 4 = small batched (thread per epoch),
  *             5 = register-blocked u32 over a flattened (epoch, block) space,
  *             6 = branch and bound (mcl_map_queues_pruned), 7 = warp-per-epoch batched u32,
- *             8 = register-blocked u32, one-CTA-per-SM build (single epochs, D = 5))
+ *             8 = register-blocked u32, one-CTA-per-SM build (single epochs, D = 5),
+ *             9 / 10 = mixed-radix constrained search over the feasible mappings, u32 / u64)
  *   info[1] = number of kernels launched by the call, info[2] = CTAs of the main kernel,
  *   info[3] = threads per CTA, info[4] = 1 if an NCCL all-reduce ran, 2 if the fused peer
  *   exchange ran, info[5] = index bits of the packed key, info[6] = 1 if the two-step

@@ -48,7 +48,9 @@ mcl_status_t mcl_probe_int_rate(int device, int op, double* lane_ops_per_s,
    blocked u32 over a flattened (epoch, block) space (batched calls), 6 = always run the
    branch-and-bound kernel in mcl_map_queues_pruned (no small-space cutover), 7 = warp-per-
    epoch batched kernel (unconstrained single-GPU batches of the shapes it is instantiated
-   for; chosen automatically from one full wave of epochs). A path that does
+   for; chosen automatically from one full wave of epochs), 8 = mixed-radix constrained
+   kernel (calls with eligible-device masks, 2 <= D <= 8, Q >= 3; the automatic choice for
+   them -- force 1 for the INF-masked full-space blocked kernel instead). A path that does
    not support (Q, D) or the handle's sharding makes the call fail with MCL_E_INVAL. */
 mcl_status_t mcl_force_path(mcl_mapper_t* h, int path);
 

@@ -103,6 +103,7 @@ struct BlockedArgs {
   const uint64_t* base;  // [E][D] pre-existing device loads, or nullptr (constrained variant)
   const uint16_t* elig;  // [E][Q] eligible-device masks (0 = any), or nullptr
   PeerArgs peer;         // fused cross-GPU exchange (out.key / out.pair set), or world = 0
+  int rank, world;       // mixed-radix kernel: shard of the reduced block space (world <= 1: all)
 };
 
 // ceil(log2(N)): bits of the packed key's index field (N >= 1).
@@ -123,6 +124,14 @@ size_t blocked_smem_bytes(uint32_t Q, uint32_t D, bool wide, int threads, size_t
 cudaError_t launch_hold(uint64_t ns, cudaStream_t st);
 cudaError_t launch_blocked(const BlockedArgs& a, bool wide, dim3 grid, int threads, size_t smem,
                            cudaStream_t st, bool lean = false);
+
+// Constrained search over the feasible mappings only (search_mixed.cu, NEXT-3): pinned
+// queues folded into the base loads, mixed-radix outer digits; same arguments and shared
+// memory layout as the blocked kernel (rlo / rhi unused: the shard is a.rank / a.world of
+// each epoch's reduced block space).
+int mixed_ctas_per_sm(uint32_t D, bool wide, int threads, size_t smem);
+cudaError_t launch_mixed(const BlockedArgs& a, bool wide, dim3 grid, int threads, size_t smem,
+                         cudaStream_t st);
 
 // Batched epochs over a flattened (epoch, block) space (search_flat.cu): u32 loads, whole
 // index space per epoch (no sharding), packed keys (index bits <= 32).

@@ -388,7 +388,7 @@ mcl_status_t mcl_set_pipeline_chunks(mcl_mapper_t* h, int chunks) {
 }
 
 mcl_status_t mcl_force_path(mcl_mapper_t* h, int path) {
-  if (!h || path < 0 || path > 7) return MCL_E_INVAL;
+  if (!h || path < 0 || path > 8) return MCL_E_INVAL;
   h->force_path = path;
   return MCL_OK;
 }
@@ -768,13 +768,17 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
   int path;
   // warp-per-epoch kernel: batches of at least one epoch per resident CTA (4 per SM)
   const bool batch_ok = !shard_mode && !multi && !constrained && mcl::batch_supported(Q, D);
+  // eligible-device masks: the mixed-radix kernel enumerates the feasible mappings only
+  const bool mixed_ok = eligible != nullptr && mcl::blocked_supported(Q, D);
   if (!shard_mode && !multi && !constrained && mcl::small_supported(Q, D)) path = 4;
   else if (batch_ok && epochs >= (uint64_t)h->num_sms * 4) path = 7;
+  else if (mixed_ok) path = 9;
   else if (mcl::blocked_supported(Q, D)) path = 1;
   else path = 3;
   if (h->force_path && h->force_path != 6) {  // 6 only affects mcl_map_queues_pruned
     const int f = h->force_path;
     const bool ok = (f == 3) || ((f == 1 || f == 2) && mcl::blocked_supported(Q, D)) ||
+                    (f == 8 && mixed_ok) ||
                     (f == 7 && batch_ok) ||
                     (f == 5 && epochs > 1 && !shard_mode && !multi && !constrained &&
                      mcl::flat_supported(Q, D, mcl::index_bits_host(N))) ||
@@ -783,7 +787,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
       h->last_err = "forced kernel path does not support this shape / sharding";
       return MCL_E_INVAL;
     }
-    path = (f == 5) ? 1 : f;  // 5 = the flattened form of the blocked u32 kernel
+    path = (f == 5) ? 1 : (f == 8 ? 9 : f);  // 5 = the flattened form of the blocked u32 kernel
   }
 
   int nlaunch = 0;
@@ -825,6 +829,45 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
       grid.x = gx;
       threads = 32;
       path = 5;
+    } else if (path == 9 || path == 10) {
+      // constrained: mixed-radix search of the feasible mappings (search_mixed.cu); the
+      // shard is taken per epoch on the device from the reduced block count
+      const bool wide = (path == 10);
+      threads = 256;
+      const uint64_t units = N / ((uint64_t)D * D * D);  // upper bound of the reduced blocks
+      if (epochs > 1)
+        while (threads > 32 && units / (uint64_t)std::max(1, h->world) / threads < 32) threads >>= 1;
+      mcl::BlockedArgs a{};
+      a.Q = Q; a.D = D; a.E = epochs; a.K = K; a.X = X; a.rlo = 0; a.rhi = 0;
+      a.out = out; a.ibits = ibits; a.flags = h->flags_dev; a.one = 1;
+      a.base = Bd; a.elig = Ed; a.peer = peer;
+      a.rank = shard_mode ? h->rank : 0;
+      a.world = shard_mode ? h->world : 1;
+      const size_t smem = mcl::blocked_smem_bytes(Q, D, wide, threads, &a.off_red, &a.off_dig);
+      const int occ = mcl::mixed_ctas_per_sm(D, wide, threads, smem);
+      const uint64_t slots = (uint64_t)h->num_sms * std::max(1, occ);
+      uint64_t e_full = 0, tail_cpe = 1;
+      if (epochs >= slots) {
+        e_full = epochs / slots * slots;
+        const uint64_t rem = epochs - e_full;
+        const uint64_t max_cpe = std::max<uint64_t>(1, units / (uint64_t)threads);
+        tail_cpe = rem ? std::max<uint64_t>(1, std::min(slots / rem, max_cpe)) : 1;
+      } else {
+        tail_cpe = (slots + epochs - 1) / epochs;
+        tail_cpe = std::min<uint64_t>(tail_cpe, std::max<uint64_t>(1, (units + threads - 1) / threads));
+      }
+      tail_cpe = std::min<uint64_t>(tail_cpe, 65535);
+      a.e_full = e_full;
+      a.tail_cpe = (uint32_t)tail_cpe;
+      const uint64_t ncta = e_full + (epochs - e_full) * tail_cpe;
+      grid = dim3((unsigned)std::min<uint64_t>(ncta, 0x7fffffffu), 1, 1);
+      if (tail_cpe > 1) {
+        MCL_CUDA(h, h->scratch.ensure((size_t)(epochs - e_full) * tail_cpe * sizeof(Cand)),
+                 "cudaMalloc(scratch)");
+        a.scratch = (Cand*)h->scratch.p;
+      }
+      a.done = (uint32_t*)h->done.p;
+      MCL_CUDA(h, mcl::launch_mixed(a, wide, grid, threads, smem, s), "search_mixed launch");
     } else if (path == 1 || path == 2) {
       const bool wide = (path == 2);
       const uint64_t nb = N / ((uint64_t)D * D * D);
@@ -928,11 +971,11 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
       h->info[6] = (flags & mcl::kFlagTwoStep) ? 1 : 0;
     }
     if (flags & mcl::kFlagNeedU64) {  // some epoch's bound needs 64-bit loads: rerun the wide kernel
-      if (path != 1 && path != 5 && path != 7) {
+      if (path != 1 && path != 5 && path != 7 && path != 9) {
         h->last_err = "internal: 64-bit request from a 64-bit kernel";
         return MCL_E_CUDA;
       }
-      path = 2;
+      path = (path == 9) ? 10 : 2;
       continue;
     }
     if (use_nccl && (flags & mcl::kFlagNoPack)) {  // key does not pack: two-step lexicographic all-reduce

@@ -37,19 +37,45 @@ def timed(m, fn, mappings):
     return {"kernel_ms": k, "mappings_per_s": mappings / (k / 1e3)}
 
 
+def feasible_count(elig, D):
+    """Mappings allowed by the masks (product of the eligible-device counts), per epoch."""
+    full = (1 << D) - 1
+    m = np.where(elig == 0, full, elig.astype(np.int64) & full)
+    cnt = np.vectorize(lambda v: bin(int(v)).count("1"))(m)
+    return np.prod(cnt.astype(np.float64), axis=1)
+
+
+def verdict_cfg5_constraints():
+    """cfg5 with 3 pinned + 3 masked queues."""
+    base, elig = workloads.constraints(77, 1, 12, 8)
+    elig[0] = 0
+    elig[0, [1, 5, 10]] = [1 << 3, 1 << 0, 1 << 6]
+    elig[0, [2, 7, 11]] = [0b00110110, 0b11000001, 0b0111]
+    return base, elig
+
+
 with Mapper(0) as m:
     m.set_timing(1)
-    for name in ("cfg5", "cfg4", "cfg2"):
+    cases = [(name, workloads.constraints(11, *workloads.make(name)[0].shape), "25% queues pinned, 25% masked, "
+              "base loads U[0,2^20)") for name in ("cfg5", "cfg4", "cfg2")]
+    cases.insert(1, ("cfg5", verdict_cfg5_constraints(), "3 pinned + 3 masked (queue 11 inner), base U[0,2^20)"))
+    for name, (base, elig), what in cases:
         K, X = workloads.make(name)
         E, Q, D = K.shape
         N = E * D**Q
-        base, elig = workloads.constraints(11, E, Q, D)
+        feas = float(feasible_count(elig, D).sum())
         Kd, Xd, Bd, Ed = t(K), t(X), t(base), t(elig)
         r0 = timed(m, lambda: m.map_queues(Kd, Xd), N)
-        r1 = timed(m, lambda: m.map_queues_constrained(Kd, Xd, Bd, Ed), N)
-        print(json.dumps({"measure": "constrained_vs_plain", "workload": name, "plain": r0,
-                          "constrained": r1, "path": m.launch_info()["path"],
-                          "constraints": "25% queues pinned, 25% masked, base loads U[0,2^20)"}), flush=True)
+        r1 = timed(m, lambda: m.map_queues_constrained(Kd, Xd, Bd, Ed), feas)
+        path = m.launch_info()["path"]
+        m.force_path(1)
+        r2 = timed(m, lambda: m.map_queues_constrained(Kd, Xd, Bd, Ed), feas)
+        m.force_path(0)
+        print(json.dumps({"measure": "constrained_mixed_radix", "workload": name, "constraints": what,
+                          "full_space_mappings": N, "feasible_mappings": feas,
+                          "plain": r0, "mixed_radix": {**r1, "path": path, "unit": "feasible mappings/s"},
+                          "full_space_inf_masked": {**r2, "unit": "feasible mappings/s"},
+                          "speedup_vs_full_space": r2["kernel_ms"] / r1["kernel_ms"]}), flush=True)
     K, X = workloads.cfg2()
     Kd, Xd = t(K), t(X)
     for path, label in ((1, "cta_per_epoch"), (5, "flattened")):
@@ -89,11 +115,12 @@ with Mapper(0) as m:
         ex = timed(m, lambda: m.map_queues(Kd, Xd), E * D**Q)
         pr = timed(m, lambda: m.map_queues_pruned(Kd, Xd), E * D**Q)
         a = m.map_queues_pruned(Kd, Xd)
+        nodes = m.launch_info()["nodes"]  # read before the exhaustive call replaces it
         b = m.map_queues(Kd, Xd)
         same = bool((a[0] == b[0]).all().item() and (a[2] == b[2]).all().item())
         print(json.dumps({"measure": "pruned_vs_exhaustive", "workload": name,
                           "exhaustive_kernel_ms": ex["kernel_ms"], "pruned_kernel_ms": pr["kernel_ms"],
-                          "speedup": ex["kernel_ms"] / pr["kernel_ms"], "nodes": m.launch_info()["nodes"],
+                          "speedup": ex["kernel_ms"] / pr["kernel_ms"], "nodes": nodes,
                           "identical_result": same}), flush=True)
     for seed, (Q, D) in enumerate(((16, 8), (20, 4), (24, 3))):
         K, X = workloads.random_tables(500 + seed, 1, Q, D, hi=1 << 22)

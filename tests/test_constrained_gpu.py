@@ -66,30 +66,111 @@ def test_constrained_all_paths(torch_cuda, mapper, Q, D):
     K, X = workloads.random_tables(50 + Q * D, 24, Q, D, hi=1 << 20)
     base, elig = random_constraints(60 + Q * D, 24, Q, D)
     want = oracle.oracle_map_constrained(K, X, base, elig)
-    paths = [0, 3] + ([1, 2] if Q >= 3 and 2 <= D <= 8 else [])
+    paths = [0, 3] + ([1, 2, 8] if Q >= 3 and 2 <= D <= 8 else [])
     for p in paths:
         for b, el in ((base, elig), (None, elig), (base, None)):
+            if p == 8 and el is None:
+                continue  # the mixed-radix kernel serves calls with eligible masks
             w = want if (b is base and el is elig) else oracle.oracle_map_constrained(K, X, b, el)
             check(run(torch_cuda, mapper, K, X, b, el, p), w, f"Q={Q} D={D} path={p}")
 
 
+def mixed_shard_ranges(elig_row, Q, D, G, wide=False):
+    """Full-index ranges [lo, hi) of the G shards of a masked single-epoch call
+    (include/mcl.h: the feasible enumeration cut into contiguous pieces). The mixed-radix
+    kernel's reduced space: pinned queues (one eligible device) leave it; the other queues
+    keep their order; blocks are the digits of all but the last three of them, each over
+    its eligible devices (for u32 with D <= 5 the last of those over all D devices); shard r
+    takes blocks [nb r / G, nb (r + 1) / G). A block's first leaf (inner digits 0) bounds
+    its full indices from below, so every feasible mapping of shard r lies in
+    [first(block lo), first(block hi))."""
+    full = (1 << D) - 1
+    masks = [(int(m) & full) if int(m) else full for m in elig_row]
+    devs = [[d for d in range(D) if (m >> d) & 1] for m in masks]
+    w = [D ** (Q - 1 - q) for q in range(Q)]
+    pinned = [q for q in range(Q) if len(devs[q]) == 1]
+    free = [q for q in range(Q) if len(devs[q]) != 1]
+    O = max(0, len(free) - 3)
+    outer = free[:O]
+    lists = [devs[q] for q in outer]
+    if not wide and D <= 5 and O >= 1:
+        lists[-1] = list(range(D))
+    nb = int(np.prod([len(x) for x in lists])) if lists else 1
+    pin_idx = sum(devs[q][0] * w[q] for q in pinned)
+
+    def first(b):
+        if b >= nb:
+            return D**Q
+        f = pin_idx
+        for p in range(O - 1, -1, -1):
+            r = len(lists[p])
+            f += lists[p][b % r] * w[outer[p]]
+            b //= r
+        return f
+
+    return [(first(nb * r // G), first(nb * (r + 1) // G)) for r in range(G)]
+
+
+def test_mixed_shard_ranges_helper():
+    """The test helper's ranges tile [first feasible block, D^Q) and grow monotonically."""
+    rng = np.random.default_rng(0)
+    for _ in range(50):
+        Q, D, G = int(rng.integers(3, 9)), int(rng.integers(2, 7)), int(rng.integers(1, 9))
+        _, elig = random_constraints(int(rng.integers(1 << 30)), 1, Q, D)
+        rs = mixed_shard_ranges(elig[0], Q, D, G)
+        assert rs[-1][1] == D**Q
+        assert all(rs[i][1] == rs[i + 1][0] for i in range(G - 1))
+        assert all(lo <= hi for lo, hi in rs)
+
+
+def _shards_vs_oracle(torch, K, X, base, elig, G, ranges):
+    best = None
+    for r in range(G):
+        with Mapper(0, rank=r, world=G) as m:
+            i, mp, ms = m.map_queues_constrained(dev(torch, K), dev(torch, X), dev(torch, base), dev(torch, elig))
+        got = (int(ms.cpu().numpy()[0]), int(i.cpu().numpy()[0]))
+        lo, hi = ranges[r]
+        try:
+            if lo >= hi:
+                raise oracle.OracleError(-1)
+            oi, oms, _ = oracle.oracle_map_constrained(K, X, base, elig, lo=lo, hi=hi)
+            assert got == (int(oms[0]), int(oi[0])), f"shard {r}/{G} [{lo}, {hi})"
+        except oracle.OracleError:  # no feasible mapping in this shard: (UINT64_MAX, UINT64_MAX)
+            assert got == (2**64 - 1, 2**64 - 1), f"empty shard {r}"
+            assert (mp.cpu().numpy() == 0xFF).all()
+        best = got if best is None else min(best, got)
+    return best
+
+
 def test_constrained_cfg4_scale_u64_fallback_and_shards(torch_cuda, mapper):
     """A full-size-shaped search (12 queues x 4 devices) with pins; large base loads force
-    64-bit loads; shard-mode handles check the sub-ranges."""
+    64-bit loads; shard-mode handles check the sub-ranges (the mixed-radix kernel's shards
+    of the feasible enumeration, and the INF-masked blocked kernel's full-space shards)."""
     torch = torch_cuda
     K, X = workloads.cfg4(seed=9, Q=12)
     base, elig = random_constraints(9, 1, 12, 4, pin_frac=0.25)
     want = oracle.oracle_map_constrained(K, X, base, elig)
     check(run(torch, mapper, K, X, base, elig), want, "cfg4-12")
+    assert mapper.launch_info()["path"] == "mixed_u32"
+    check(run(torch, mapper, K, X, base, elig, 1), want, "cfg4-12 full space")
     big = base + np.uint64(1 << 40)
     check(run(torch, mapper, K, X, big, elig), oracle.oracle_map_constrained(K, X, big, elig), "u64")
+    assert mapper.launch_info()["path"] == "mixed_u64"
+    G = 7
+    best = _shards_vs_oracle(torch, K, X, base, elig, G, mixed_shard_ranges(elig[0], 12, 4, G))
+    assert best == (int(want[1][0]), int(want[0][0]))
+    # 64-bit loads: no super-block, every outer queue over its eligible devices only
+    wide = _shards_vs_oracle(torch, K, X, big, elig, 5, mixed_shard_ranges(elig[0], 12, 4, 5, wide=True))
+    wb = oracle.oracle_map_constrained(K, X, big, elig)
+    assert wide == (int(wb[1][0]), int(wb[0][0]))
+    # the INF-masked blocked kernel (force 1) shards the full index space
     N = 4**12
     unit = 4**3
     nb = N // unit
     best = None
-    G = 7
     for r in range(G):
         with Mapper(0, rank=r, world=G) as m:
+            m.force_path(1)
             i, mp, ms = m.map_queues_constrained(dev(torch, K), dev(torch, X), dev(torch, base), dev(torch, elig))
         got = (int(ms.cpu().numpy()[0]), int(i.cpu().numpy()[0]))
         lo, hi = (nb * r // G) * unit, (nb * (r + 1) // G) * unit
@@ -162,3 +243,91 @@ def test_score_mappings_every_device_count(torch_cuda, mapper, Q, D):
     assert (got == want).all()
     got = mapper.score_mappings(K, X, mps)
     assert (got == np.array([oracle.oracle_score(K[e], X[e], mps[e]) for e in range(E)], np.uint64)).all()
+
+
+# ------------------------------------------------- mixed radix (feasible mappings only) --
+@pytest.mark.parametrize("Q,D", [(3, 2), (4, 3), (5, 4), (6, 5), (7, 3), (6, 6), (5, 7), (5, 8), (8, 4), (9, 3)])
+def test_mixed_radix_random_and_ties(torch_cuda, mapper, Q, D):
+    """The mixed-radix kernel (auto for masked calls) == the constrained oracle, bit-exact,
+    on random and tie-heavy tables, with pins / masks / bits >= D / zero masks, batched."""
+    torch = torch_cuda
+    E = 40
+    for seed, maker in ((Q * 100 + D, workloads.random_tables), (Q * 100 + D + 1, workloads.small_int_tables)):
+        K, X = maker(seed, E, Q, D)
+        base, elig = random_constraints(seed + 7, E, Q, D, pin_frac=0.35)
+        elig[::5, 0] = np.where(elig[::5, 0] != 0, elig[::5, 0] | np.uint16(1 << 15), 0)  # bits >= D: ignored
+        elig[1::7, :] = 0                   # every queue on any device
+        for b in (base, None):
+            want = oracle.oracle_map_constrained(K, X, b, elig)
+            check(run(torch, mapper, K, X, b, elig), want, f"Q={Q} D={D} {maker.__name__}")
+            assert mapper.launch_info()["path"] == "mixed_u32"
+
+
+@pytest.mark.parametrize("Q,D", [(4, 3), (6, 4), (9, 5), (8, 8)])
+def test_mixed_radix_pins_everywhere(torch_cuda, mapper, Q, D):
+    """Every pinned-queue count, including all queues pinned (a single feasible mapping: the
+    reduced problem is padded with zero-cost virtual inner queues) and pins after the inner
+    queues (their digits are the least significant)."""
+    torch = torch_cuda
+    rng = np.random.default_rng(Q * D)
+    K, X = workloads.random_tables(Q + D, Q + 1, Q, D, hi=1 << 16)
+    base = rng.integers(0, 1 << 16, size=(Q + 1, D), dtype=np.uint64)
+    elig = np.zeros((Q + 1, Q), np.uint16)
+    for e in range(Q + 1):  # epoch e pins e queues (a random subset), masks two more
+        pin = rng.permutation(Q)[:e]
+        elig[e, pin] = (1 << rng.integers(0, D, size=e)).astype(np.uint16)
+        rest = [q for q in range(Q) if q not in set(pin.tolist())][:2]
+        for q in rest:
+            elig[e, q] = np.uint16(int(rng.integers(1, 1 << D)) | (1 << int(rng.integers(0, D))))
+    want = oracle.oracle_map_constrained(K, X, base, elig)
+    check(run(torch, mapper, K, X, base, elig), want, f"pins Q={Q} D={D}")
+    check(run(torch, mapper, K, X, base, elig, 8), want, f"pins Q={Q} D={D} forced")
+
+
+def test_mixed_radix_cfg5_feasible_work(torch_cuda, mapper):
+    """cfg5 (12 x 8) with 3 pinned and 3 masked queues: the mixed-radix kernel scores the
+    feasible space (<= 8^9 leaves here instead of 8^12) and equals the oracle (which also
+    enumerates only what the masks allow, one by one) and the INF-masked full-space kernel."""
+    torch = torch_cuda
+    K, X = workloads.cfg5()
+    base, elig = workloads.constraints(77, 1, 12, 8)
+    elig[0] = 0
+    elig[0, [1, 5, 10]] = [1 << 3, 1 << 0, 1 << 6]          # pinned
+    elig[0, [2, 7, 11]] = [0b00110110, 0b11000001, 0b0111]  # masked (queue 11 is inner)
+    want = pinned_reduced_oracle(K, X, base, elig)
+    check(run(torch, mapper, K, X, base, elig), want, "cfg5 constrained")
+    assert mapper.launch_info()["path"] == "mixed_u32"
+    check(run(torch, mapper, K, X, base, elig, 1), want, "cfg5 constrained full space")
+    # a smaller space the oracle enumerates in full (10 x 8 = 1.1e9 mappings, one by one)
+    K10, X10, b10, e10 = K[:, :10], X[:, :10], base, elig[:, :10].copy()
+    want10 = oracle.oracle_map_constrained(K10, X10, b10, e10)
+    check(run(torch, mapper, K10, X10, b10, e10), want10, "10 x 8 constrained")
+    assert (pinned_reduced_oracle(K10, X10, b10, e10)[0] == want10[0]).all()
+
+
+def pinned_reduced_oracle(K, X, base, elig):
+    """The constrained oracle on the reduced problem of one epoch: every pinned queue's cost
+    moved into its device's base load and the queue removed (test_oracle_constrained.py pins
+    this equivalence, P12), then its digit re-inserted into the returned index. Lets the
+    oracle check full cfg5-sized constrained searches in a fraction of a second."""
+    E, Q, D = K.shape
+    assert E == 1
+    full = (1 << D) - 1
+    m = [(int(v) & full) if int(v) else full for v in elig[0]]
+    pins = {q: m[q].bit_length() - 1 for q in range(Q) if bin(m[q]).count("1") == 1}
+    keep = [q for q in range(Q) if q not in pins]
+    b = (np.zeros(D, np.uint64) if base is None else base[0].astype(np.uint64)).copy()
+    for q, d in pins.items():
+        b[d] += K[0, q, d] + X[0, q, d]
+    if keep:
+        i, ms, mp = oracle.oracle_map_constrained(K[:, keep], X[:, keep], b[None], elig[:, keep])
+        sub = list(mp[0])
+    else:
+        ms = np.array([int(b.max())], np.uint64)
+        sub = []
+    digits = np.zeros(Q, np.uint8)
+    it = iter(sub)
+    for q in range(Q):
+        digits[q] = pins[q] if q in pins else next(it)
+    idx = sum(int(digits[q]) * D ** (Q - 1 - q) for q in range(Q))
+    return np.array([idx], np.uint64), np.asarray(ms, np.uint64).reshape(1), digits[None]
