@@ -252,6 +252,31 @@ mcl_status_t mcl_score_mappings(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_
                                 const uint64_t* base_load, const uint8_t* mappings,
                                 uint64_t* makespan);
 
+/*
+ * Static command-queue scheduling, the SCHED_AUTO_STATIC policy baseline (PAPER.md
+ * L1088-1116, SS V.B: "we statically decide the command queue schedules based only on the
+ * device profiles ... uses the command queue properties (compute intensive, memory
+ * intensive, or I/O intensive) as the selection criterion and chooses the best available
+ * device for the given command queue"; Table I's SCHED_COMPUTE_BOUND / SCHED_MEMORY_BOUND /
+ * SCHED_IO_BOUND hints). No kernel profiles, no search: each queue independently.
+ *   hints        : [E][Q] uint8 class of each queue, < num_classes (e.g. 0 = compute-bound,
+ *                  1 = memory-bound, 2 = I/O-bound)
+ *   num_classes  : 1..16
+ *   device_score : [num_classes][D] uint64 device-profile cost of class c on device d (lower
+ *                  is better, e.g. ns of the class's device benchmark)
+ *   eligible     : [E][Q] uint16 or NULL -- as in mcl_map_queues_constrained ("available")
+ *   mappings     : [E][Q] uint8 out: the eligible device with the lowest score for the
+ *                  queue's class, ties to the lowest device id.
+ * Score the result with mcl_score_mappings to compare the policy with the optimum.
+ * Host or device pointers; synchronous. Errors: MCL_E_INVAL (NULL pointer, bad shape,
+ * num_classes outside 1..16, a hint >= num_classes, a queue with no eligible device < D),
+ * MCL_E_CUDA.
+ */
+mcl_status_t mcl_static_mappings(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                                 const uint8_t* hints, uint32_t num_classes,
+                                 const uint64_t* device_score, const uint16_t* eligible,
+                                 uint8_t* mappings);
+
 /* Destroy a handle (NULL-safe). Frees the handle's scratch; never the caller's buffers and
    never the NCCL communicator (its owner, e.g. the torch process group, keeps it). */
 void mcl_mapper_destroy(mcl_mapper_t* h);

@@ -20,6 +20,7 @@ enum : uint32_t {
   kFlagBadModel = 32u,   // cost model: bad kernel id / source / offsets / curve
   kFlagPeerTimeout = 64u,  // fused exchange: some rank did not signal in time
   kFlagTwoStep = 128u,     // fused exchange ran the two-step reduction (informational)
+  kFlagBadHint = 256u,     // static policy: a queue hint names a class >= num_classes
 };
 
 // Fused cross-GPU exchange (peer.cuh). Slab of each rank, in u64 words:
@@ -221,6 +222,11 @@ cudaError_t launch_score(uint32_t Q, uint32_t D, uint64_t E, const uint64_t* K, 
                          volatile uint32_t* flags, cudaStream_t st);
 cudaError_t launch_generic(const GenericArgs& a, dim3 grid, int threads, size_t smem,
                            cudaStream_t st);
+// Static hint-based mappings (score.cu, SCHED_AUTO_STATIC): per (epoch, queue) the eligible
+// device with the lowest device-profile cost of the queue's class.
+cudaError_t launch_static_map(uint32_t Q, uint32_t D, uint64_t E, const uint8_t* hints,
+                              uint32_t num_classes, const uint64_t* score, const uint16_t* elig,
+                              uint8_t* mapping, volatile uint32_t* flags, cudaStream_t st);
 
 // Batched search, one warp per epoch, compile-time (Q, D) (search_batch.cu): u32 loads,
 // unconstrained, single GPU, shapes with >= ~32 chunks of D^2 blocks per epoch.

@@ -521,6 +521,10 @@ mcl_status_t status_from_flags(mcl_mapper* h) {
     h->last_err = "a cost entry, built cost or base load is >= 2^48";
     return MCL_E_RANGE;
   }
+  if (flags & mcl::kFlagBadHint) {
+    h->last_err = "a queue hint names a class >= num_classes";
+    return MCL_E_INVAL;
+  }
   if (flags & mcl::kFlagInfeasible) {
     h->last_err = "a queue has no eligible device below D";
     return MCL_E_INVAL;
@@ -1334,6 +1338,39 @@ mcl_status_t mcl_score_mappings(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_
            "score launch");
   if ((st = copy_outputs_back(h, epochs, Q, o)) != MCL_OK) return st;
   MCL_CUDA(h, cudaStreamSynchronize(h->stream), "score kernel");
+  return status_from_flags(h);
+}
+
+mcl_status_t mcl_static_mappings(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
+                                 const uint8_t* hints, uint32_t num_classes,
+                                 const uint64_t* device_score, const uint16_t* eligible,
+                                 uint8_t* mappings) {
+  if (!h) return MCL_E_INVAL;
+  h->last_err.clear();
+  mcl_status_t st = check_shape(h, Q, D, epochs, nullptr);
+  if (st != MCL_OK || epochs == 0) return st;
+  if (!hints || !device_score || !mappings || num_classes == 0 || num_classes > MCL_MAX_DEVICES) {
+    h->last_err = "NULL required pointer or num_classes outside 1..16";
+    return MCL_E_INVAL;
+  }
+  DeviceGuard g(h->device);
+  const void *Hd, *Sd, *Ed;
+  if ((st = classify_stage_in(h, h->in_k, hints, epochs * Q, &Hd)) != MCL_OK) return st;
+  if ((st = classify_stage_in(h, h->in_x, device_score, (size_t)num_classes * D * 8, &Sd)) != MCL_OK) return st;
+  if ((st = classify_stage_in(h, h->in_elig, eligible, epochs * Q * 2, &Ed)) != MCL_OK) return st;
+  bool on = true;
+  if ((st = classify(h, mappings, &on)) != MCL_OK) return st;
+  uint8_t* Md = mappings;
+  if (!on) {
+    MCL_CUDA(h, h->out_map.ensure(epochs * Q), "cudaMalloc(staging)");
+    Md = (uint8_t*)h->out_map.p;
+  }
+  clear_flags(h);
+  MCL_CUDA(h, mcl::launch_static_map(Q, D, epochs, (const uint8_t*)Hd, num_classes, (const uint64_t*)Sd,
+                                     (const uint16_t*)Ed, Md, h->flags_dev, h->stream),
+           "static_map launch");
+  if (!on) MCL_CUDA(h, cudaMemcpyAsync(mappings, Md, epochs * Q, cudaMemcpyDeviceToHost, h->stream), "D2H");
+  MCL_CUDA(h, cudaStreamSynchronize(h->stream), "static_map kernel");
   return status_from_flags(h);
 }
 

@@ -76,4 +76,60 @@ cudaError_t launch_score(uint32_t Q, uint32_t D, uint64_t E, const uint64_t* K, 
   return cudaGetLastError();
 }
 
+// Static command-queue scheduling (SCHED_AUTO_STATIC): "we statically
+// decide the command queue schedules based only on the device profiles ... [using] the
+// command queue properties (compute intensive, memory intensive, or I/O intensive) as the
+// selection criterion and [choose] the best available device for the given command queue"
+// (reading R18). Thread per (epoch, queue): among the queue's eligible devices,
+// the one whose device-profile cost for the queue's class is lowest (ties: lowest device).
+// No kernel profiles and no search: the policy baseline the mapper is compared with.
+__global__ void __launch_bounds__(256) static_map_kernel(uint32_t Q, uint32_t D, uint64_t EQ,
+                                                         const uint8_t* __restrict__ hints,
+                                                         uint32_t num_classes,
+                                                         const uint64_t* __restrict__ score,
+                                                         const uint16_t* __restrict__ elig,
+                                                         uint8_t* __restrict__ mapping,
+                                                         volatile uint32_t* flags) {
+  __shared__ uint64_t s_score[kMaxDevices * kMaxDevices];
+  for (uint32_t t = threadIdx.x; t < num_classes * D; t += blockDim.x) s_score[t] = score[t];
+  __syncthreads();
+  uint32_t status = 0;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < EQ;
+       i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t c = hints[i];
+    const uint32_t m = elig ? (uint32_t)elig[i] : 0u;
+    uint32_t best_d = 0xffu;
+    uint64_t best = ~0ull;
+    if (c >= num_classes) {
+      status |= kFlagBadHint;
+    } else {
+      for (uint32_t d = 0; d < D; ++d) {
+        if (m != 0 && !((m >> d) & 1u)) continue;
+        const uint64_t v = s_score[c * D + d];
+        if (best_d == 0xffu || v < best) {  // strict: the lowest device among equal scores
+          best = v;
+          best_d = d;
+        }
+      }
+      if (best_d == 0xffu) status |= kFlagInfeasible;
+    }
+    mapping[i] = (uint8_t)best_d;
+  }
+  if (__any_sync(0xffffffffu, status != 0)) {
+    const uint32_t all = __reduce_or_sync(0xffffffffu, status);
+    if ((threadIdx.x & 31) == 0) raise_flag(flags, all);
+  }
+}
+
+cudaError_t launch_static_map(uint32_t Q, uint32_t D, uint64_t E, const uint8_t* hints,
+                              uint32_t num_classes, const uint64_t* score, const uint16_t* elig,
+                              uint8_t* mapping, volatile uint32_t* flags, cudaStream_t st) {
+  const uint64_t EQ = E * Q;
+  uint64_t grid = (EQ + 255) / 256;
+  if (grid > 148 * 16) grid = 148 * 16;
+  if (grid == 0) grid = 1;
+  static_map_kernel<<<(unsigned)grid, 256, 0, st>>>(Q, D, EQ, hints, num_classes, score, elig, mapping, flags);
+  return cudaGetLastError();
+}
+
 }  // namespace mcl

@@ -175,7 +175,7 @@ __device__ __forceinline__ uint64_t mixed_span_first_warp(uint64_t bb, uint32_t 
 }  // namespace
 
 template <typename T, int D>
-__global__ void __launch_bounds__(256, 1) search_mixed_kernel(BlockedArgs a) {
+__global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1) search_mixed_kernel(BlockedArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const uint32_t Q = a.Q;
   const int nthr = blockDim.x, tid = threadIdx.x;
@@ -239,60 +239,64 @@ __global__ void __launch_bounds__(256, 1) search_mixed_kernel(BlockedArgs a) {
     // INF of an ineligible entry: above every feasible makespan (epoch_prologue put
     // UB_f + 1 into the masked entries; without masks the bound UB itself)
     const uint64_t inf = (s_feas != kNone ? s_feas : s_ub) + 1;
-    // ---- the reduced problem (one thread: Q <= 32 queues, once per epoch) ----
-    if (tid == 0) {
-      const uint32_t full = (1u << D) - 1u;
-      uint64_t wq = 1;  // D^(Q-1-q): D^(Q-1) <= 2^48 (D^Q <= 2^48 is checked on the host)
-      for (uint32_t q = 1; q < Q; ++q) wq *= D;
-      uint64_t pin = 0;
-      uint32_t n = 0;
-      for (uint32_t q = 0; q < Q; ++q, wq /= D) {
-        uint32_t m = elig_e ? (uint32_t)elig_e[q] & full : full;
-        if (!elig_e || elig_e[q] == 0) m = full;
-        if (__popc(m) == 1) {  // pinned: its cost joins the device's base load (radix 1)
-          const uint32_t d = __ffs(m) - 1;
-          s_base[d] += C64[q * D + d];
-          pin += (uint64_t)d * wq;
-          continue;
-        }
-        mt.orig[n] = (int8_t)q;
-        mt.w[n] = wq;
+    // ---- the reduced problem (one warp: lane q handles queue q, Q <= 32) ----
+    if (tid < 32) {
+      const uint32_t lane = tid, full = (1u << D) - 1u;
+      const bool act = lane < Q;
+      uint32_t m = full;
+      if (act && elig_e && elig_e[lane] != 0) m = (uint32_t)elig_e[lane] & full;
+      const bool pinned = act && __popc(m) == 1;
+      uint64_t wq = 1;  // D^(Q-1-q) <= 2^48 (D^Q <= 2^48 is checked on the host)
+      for (uint32_t t = lane + 1; t < Q; ++t) wq *= D;
+      const uint32_t freeb = __ballot_sync(0xffffffffu, act && !pinned);
+      const uint32_t n = __popc(freeb);
+      uint64_t pin = 0, rm = 0;
+      if (pinned) {  // its cost joins the device's base load; its digit is a constant (radix 1)
+        const uint32_t d = __ffs(m) - 1;
+        atomicAdd(reinterpret_cast<unsigned long long*>(&s_base[d]), (unsigned long long)C64[lane * D + d]);
+        pin = (uint64_t)d * wq;
+      } else if (act) {  // reduced queue p keeps its order among the unpinned queues
+        const uint32_t p = __popc(freeb & ((1u << lane) - 1u));
+        mt.orig[p] = (int8_t)lane;
+        mt.w[p] = wq;
         uint32_t r = 0;
-        for (uint32_t d = 0; d < D; ++d)
-          if ((m >> d) & 1u) mt.dev[n][r++] = (uint8_t)d;
-        mt.radix[n] = (uint8_t)r;
-        ++n;
+        for (uint32_t d = 0; d < D; ++d) {
+          if ((m >> d) & 1u) mt.dev[p][r++] = (uint8_t)d;
+          rm = max(rm, C64[lane * D + d]);  // INF entries included: a bound of every leaf
+        }
+        mt.radix[p] = (uint8_t)r;
       }
-      while (n < 3) {  // virtual inner queues: zero cost on device 0 only, weight 0
-        mt.orig[n] = -1;
-        mt.w[n] = 0;
-        mt.radix[n] = 1;
-        mt.dev[n][0] = 0;
-        ++n;
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) {
+        pin += __shfl_xor_sync(0xffffffffu, pin, off);
+        rm += __shfl_xor_sync(0xffffffffu, rm, off);
       }
-      mt.Qr = n;
-      mt.O = n - 3;
-      // the super-block queue (outer position O-1, D <= 5) keeps all D devices (INF entries)
-      if (sizeof(T) == 4 && D <= kSuperMaxD && mt.O >= 1 && mt.orig[mt.O - 1] >= 0) {
-        mt.radix[mt.O - 1] = D;
-        for (uint32_t d = 0; d < D; ++d) mt.dev[mt.O - 1][d] = (uint8_t)d;
+      __syncwarp();
+      if (lane == 0) {
+        uint32_t nn = n;
+        for (; nn < 3; ++nn) {  // virtual inner queues: zero cost on device 0 only, weight 0
+          mt.orig[nn] = -1;
+          mt.w[nn] = 0;
+          mt.radix[nn] = 1;
+          mt.dev[nn][0] = 0;
+          rm += inf;
+        }
+        mt.Qr = nn;
+        mt.O = nn - 3;
+        // the super-block queue (outer position O-1, D <= 5) keeps all D devices (INF entries)
+        if (sizeof(T) == 4 && D <= kSuperMaxD && mt.O >= 1) {
+          mt.radix[mt.O - 1] = D;
+          for (uint32_t d = 0; d < D; ++d) mt.dev[mt.O - 1][d] = (uint8_t)d;
+        }
+        uint64_t nb = 1;
+        for (uint32_t p = 0; p < mt.O; ++p) nb *= mt.radix[p];
+        mt.nb = nb;
+        mt.pin_idx = pin;
+        // bound of every leaf the kernel forms: max base' + sum of the reduced rows' maxima
+        uint64_t bm = 0;
+        for (uint32_t d = 0; d < D; ++d) bm = max(bm, s_base[d]);
+        s_ub = bm + rm;
       }
-      uint64_t nb = 1;
-      for (uint32_t p = 0; p < mt.O; ++p) nb *= mt.radix[p];
-      mt.nb = nb;
-      mt.pin_idx = pin;
-      // bound of every leaf the kernel forms (INF entries included): max base' + sum over
-      // the reduced queues of their largest entry -- decides 32- vs 64-bit loads
-      uint64_t ub = 0;
-      for (uint32_t d = 0; d < D; ++d) ub = max(ub, s_base[d]);
-      for (uint32_t p = 0; p < n; ++p) {
-        const int q = mt.orig[p];
-        uint64_t rm = (q >= 0) ? 0 : inf;
-        if (q >= 0)
-          for (uint32_t d = 0; d < D; ++d) rm = max(rm, C64[q * D + d]);
-        ub += rm;
-      }
-      s_ub = ub;
     }
     __syncthreads();
     if (sizeof(T) == 4 && s_ub >= 0xffffffffull) {  // UB < 2^32 - 1 for 32-bit loads

@@ -29,7 +29,7 @@ EXPORTED = [
     "mcl_comm_unique_id", "mcl_comm_init", "mcl_comm_destroy",
     "mcl_map_queues_constrained", "mcl_score_mappings", "mcl_map_queues_pruned",
     "mcl_build_costs", "mcl_map_from_profiles",
-    "mcl_peer_export", "mcl_peer_import",
+    "mcl_peer_export", "mcl_peer_import", "mcl_static_mappings",
 ]
 
 
@@ -112,6 +112,7 @@ def load_library(path: str | None = None) -> ctypes.CDLL:
                                         ctypes.POINTER(mcl_constraints_t), vp, vp, vp]),
         "mcl_peer_export": (i32, [vp, u64, ctypes.c_char_p]),
         "mcl_peer_import": (i32, [vp, ctypes.c_char_p, u32]),
+        "mcl_static_mappings": (i32, [vp, u32, u32, u64, vp, u32, vp, vp, vp]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -484,6 +485,32 @@ class Mapper:
         if st != MCL_OK:
             raise MclError(st, "mcl_score_mappings", mcl_last_error_string(self.handle))
         return ms
+
+    def static_mappings(self, hints, device_score, eligible=None):
+        """SCHED_AUTO_STATIC policy baseline (include/mcl.h mcl_static_mappings): hints
+        [E, Q] uint8 queue classes, device_score [C, D] uint64 (lower is better), eligible
+        [E, Q] uint16 or None. Returns mappings [E, Q] uint8 like ``hints`` (torch / numpy)."""
+        if hints.ndim != 2 or device_score.ndim != 2:
+            raise ValueError("hints: [E, Q]; device_score: [C, D]")
+        E, Q = (int(s) for s in hints.shape)
+        C, D = (int(s) for s in device_score.shape)
+        _check("eligible", eligible, (E, Q))
+        try:
+            import torch
+        except ImportError:  # pragma: no cover
+            torch = None
+        if torch is not None and isinstance(hints, torch.Tensor):
+            out = torch.empty((E, Q), dtype=torch.uint8, device=hints.device)
+        else:
+            out = np.empty((E, Q), np.uint8)
+        ph, _h = _ptr_and_keepalive(hints, np.uint8)
+        ps, _s = _ptr_and_keepalive(device_score, np.uint64, convert=True)
+        pe, _e = _ptr_and_keepalive(eligible, np.uint16) if eligible is not None else (None, None)
+        po, _o = _ptr_and_keepalive(out, np.uint8)
+        st = load_library().mcl_static_mappings(self.handle, Q, D, E, ph, C, ps, pe, po)
+        if st != MCL_OK:
+            raise MclError(st, "mcl_static_mappings", mcl_last_error_string(self.handle))
+        return out
 
     @staticmethod
     def _alloc_outputs(K, E, Q, with_mapping):

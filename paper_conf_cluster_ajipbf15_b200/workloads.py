@@ -209,3 +209,33 @@ def cost_model(seed: int, E: int, Q: int, D: int, n_kernels: int = 64, max_kerne
     d2h = (peak_d2h[:, None] * s[None, :] / (s[None, :] + half)).astype(np.float64)
     return dict(profile=profile, offsets=offsets, kernel_ids=kernel_ids, bytes=nbytes, source=source,
                 cached=cached, sizes=sizes, h2d_bw=h2d, d2h_bw=d2h, host_shared=1)
+
+
+def static_hints(K, X):
+    """SCHED_COMPUTE_BOUND / SCHED_MEMORY_BOUND / SCHED_IO_BOUND hints (Table I, PAPER.md
+    L1100-1116) a programmer would annotate the queues of a synthetic epoch with -- input
+    synthesis for the SCHED_AUTO_STATIC baseline, [E, Q] uint8: I/O-bound (2) when moving the
+    queue's data to a GPU costs more on average than its kernels there, else compute-bound
+    (0) when some GPU runs its kernels faster than the CPU (device 0), else memory-bound (1).
+    D = 1 (no GPU): every queue is compute-bound."""
+    K = np.asarray(K)
+    X = np.asarray(X)
+    if K.shape[-1] < 2:
+        return np.zeros(K.shape[:-1], np.uint8)
+    gk, gx = K[..., 1:].astype(np.float64), X[..., 1:].astype(np.float64)
+    io = gx.mean(-1) > gk.mean(-1)
+    compute = K[..., 1:].min(-1) < K[..., 0]
+    return np.where(io, 2, np.where(compute, 0, 1)).astype(np.uint8)
+
+
+def static_device_scores(D: int):
+    """Device-profile cost of each hint class on each device ([3, D] uint64, lower is
+    better; device 0 = the CPU): compute-bound work is 4x faster on a GPU,
+    memory-bound work 2x faster on the CPU (the SNU-NPB pattern of Fig. 3),
+    I/O-bound queues cost nothing to keep on the host-resident CPU. Every GPU has the same
+    profile (a homogeneous node), so the static policy sends all compute-bound queues to the
+    first GPU -- the load imbalance the dynamic mapper avoids (L1096-1100)."""
+    s = np.ones((3, D), np.uint64)
+    s[0, 0], s[1, 0], s[2, 0] = 4, 1, 0
+    s[1, 1:] = 2
+    return s

@@ -76,8 +76,25 @@ with Mapper(0) as m:
                           "plain": r0, "mixed_radix": {**r1, "path": path, "unit": "feasible mappings/s"},
                           "full_space_inf_masked": {**r2, "unit": "feasible mappings/s"},
                           "speedup_vs_full_space": r2["kernel_ms"] / r1["kernel_ms"]}), flush=True)
+    # policy baselines vs the optimum (PAPER.md L584-587 ROUND_ROBIN, L1088-1116 AUTO_STATIC)
     K, X = workloads.cfg2()
+    E, Q, D = K.shape
     Kd, Xd = t(K), t(X)
+    opt = m.map_queues(Kd, Xd)[2].double()
+    hints, score = workloads.static_hints(K, X), workloads.static_device_scores(D)
+    st_map = m.static_mappings(t(hints), t(score))
+    rr_map = t(np.tile((np.arange(Q) % D).astype(np.uint8), (E, 1)))
+    for label, mp in (("auto_static_hints", st_map), ("round_robin", rr_map)):
+        ms = m.score_mappings(Kd, Xd, mp).double()
+        ratio = (ms / opt.clamp(min=1)).cpu().numpy()
+        nz = (opt > 0).cpu().numpy()
+        print(json.dumps({"measure": "policy_vs_optimum", "workload": "cfg2", "policy": label,
+                          "makespan_ratio_mean": float(ratio[nz].mean()),
+                          "makespan_ratio_median": float(np.median(ratio[nz])),
+                          "makespan_ratio_max": float(ratio[nz].max()),
+                          "epochs_optimal": float((ms == opt).double().mean()),
+                          "note": "makespan of the policy's mapping / the mapper's optimum, per epoch "
+                                  "(epochs with optimum 0 excluded from the ratios)"}), flush=True)
     for path, label in ((1, "cta_per_epoch"), (5, "flattened")):
         m.force_path(path)
         r = timed(m, lambda: m.map_queues(Kd, Xd), K.shape[0] * 4**8)

@@ -331,3 +331,30 @@ def pinned_reduced_oracle(K, X, base, elig):
         digits[q] = pins[q] if q in pins else next(it)
     idx = sum(int(digits[q]) * D ** (Q - 1 - q) for q in range(Q))
     return np.array([idx], np.uint64), np.asarray(ms, np.uint64).reshape(1), digits[None]
+
+
+def test_static_policy_baseline(torch_cuda, mapper):
+    """SCHED_AUTO_STATIC: the GPU's hint-based mappings equal the
+    policy oracle's (with and without eligible masks); scored through mcl_score_mappings they
+    never beat the mapper's optimum, and do worse on most epochs."""
+    from oracle import policies
+
+    torch = torch_cuda
+    K, X = workloads.cfg2(E=2000, seed=31)
+    E, Q, D = K.shape
+    hints = workloads.static_hints(K, X)
+    score = workloads.static_device_scores(D)
+    _, elig = random_constraints(31, E, Q, D, pin_frac=0.0)
+    for el in (None, elig):
+        want = policies.static_mapping(hints, score, el)
+        got = mapper.static_mappings(dev(torch, hints), dev(torch, score), None if el is None else dev(torch, el))
+        assert (got.cpu().numpy() == want).all()
+        assert (mapper.static_mappings(hints, score, el) == want).all()  # host buffers
+    st = mapper.score_mappings(dev(torch, K), dev(torch, X), dev(torch, want)).cpu().numpy()
+    assert (st == np.array([oracle.oracle_score(K[e], X[e], want[e]) for e in range(E)], np.uint64)).all()
+    opt = oracle.oracle_map(K, X)[1]
+    assert (opt <= st).all() and (opt < st).mean() > 0.5
+    with pytest.raises(MclError):
+        mapper.static_mappings(np.full((1, Q), 3, np.uint8), score)  # hint >= classes
+    with pytest.raises(MclError):
+        mapper.static_mappings(hints[:1], score, np.full((1, Q), 1 << 15, np.uint16))  # no device
