@@ -62,8 +62,8 @@ def _load():
         lib.oracle_build_costs.argtypes = [
             ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_uint32,
             ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
-            ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
-            ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p,
+            ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p,
+            ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p,
         ]
         lib.oracle_score_base.restype = ctypes.c_uint64
         lib.oracle_score_base.argtypes = [
@@ -164,8 +164,9 @@ def oracle_score_base(K, X, base, mapping) -> int:
 def oracle_build_costs(Q: int, D: int, model: dict):
     """Cost tables (NEXT-1) from a cost model dict with keys: profile [n_kernels, D] u64,
     offsets [E*Q+1] u64, kernel_ids [nnz] u32, bytes [E, Q] u64, source [E, Q] i32
-    (-1 = host), cached [E, Q] u16 or None, sizes [M] u64, h2d_bw / d2h_bw [D, M] f64,
-    host_shared (int bit mask). Returns (K, X) uint64 [E, Q, D]."""
+    (-1 = host), cached [E, Q] u16 or None, sizes [M] u64, h2d_bw / d2h_bw [D, M] or
+    [S, D, M] f64 (per host socket), host_socket [E, Q] u8 or None (socket 0), host_shared
+    (int bit mask). Returns (K, X) uint64 [E, Q, D]."""
     prof = np.ascontiguousarray(model["profile"], dtype=np.uint64)
     off = np.ascontiguousarray(model["offsets"], dtype=np.uint64)
     ids = np.ascontiguousarray(model["kernel_ids"], dtype=np.uint32)
@@ -176,6 +177,9 @@ def oracle_build_costs(Q: int, D: int, model: dict):
     sizes = np.ascontiguousarray(model["sizes"], dtype=np.uint64)
     h2d = np.ascontiguousarray(model["h2d_bw"], dtype=np.float64)
     d2h = np.ascontiguousarray(model["d2h_bw"], dtype=np.float64)
+    S = 1 if h2d.ndim == 2 else int(h2d.shape[0])
+    hs = model.get("host_socket")
+    hs = None if hs is None else np.ascontiguousarray(hs, dtype=np.uint8)
     E = nbytes.shape[0]
     K = np.zeros((E, Q, D), dtype=np.uint64)
     X = np.zeros((E, Q, D), dtype=np.uint64)
@@ -183,7 +187,8 @@ def oracle_build_costs(Q: int, D: int, model: dict):
     rc = _load().oracle_build_costs(
         Q, D, E, prof.shape[0], prof.ctypes.data, off.ctypes.data, ids_ptr, nbytes.ctypes.data,
         src.ctypes.data, None if cached is None else cached.ctypes.data, sizes.shape[0],
-        sizes.ctypes.data, h2d.ctypes.data, d2h.ctypes.data, int(model.get("host_shared", 0)),
+        sizes.ctypes.data, S, None if hs is None else hs.ctypes.data,
+        h2d.ctypes.data, d2h.ctypes.data, int(model.get("host_shared", 0)),
         K.ctypes.data, X.ctypes.data,
     )
     if rc != 0:

@@ -106,3 +106,80 @@ def test_errors():
         oracle.oracle_build_costs(2, 3, model_one(source=np.array([[-1, 3]], np.int32)))
     with pytest.raises(oracle.OracleError):
         oracle.oracle_build_costs(2, 3, model_one(sizes=np.array([5, 5], np.uint64)))
+
+
+# ------------------------------------------- per-socket curves (R19) and range (R10) ---
+def model_two_sockets(**over):
+    """model_one on a two-socket host: socket 0 keeps 4 / 2 bytes/ns (H2D / D2H), socket 1 is
+    the far socket at 1 / 0.5 bytes/ns (the GPUs have affinity to one
+    socket, so the host thread's socket changes the transfer cost)."""
+    h2d = np.stack([np.full((3, 2), 4.0), np.full((3, 2), 1.0)])
+    d2h = np.stack([np.full((3, 2), 2.0), np.full((3, 2), 0.5)])
+    return model_one(h2d_bw=h2d, d2h_bw=d2h, **over)
+
+
+def test_socket_curves_closed_forms():
+    hs = np.array([[1, 1]], np.uint8)
+    K, X = oracle.oracle_build_costs(2, 3, model_two_sockets(host_socket=hs))
+    assert list(X[0, 0]) == [4096, 4096, 4096]                  # H2D from socket 1: 4096 / 1
+    assert list(X[0, 1]) == [2000 + 1000, 0, 2000 + 1000]        # D2H + H2D both via socket 1
+    K0, X0 = oracle.oracle_build_costs(2, 3, model_two_sockets(host_socket=np.zeros((1, 2), np.uint8)))
+    K1, X1 = oracle.oracle_build_costs(2, 3, model_one())
+    assert (X0 == X1).all() and (K0 == K1).all() and (K == K1).all()  # socket 0 = the plain model
+    # mixed: queue 0 near, queue 1 far
+    _, Xm = oracle.oracle_build_costs(2, 3, model_two_sockets(host_socket=np.array([[0, 1]], np.uint8)))
+    assert list(Xm[0, 0]) == [1024, 1024, 1024] and list(Xm[0, 1]) == [3000, 0, 3000]
+
+
+def test_one_socket_axis_is_the_plain_model():
+    m = workloads.cost_model(7, 30, 5, 4)
+    K, X = oracle.oracle_build_costs(5, 4, m)
+    m3 = dict(m, h2d_bw=m["h2d_bw"][None], d2h_bw=m["d2h_bw"][None], host_socket=np.zeros((30, 5), np.uint8))
+    K3, X3 = oracle.oracle_build_costs(5, 4, m3)
+    assert (K == K3).all() and (X == X3).all()
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_socket_relabeling_invariance(seed):
+    """Permuting the sockets (their curves and every queue's label alike) changes nothing."""
+    rng = np.random.default_rng(seed)
+    E, Q, D, S = 12, 4, 3, 3
+    m = workloads.cost_model(300 + seed, E, Q, D)
+    h2d = np.stack([m["h2d_bw"] * f for f in (1.0, 0.5, 0.25)])
+    d2h = np.stack([m["d2h_bw"] * f for f in (1.0, 0.7, 0.3)])
+    hs = rng.integers(0, S, size=(E, Q)).astype(np.uint8)
+    K, X = oracle.oracle_build_costs(Q, D, dict(m, h2d_bw=h2d, d2h_bw=d2h, host_socket=hs))
+    perm = rng.permutation(S)            # new socket i = old socket perm[i]
+    inv = np.argsort(perm)
+    Kp, Xp = oracle.oracle_build_costs(Q, D, dict(m, h2d_bw=h2d[perm], d2h_bw=d2h[perm],
+                                                  host_socket=inv[hs].astype(np.uint8)))
+    assert (K == Kp).all() and (X == Xp).all()
+    # a slower socket never costs less
+    _, Xs = oracle.oracle_build_costs(Q, D, dict(m, h2d_bw=h2d, d2h_bw=d2h, host_socket=np.full((E, Q), 2, np.uint8)))
+    _, Xf = oracle.oracle_build_costs(Q, D, dict(m, h2d_bw=h2d, d2h_bw=d2h, host_socket=np.zeros((E, Q), np.uint8)))
+    assert (Xs >= Xf).all() and (Xs > Xf).any()
+
+
+def test_profile_and_sum_range():
+    """Entries must be < 2^48 and a kernel sum that reaches 2^48 is out of range (checked as
+    it grows, so it can never wrap around to a small accepted value)."""
+    big = np.array([[1 << 47, 1, 1], [(1 << 47) - 1, 1, 1], [1 << 48, 1, 1]], np.uint64)
+    ok = model_one(profile=big, offsets=np.array([0, 1, 2], np.uint64), kernel_ids=np.array([0, 1], np.uint32))
+    K, _ = oracle.oracle_build_costs(2, 3, dict(ok, profile=big[:2]))
+    assert int(K[0, 0, 0]) == 1 << 47
+    two = dict(ok, profile=big[:2], offsets=np.array([0, 2, 2], np.uint64), kernel_ids=np.array([0, 1], np.uint32))
+    K, _ = oracle.oracle_build_costs(2, 3, two)          # 2^47 + 2^47 - 1 = 2^48 - 1: fine
+    assert int(K[0, 0, 0]) == (1 << 48) - 1
+    with pytest.raises(oracle.OracleError):             # 2^47 + 2^47 = 2^48
+        oracle.oracle_build_costs(2, 3, dict(two, kernel_ids=np.array([0, 0], np.uint32)))
+    with pytest.raises(oracle.OracleError):             # an entry of 2^48, even if never invoked
+        oracle.oracle_build_costs(2, 3, dict(ok, kernel_ids=np.array([0, 1], np.uint32)))
+    many = dict(ok, profile=big[:2], offsets=np.array([0, 70000, 70000], np.uint64),
+                kernel_ids=np.zeros(70000, np.uint32))   # 70000 x 2^47 would wrap a u64 sum
+    with pytest.raises(oracle.OracleError):
+        oracle.oracle_build_costs(2, 3, many)
+
+
+def test_socket_out_of_range():
+    with pytest.raises(oracle.OracleError):
+        oracle.oracle_build_costs(2, 3, model_two_sockets(host_socket=np.array([[0, 2]], np.uint8)))
