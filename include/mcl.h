@@ -206,7 +206,13 @@ mcl_status_t mcl_map_queues_pruned(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint
  *                sampled sizes and clamped outside them (device profiler: bandwidths over
  *                sizes "from latency bound to bandwidth bound", "simple interpolation
  *                techniques" for other sizes, L877-913); IEEE fp64, no fused multiply-add.
- * Every array may be host or device memory (host arrays are staged).
+ *                The curves are per host socket ("H2D bandwidths are run for all the CPU
+ *                socket-device combinations", L897-901; nonuniform host-device distances,
+ *                L1349-1361): queue q's host memory -- its data, or the staging buffer of a
+ *                D2H-H2D double operation -- is on socket host_socket[e][q], and both legs
+ *                use that socket's curves.
+ * Every array may be host or device memory (host arrays are staged). K sums are exact: a
+ * profile entry >= 2^48 or a sum reaching 2^48 is MCL_E_RANGE (never a wrapped value).
  */
 typedef struct {
   uint32_t num_kernels;            /* rows of kernel_profile                             */
@@ -219,15 +225,18 @@ typedef struct {
   const uint16_t* cached;          /* [E][Q] devices already holding a copy, or NULL      */
   uint32_t num_sizes;              /* M sampled sizes, 1..64                              */
   const uint64_t* sizes;           /* [M] strictly ascending bytes                        */
-  const double* h2d_bw;            /* [D][M] host->device bandwidth, bytes/ns, > 0        */
-  const double* d2h_bw;            /* [D][M] device->host bandwidth, bytes/ns, > 0        */
+  const double* h2d_bw;            /* [S][D][M] host->device bandwidth, bytes/ns, > 0     */
+  const double* d2h_bw;            /* [S][D][M] device->host bandwidth, bytes/ns, > 0     */
   uint32_t host_shared;            /* bit d: device d works on host memory                */
+  uint32_t num_sockets;            /* S host sockets, 1..8 (0 = 1)                        */
+  const uint8_t* host_socket;      /* [E][Q] socket of each queue's host memory (< S), or
+                                      NULL = socket 0                                      */
 } mcl_cost_model_t;
 
 /* Build K and X ([E][Q][D] uint64, host or device outputs). Errors: MCL_E_INVAL (NULL
-   pointer, Q/D out of bounds, num_sizes outside 1..64, a kernel id >= num_kernels, a source
-   outside -1..D-1, bad offsets, sizes not ascending or a bandwidth <= 0), MCL_E_RANGE (a
-   cost >= 2^48), MCL_E_CUDA. */
+   pointer, Q/D out of bounds, num_sizes outside 1..64, num_sockets above 8, a kernel id >=
+   num_kernels, a source outside -1..D-1, a socket >= S, bad offsets, sizes not ascending or a
+   bandwidth <= 0), MCL_E_RANGE (a profile entry, kernel sum or cost >= 2^48), MCL_E_CUDA. */
 mcl_status_t mcl_build_costs(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
                              const mcl_cost_model_t* model, uint64_t* cost_kernel,
                              uint64_t* cost_xfer);

@@ -189,36 +189,38 @@ __device__ __forceinline__ void load_vec(T (&v)[D], const T* __restrict__ src) {
 }
 
 // Lowest leaf of a block whose makespan equals `target` (the block is known to hold one),
-// found cooperatively: called by all 32 lanes with the same (P, target),
-// lane l evaluates leaves l, l + 32, ... directly from the definition (runtime digits
-// i, j, k; loads P[d] plus the inner queues' costs on their devices; max over devices) and
-// a ballot per round finds the lowest leaf equal to `target`. Replaces a serial re-scan of
-// the whole block by one lane.
+// found cooperatively by the 32 lanes (same P, same target): lane l takes the (i, j) pairs
+// p = l, l + 32, ... of the two outer inner queues (runtime digits, loads formed by static
+// per-device selects), then scores the D leaves k of the pair with static k, directly from
+// the definition (loads P[d] plus the inner queues' costs on their devices, max over
+// devices); leaf = p * D + k, and the warp minimum of every lane's first hit is the lowest
+// leaf. One pass of at most two pairs per lane instead of D^3 / 32 rounds of runtime-digit
+// scoring (the rescan sits on the kernel's critical tail).
 template <typename T, int D>
 __device__ __forceinline__ uint32_t block_first_warp(const T (&P)[D], const T* __restrict__ in,
                                                      T target) {
-  constexpr uint32_t kLeaves = (uint32_t)D * D * D;
+  constexpr uint32_t kPairs = (uint32_t)D * D;
   const uint32_t lane = threadIdx.x & 31;
-  for (uint32_t r0 = 0; r0 < kLeaves; r0 += 32) {
-    const uint32_t l = r0 + lane;
-    bool hit = false;
-    if (l < kLeaves) {
-      const uint32_t i = l / (D * D), j = (l / D) % D, k = l % D;
-      T ms = 0;
+  uint32_t first = 0xffffffffu;
+  for (uint32_t p = lane; p < kPairs; p += 32) {
+    const uint32_t i = p / D, j = p % D;
+    T L[D];
+    T Mp = 0;
 #pragma unroll
-      for (int d = 0; d < D; ++d) {
-        T L = P[d];
-        if (i == (uint32_t)d) L += in[0 * D + d];
-        if (j == (uint32_t)d) L += in[1 * D + d];
-        if (k == (uint32_t)d) L += in[2 * D + d];
-        ms = max2(ms, L);
-      }
-      hit = (ms == target);
+    for (int d = 0; d < D; ++d) {
+      T v = P[d];
+      if (i == (uint32_t)d) v += in[0 * D + d];
+      if (j == (uint32_t)d) v += in[1 * D + d];
+      L[d] = v;
+      Mp = max2(Mp, v);
     }
-    const uint32_t b = __ballot_sync(0xffffffffu, hit);
-    if (b) return r0 + (uint32_t)(__ffs(b) - 1);
+    uint32_t hit = 0xffffffffu;
+#pragma unroll
+    for (int k = D - 1; k >= 0; --k)
+      if (max2(Mp, (T)(L[k] + in[2 * D + k])) == target) hit = p * D + (uint32_t)k;
+    if (hit < first) first = hit;  // pairs ascend per lane: the first hit is its lowest
   }
-  return 0xffffffffu;
+  return __reduce_min_sync(0xffffffffu, first);
 }
 
 // Prefix loads P of block `blk` (outer digits of queues 0..O-1), decoded from scratch,

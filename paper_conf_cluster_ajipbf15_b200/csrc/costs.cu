@@ -11,8 +11,13 @@
 //                                                     double operation via the host", L1293-1301
 //  with no H2D/D2H leg for a device flagged host_shared, and t(curve, b) = ceil(b / bw(b))
 //  ns, bw linearly interpolated between the sampled sizes and clamped at the ends ("simple
-//  interpolation techniques", L905-907). fp64 with explicitly rounded operations (no FMA
-//  contraction), so the result is bit-identical to a plain IEEE evaluation.
+//  interpolation techniques", L905-907). The curves are per (host socket, device) ("all the
+//  CPU socket-device combinations", L897-901; nonuniform host-device distances, L1349-1361):
+//  a queue's host memory is on socket host_socket[e][q], whose curves both legs use (DESIGN.md
+//  R19). fp64 with explicitly rounded operations (no FMA contraction), so the result is
+//  bit-identical to a plain IEEE evaluation. Range (R10): a profile entry >= 2^48, or a kernel
+//  sum reaching 2^48, raises kFlagRange (lists of >= 2^16 invocations check every addition,
+//  shorter ones cannot wrap a u64 and are checked once).
 //
 // Tiles of 256 (epoch, queue) pairs per CTA, one thread per pair: it sums its invocations'
 // profile rows and interpolates the curves (sizes and bandwidths in shared memory; one
@@ -59,18 +64,19 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const uint32_t M = a.M;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  // layout: outK[kCostTile*D] u64 | outX[kCostTile*D] u64 | sizes[M] u64 | h2d[D][M] f64 |
-  //         d2h[D][M] f64 | prof[num_kernels][D] u64 (if it fits)
+  // layout: outK[kCostTile*D] u64 | outX[kCostTile*D] u64 | sizes[M] u64 | h2d[S][D][M] f64 |
+  //         d2h[S][D][M] f64 | prof[num_kernels][D] u64 (if it fits)
+  const uint32_t S = a.S;
   uint64_t* s_outK = reinterpret_cast<uint64_t*>(smem_raw);
   uint64_t* s_outX = s_outK + (size_t)kCostTile * D;
   uint64_t* s_sizes = s_outX + (size_t)kCostTile * D;
   double* s_h2d = reinterpret_cast<double*>(s_sizes + M);
-  double* s_d2h = s_h2d + (size_t)D * M;
-  uint64_t* s_prof = reinterpret_cast<uint64_t*>(s_d2h + (size_t)D * M);
+  double* s_d2h = s_h2d + (size_t)S * D * M;
+  uint64_t* s_prof = reinterpret_cast<uint64_t*>(s_d2h + (size_t)S * D * M);
   constexpr int PS = prof_stride<D>();
   const bool prof_in_smem = (size_t)a.num_kernels * PS * 8 <= (size_t)kProfCapBytes;
   for (uint32_t t = tid; t < M; t += blockDim.x) s_sizes[t] = a.sizes[t];
-  for (uint32_t t = tid; t < D * M; t += blockDim.x) {
+  for (uint32_t t = tid; t < S * D * M; t += blockDim.x) {
     s_h2d[t] = a.h2d[t];
     s_d2h[t] = a.d2h[t];
   }
@@ -93,18 +99,22 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
   __syncthreads();
   const uint64_t* prof = prof_in_smem ? s_prof : a.profile;
   uint32_t status = 0;
-  if (blockIdx.x == 0 && tid == 0) {  // model validation (once)
-    for (uint32_t i = 0; i + 1 < M; ++i)
-      if (!(s_sizes[i] < s_sizes[i + 1])) status |= kFlagBadModel;
-    for (uint32_t i = 0; i < D * M; ++i)
-      if (!(s_h2d[i] > 0.0) || !(s_d2h[i] > 0.0)) status |= kFlagBadModel;
-    if (a.offsets[a.EQ] != a.nnz) status |= kFlagBadModel;
+  if (blockIdx.x == 0) {  // model validation (once)
+    if (tid == 0) {
+      for (uint32_t i = 0; i + 1 < M; ++i)
+        if (!(s_sizes[i] < s_sizes[i + 1])) status |= kFlagBadModel;
+      for (uint32_t i = 0; i < S * D * M; ++i)
+        if (!(s_h2d[i] > 0.0) || !(s_d2h[i] > 0.0)) status |= kFlagBadModel;
+      if (a.offsets[a.EQ] != a.nnz) status |= kFlagBadModel;
+    }
+    for (uint32_t t = tid; t < a.num_kernels * D; t += blockDim.x)
+      if (a.profile[t] >= kEntryLimit) status |= kFlagRange;  // every entry, invoked or not
   }
 
   // this thread's pair of a tile, loaded one tile ahead
   uint64_t n_j0 = 0, n_j1 = 0, n_bytes = 0;
   int32_t n_src = 0;
-  uint32_t n_cached = 0;
+  uint32_t n_cached = 0, n_sock = 0;
   auto fetch = [&](uint64_t tile) {
     const uint64_t eq = tile * kCostTile + tid;
     if (eq < a.EQ) {
@@ -113,6 +123,7 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
       n_bytes = a.bytes[eq];
       n_src = a.source[eq];
       n_cached = a.cached ? (uint32_t)a.cached[eq] : 0u;
+      n_sock = a.host_socket ? (uint32_t)a.host_socket[eq] : 0u;
     }
   };
   const uint64_t ntiles = (a.EQ + kCostTile - 1) / kCostTile;
@@ -120,7 +131,7 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
   for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const uint64_t j0 = n_j0, j1 = n_j1, bytes = n_bytes;
     const int32_t src = n_src;
-    const uint32_t cached = n_cached;
+    const uint32_t cached = n_cached, sock = n_sock;
     if (tile + gridDim.x < ntiles) fetch(tile + gridDim.x);
     const uint64_t eq = tile * kCostTile + tid;
     if (eq < a.EQ) {
@@ -129,7 +140,27 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
 #pragma unroll
       for (int d = 0; d < D; ++d) k[d] = 0;
       bool ok = j0 <= j1 && j1 <= a.nnz;
-      if (ok && fits32) {
+      if (ok && j1 - j0 >= 65536u) {
+        // a long list could wrap a u64 sum of entries < 2^48: check every addition, stop at
+        // 2^48 (the range error), as the definition's running sum does
+        for (uint64_t j = j0; j < j1 && ok; ++j) {
+          const uint32_t kid = __ldg(a.ids + j);
+          if (kid >= a.num_kernels) {
+            ok = false;
+            break;
+          }
+          bool over = false;
+#pragma unroll
+          for (int d = 0; d < D; ++d) {
+            if (k[d] < kEntryLimit) k[d] += a.profile[(uint64_t)kid * D + d];
+            over |= k[d] >= kEntryLimit;
+          }
+          if (over) {
+            status |= kFlagRange;
+            break;
+          }
+        }
+      } else if (ok && fits32) {
 #pragma unroll 4
         for (uint64_t j = j0; j < j1; ++j) {
           const uint32_t kid = __ldg(a.ids + j);
@@ -155,8 +186,10 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
         }
       }
       // ---- transfer part ----
-      ok = ok && src >= -1 && src < (int32_t)D;
+      ok = ok && src >= -1 && src < (int32_t)D && sock < S;
       if (!ok) status |= kFlagBadModel;
+      const double* h2d_s = s_h2d + (size_t)(ok ? sock : 0) * D * M;
+      const double* d2h_s = s_d2h + (size_t)(ok ? sock : 0) * D * M;
       const bool clo = bytes <= s_sizes[0], chi = bytes >= s_sizes[M - 1];
       uint32_t seg = 0;
       double f = 0.0;
@@ -173,14 +206,14 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
       }
       uint64_t down = 0;
       if (ok && src >= 0 && !((a.host_shared >> src) & 1u))
-        down = transfer_ns(bytes, lerp_bw(s_d2h + (size_t)src * M, seg, f, clo, chi, M));
+        down = transfer_ns(bytes, lerp_bw(d2h_s + (size_t)src * M, seg, f, clo, chi, M));
 #pragma unroll
       for (int d = 0; d < D; ++d) {
         uint64_t x = 0;
         if (ok && !(src == d || ((cached >> d) & 1u))) {
           const uint64_t up = ((a.host_shared >> d) & 1u)
                                   ? 0
-                                  : transfer_ns(bytes, lerp_bw(s_h2d + (size_t)d * M, seg, f, clo, chi, M));
+                                  : transfer_ns(bytes, lerp_bw(h2d_s + (size_t)d * M, seg, f, clo, chi, M));
           x = down + up;
         }
         if (k[d] >= kEntryLimit || x >= kEntryLimit) status |= kFlagRange;
@@ -211,22 +244,25 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
 namespace {
 template <int D>
 cudaError_t launch_build_costs_t(const CostArgs& a, int num_sms, cudaStream_t st) {
-  size_t smem = 2 * (size_t)kCostTile * D * 8 + (size_t)a.M * 8 + 2 * (size_t)D * a.M * 8;
+  size_t smem = 2 * (size_t)kCostTile * D * 8 + (size_t)a.M * 8 + 2 * (size_t)a.S * D * a.M * 8;
   if ((size_t)a.num_kernels * prof_stride<D>() * 8 <= (size_t)kProfCapBytes)
     smem += (size_t)a.num_kernels * prof_stride<D>() * 8;
   auto k = build_costs_kernel<D>;
   static SmemAttrCache cache;
   cudaError_t err = ensure_smem(k, smem, cache);
   if (err != cudaSuccess) return err;
-  static std::atomic<int> occ[64];
+  // resident CTAs per SM at this shared-memory size (persistent grid); the last query is
+  // cached per device, keyed by the size (it depends on sockets, samples and the profile)
+  static std::atomic<uint64_t> occ[64];
   int dev = 0;
   cudaGetDevice(&dev);
-  int per_sm = occ[dev & 63].load(std::memory_order_relaxed);
-  if (per_sm == 0) {  // resident CTAs per SM at this shared-memory size (persistent grid)
+  const uint64_t hit = occ[dev & 63].load(std::memory_order_relaxed);
+  int per_sm = (hit >> 8) == (uint64_t)smem + 1 ? (int)(hit & 0xff) : 0;
+  if (per_sm == 0) {
     err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kCostTile, smem);
     if (err != cudaSuccess) return err;
-    per_sm = per_sm < 1 ? 1 : per_sm;
-    occ[dev & 63].store(per_sm, std::memory_order_relaxed);
+    per_sm = per_sm < 1 ? 1 : (per_sm > 255 ? 255 : per_sm);
+    occ[dev & 63].store((((uint64_t)smem + 1) << 8) | (uint64_t)per_sm, std::memory_order_relaxed);
   }
   uint64_t grid = (a.EQ + kCostTile - 1) / kCostTile;
   const uint64_t cap = (uint64_t)num_sms * per_sm;

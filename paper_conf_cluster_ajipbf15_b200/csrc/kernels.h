@@ -105,6 +105,8 @@ struct BlockedArgs {
   const uint16_t* elig;  // [E][Q] eligible-device masks (0 = any), or nullptr
   PeerArgs peer;         // fused cross-GPU exchange (out.key / out.pair set), or world = 0
   int rank, world;       // mixed-radix kernel: shard of the reduced block space (world <= 1: all)
+  uint64_t* keyslot;     // [E] packed (makespan, index) keys of split epochs: all ones on
+                         // entry, self-resetting; nullptr = merge through scratch only
 };
 
 // ceil(log2(N)): bits of the packed key's index field (N >= 1).
@@ -206,8 +208,10 @@ struct CostArgs {
   const uint16_t* cached;     // [EQ] or nullptr
   uint32_t M;
   const uint64_t* sizes;      // [M]
-  const double* h2d;          // [D][M]
-  const double* d2h;          // [D][M]
+  uint32_t S;                 // host sockets (>= 1)
+  const uint8_t* host_socket; // [EQ] or nullptr (socket 0)
+  const double* h2d;          // [S][D][M]
+  const double* d2h;          // [S][D][M]
   uint32_t host_shared;
   uint64_t* K;                // [EQ][D] out
   uint64_t* X;                // [EQ][D] out

@@ -131,11 +131,12 @@ struct mcl_mapper {
   int rank = 0, world = 1;
   int num_sms = 148;
   DevBuf scratch;          // Cand per (epoch, CTA) when an epoch spans several CTAs
+  DevBuf keyslot;          // packed-key merge slot per epoch (all ones between calls)
   DevBuf done;             // uint32 per epoch, zero between calls
   DevBuf key, pair, gms, cand;
   DevBuf flat_keys, flat_done;  // flattened batched kernel: per-epoch key / block count
   DevBuf bnb_next, bnb_inc, bnb_nodes;  // pruned search: subtree counters, incumbents, nodes
-  DevBuf model_buf[9], cost_k, cost_x;  // cost-table construction: staged model, built K / X
+  DevBuf model_buf[10], cost_k, cost_x;  // cost-table construction: staged model, built K / X
   DevBuf in_k, in_x, in_base, in_elig, out_idx, out_ms, out_map;  // staging for host pointers
   // fused peer exchange (NEXT-2): own slab, kernel CTA counter, two-step scratch, and the
   // device array of every rank's slab address (peers' slabs opened through CUDA IPC)
@@ -342,7 +343,7 @@ void mcl_mapper_destroy(mcl_mapper_t* h) {
     if (h->stream) cudaStreamSynchronize(h->stream);
     for (void* p : h->peer_opened) cudaIpcCloseMemHandle(p);
     for (DevBuf* b : {&h->peer_slab, &h->peer_kdone, &h->peer_gms, &h->peer_ptrs}) b->release();
-    for (DevBuf* b : {&h->scratch, &h->done, &h->key, &h->pair, &h->gms, &h->cand, &h->flat_keys,
+    for (DevBuf* b : {&h->scratch, &h->keyslot, &h->done, &h->key, &h->pair, &h->gms, &h->cand, &h->flat_keys,
                       &h->flat_done, &h->bnb_next, &h->bnb_inc, &h->bnb_nodes, &h->in_k,
                       &h->in_base, &h->in_elig,
                       &h->in_x, &h->out_idx, &h->out_ms, &h->out_map, &h->cost_k, &h->cost_x})
@@ -920,6 +921,11 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
         MCL_CUDA(h, h->scratch.ensure((size_t)(epochs - e_full) * tail_cpe * sizeof(Cand)),
                  "cudaMalloc(scratch)");
         a.scratch = (Cand*)h->scratch.p;
+        if (h->keyslot.cap < epochs * 8) {  // per-epoch packed keys, all ones between calls
+          MCL_CUDA(h, h->keyslot.ensure(epochs * 8), "cudaMalloc(keyslot)");
+          MCL_CUDA(h, h->keyslot.fill(0xff), "cudaMemset(keyslot)");
+        }
+        a.keyslot = (uint64_t*)h->keyslot.p;
       }
       a.done = (uint32_t*)h->done.p;
       MCL_CUDA(h, mcl::launch_blocked(a, wide, grid, threads, smem, s, lean), "search_blocked launch");
@@ -1208,18 +1214,19 @@ mcl_status_t build_costs_dev(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t e
                              const mcl_cost_model_t* m, uint64_t* Kd, uint64_t* Xd) {
   if (!m || !m->kernel_profile || !m->offsets || !m->bytes || !m->source || !m->sizes ||
       !m->h2d_bw || !m->d2h_bw || (m->num_invocations && !m->kernel_ids) ||
-      m->num_sizes == 0 || m->num_sizes > 64 || m->num_kernels == 0) {
-    h->last_err = "invalid cost model (NULL array, num_sizes outside 1..64 or no kernels)";
+      m->num_sizes == 0 || m->num_sizes > 64 || m->num_kernels == 0 || m->num_sockets > 8) {
+    h->last_err = "invalid cost model (NULL array, num_sizes outside 1..64, num_sockets > 8 or no kernels)";
     return MCL_E_INVAL;
   }
   const uint64_t EQ = epochs * Q;
   const uint32_t M = m->num_sizes;
+  const uint32_t S = m->num_sockets ? m->num_sockets : 1;
   struct Arr {
     const void* src;
     size_t bytes;
     DevBuf* buf;
     const void* dev;
-  } arrs[9] = {
+  } arrs[10] = {
       {m->kernel_profile, (size_t)m->num_kernels * D * 8, &h->model_buf[0], nullptr},
       {m->offsets, (size_t)(EQ + 1) * 8, &h->model_buf[1], nullptr},
       {m->kernel_ids, (size_t)m->num_invocations * 4, &h->model_buf[2], nullptr},
@@ -1227,8 +1234,9 @@ mcl_status_t build_costs_dev(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t e
       {m->source, (size_t)EQ * 4, &h->model_buf[4], nullptr},
       {m->cached, (size_t)EQ * 2, &h->model_buf[5], nullptr},
       {m->sizes, (size_t)M * 8, &h->model_buf[6], nullptr},
-      {m->h2d_bw, (size_t)D * M * 8, &h->model_buf[7], nullptr},
-      {m->d2h_bw, (size_t)D * M * 8, &h->model_buf[8], nullptr},
+      {m->h2d_bw, (size_t)S * D * M * 8, &h->model_buf[7], nullptr},
+      {m->d2h_bw, (size_t)S * D * M * 8, &h->model_buf[8], nullptr},
+      {m->host_socket, (size_t)EQ, &h->model_buf[9], nullptr},
   };
   mcl_status_t st;
   for (auto& a : arrs) {
@@ -1242,6 +1250,7 @@ mcl_status_t build_costs_dev(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t e
   c.bytes = (const uint64_t*)arrs[3].dev; c.source = (const int32_t*)arrs[4].dev;
   c.cached = (const uint16_t*)arrs[5].dev; c.M = M; c.sizes = (const uint64_t*)arrs[6].dev;
   c.h2d = (const double*)arrs[7].dev; c.d2h = (const double*)arrs[8].dev;
+  c.S = S; c.host_socket = (const uint8_t*)arrs[9].dev;
   c.host_shared = m->host_shared; c.K = Kd; c.X = Xd; c.flags = h->flags_dev;
   MCL_CUDA(h, mcl::launch_build_costs(c, h->num_sms, h->stream), "build_costs launch");
   return MCL_OK;

@@ -28,6 +28,28 @@
 
 namespace mcl {
 
+#ifdef MCL_TRACE
+// Measurement build only (scripts/build_variant.py ... -DMCL_TRACE): per CTA, %globaltimer
+// and clock64 at the kernel start, after the tables, after every thread's walk, and at the
+// end -- to split the per-launch fixed cost into ramp, prologue, walk and reduction.
+__device__ unsigned long long g_mcl_trace[4096][8];
+__device__ __forceinline__ unsigned long long trace_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define MCL_TRACE_AT(slot)                                                                 \
+  do {                                                                                     \
+    if (threadIdx.x == 0 && blockIdx.x < 4096) {                                           \
+      g_mcl_trace[blockIdx.x][2 * (slot)] = trace_ns();                                    \
+      g_mcl_trace[blockIdx.x][2 * (slot) + 1] = (unsigned long long)clock64();             \
+    }                                                                                      \
+  } while (0)
+#else
+#define MCL_TRACE_AT(slot) \
+  do {                     \
+  } while (0)
+#endif
 
 // Kernel work layout over a 1-D grid of CTAs: the first e_full epochs get one CTA each; the
 // remaining E - e_full epochs (the "tail") get tail_cpe CTAs each, so the last wave of a
@@ -62,6 +84,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5 && !kLean) ? 2 
 
   const uint64_t ncta = a.e_full + (a.E - a.e_full) * a.tail_cpe;
   bool abandoned = false;  // an epoch skipped on an input error / for the 64-bit rerun
+  MCL_TRACE_AT(0);
   for (uint64_t cta = blockIdx.x; cta < ncta; cta += gridDim.x) {
     uint64_t e;
     uint32_t part, parts;
@@ -126,6 +149,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5 && !kLean) ? 2 
     }
     __syncthreads();
 
+    MCL_TRACE_AT(1);
     // ---- a2-a5: this thread's contiguous block range inside the rank's range ----
     // Split points are aligned to whole CHUNKS (D^2 blocks on the super-block path) so the
     // lanes of a warp walk chunks in lock-step; only the rank's two ends can be ragged.
@@ -152,10 +176,12 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5 && !kLean) ? 2 
     const WalkCtx<T, D> wctx{in, V, zero, base0, dig, O, nthr, tid, one};
     walk_blocks<T, D>(wctx, b0, nleft, best, best_blk, best_span);
     // ---- a5: lowest index inside the best block, then warp / CTA / epoch argmin ----
-    // Thread ranges ascend with the thread id, so the CTA's lowest-index optimum belongs to
-    // the LOWEST thread whose best equals the CTA minimum; only that thread re-scans its
-    // best block (one block per CTA instead of one per thread).
+    // Every block belongs to one thread and a thread's span [best_blk, best_blk + span)
+    // holds its first minimum, so among the threads whose best equals the CTA minimum the
+    // one with the LOWEST best_blk owns the CTA's lowest-index optimum; only that thread's
+    // warp re-scans its best block (one block per CTA instead of one per thread).
     __shared__ uint64_t s_gmin;
+    __shared__ unsigned long long s_winblk;
     __shared__ uint32_t s_winner;
     __shared__ Cand s_cand;
     {
@@ -164,8 +190,12 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5 && !kLean) ? 2 
 #pragma unroll
       for (int off = 16; off > 0; off >>= 1) wmin = min(wmin, __shfl_xor_sync(0xffffffffu, wmin, off));
       __syncthreads();  // `red` may still be read by a previous epoch's reduction
+      MCL_TRACE_AT(2);
       if ((tid & 31) == 0) red[tid >> 5].ms = wmin;
-      if (tid == 0) s_winner = 0xffffffffu;
+      if (tid == 0) {
+        s_winner = 0xffffffffu;
+        s_winblk = ~0ull;
+      }
       __syncthreads();
       if (tid == 0) {
         uint64_t g = kNone;
@@ -174,7 +204,10 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5 && !kLean) ? 2 
         s_cand = Cand{kNone, kNone};
       }
       __syncthreads();
-      if (bv != kNone && bv == s_gmin) atomicMin(&s_winner, (uint32_t)tid);
+      const bool holder = bv != kNone && bv == s_gmin;
+      if (holder) atomicMin(&s_winblk, (unsigned long long)best_blk);
+      __syncthreads();
+      if (holder && best_blk == s_winblk) s_winner = (uint32_t)tid;
       __syncthreads();
       const uint32_t win = s_winner;
       if (win != 0xffffffffu && (uint32_t)(tid >> 5) == (win >> 5)) {  // the winner's warp
@@ -192,17 +225,37 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5 && !kLean) ? 2 
       if (tid == 0) write_epoch(a.out, e, Q, D, a.ibits, c, a.flags, s_feas);
       continue;
     }
-    // a split epoch: per-CTA candidates in scratch; the last CTA to finish reduces them
+    // a split epoch. When (makespan, index) packs into one u64 (UB < 2^(64 - ibits); every
+    // CTA of the epoch sees the same UB), the CTAs fold their candidates into one per-epoch
+    // key with atomicMin and the last CTA only decodes it (the lexicographic minimum is the
+    // minimum key); otherwise per-CTA candidates go to scratch and the last CTA reduces them.
     __shared__ bool s_last;
+    const bool packed = a.keyslot && a.ibits > 0 && a.ibits < 64 && (s_ub >> (64 - a.ibits)) == 0;
     Cand* slots = a.scratch + (e - a.e_full) * parts;
     if (tid == 0) {
-      slots[part] = c;
+      if (packed) {
+        if (c.ms != kNone)
+          atomicMin(reinterpret_cast<unsigned long long*>(a.keyslot + e),
+                    (unsigned long long)((c.ms << a.ibits) | c.idx));
+      } else {
+        slots[part] = c;
+      }
       __threadfence();
       const uint32_t prev = atomicAdd(&a.done[e], 1u);
       s_last = (prev == parts - 1);
     }
     __syncthreads();
-    if (s_last) {
+    if (s_last && packed) {
+      if (tid == 0) {
+        __threadfence();
+        // read and reset the key in one atomic (all-ones = no candidate / the next call's start)
+        const uint64_t key = atomicExch(reinterpret_cast<unsigned long long*>(a.keyslot + e), ~0ull);
+        const Cand r = (key == kNone) ? Cand{kNone, kNone}
+                                      : Cand{key >> a.ibits, key & ((1ull << a.ibits) - 1)};
+        write_epoch(a.out, e, Q, D, a.ibits, r, a.flags, s_feas);
+        a.done[e] = 0;
+      }
+    } else if (s_last) {
       __threadfence();
       Cand r{kNone, kNone};
       for (uint32_t t = tid; t < parts; t += nthr) {
@@ -216,9 +269,18 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5 && !kLean) ? 2 
       }
     }
   }
+  MCL_TRACE_AT(3);
   // fused cross-GPU exchange (NEXT-2): the last CTA reduces over every rank and decodes
   if (a.peer.world) peer_finish(a.peer, a.out, a.E, Q, D, a.ibits, a.flags, abandoned);
 }
+
+#ifdef MCL_TRACE
+}  // namespace mcl
+extern "C" int mcl_trace_read(unsigned long long* out, int n) {
+  return (int)cudaMemcpyFromSymbol(out, mcl::g_mcl_trace, (size_t)n * 8 * sizeof(unsigned long long));
+}
+namespace mcl {
+#endif
 
 template <typename T, int D, bool L = false>
 static cudaError_t launch_blocked_t(const BlockedArgs& a, dim3 grid, int threads, size_t smem,

@@ -44,7 +44,7 @@ class mcl_cost_model_t(ctypes.Structure):
         ("num_invocations", ctypes.c_uint64), ("bytes", ctypes.c_void_p),
         ("source", ctypes.c_void_p), ("cached", ctypes.c_void_p), ("num_sizes", ctypes.c_uint32),
         ("sizes", ctypes.c_void_p), ("h2d_bw", ctypes.c_void_p), ("d2h_bw", ctypes.c_void_p),
-        ("host_shared", ctypes.c_uint32),
+        ("host_shared", ctypes.c_uint32), ("num_sockets", ctypes.c_uint32), ("host_socket", ctypes.c_void_p),
     ]
 
 
@@ -384,14 +384,17 @@ class Mapper:
         _check("source", model["source"], (E, Q))
         _check("cached", model.get("cached"), (E, Q))
         _check("sizes", model["sizes"], (M,))
+        S = 1 if model["h2d_bw"].ndim == 2 else int(model["h2d_bw"].shape[0])
         for name in ("h2d_bw", "d2h_bw"):
-            _check(name, model[name], (D, M))
+            _check(name, model[name], (D, M) if model[name].ndim == 2 else (S, D, M))
+        _check("host_socket", model.get("host_socket"), (E, Q))
         c = mcl_cost_model_t(
             int(model["profile"].shape[0]), p("profile", np.uint64), p("offsets", np.uint64),
             p("kernel_ids", np.uint32) if int(model["kernel_ids"].shape[0]) else None,
             int(model["kernel_ids"].shape[0]), p("bytes", np.uint64), p("source", np.int32),
             p("cached", np.uint16, optional=True), int(model["sizes"].shape[0]), p("sizes", np.uint64),
             p("h2d_bw", np.float64), p("d2h_bw", np.float64), int(model.get("host_shared", 0)),
+            S, p("host_socket", np.uint8, optional=True),
         )
         return c, keep, E, Q
 

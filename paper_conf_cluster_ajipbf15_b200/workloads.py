@@ -176,14 +176,19 @@ def constraints(seed: int, E: int, Q: int, D: int, pin_frac: float = 0.25, mask_
 
 
 def cost_model(seed: int, E: int, Q: int, D: int, n_kernels: int = 64, max_kernels: int = 16,
-               cached_frac: float = 0.1):
+               cached_frac: float = 0.1, sockets: int = 1):
     """Seeded inputs of the cost-table construction step (NEXT-1), shaped by the paper:
     a kernel profile table whose GPU/CPU time ratios span Fig. 3's
     range (0.05x .. 4x, L1391-1401, L2058-2060); 1..max_kernels invocations per (epoch,
     queue) (a kernel epoch, L1142-1158); working sets log-uniform in 1 KiB .. 256 MiB (Fig. 6
     axis, L1854-1876) resident on the host or a GPU; bandwidth curves sampled at powers of
     two from 1 KiB to 1 GiB, latency-bound at small sizes ("from being latency bound to
-    bandwidth bound", L896-898); device 0 is the CPU device working on host memory."""
+    bandwidth bound", L896-898); device 0 is the CPU device working on host memory.
+    With ``sockets`` > 1 the curves are per (socket, device), [S, D, M] ("all the CPU
+    socket-device combinations", L897-901): socket 0 is near the GPUs and every further
+    socket reaches them through an inter-socket link at 0.55-0.8 of the bandwidth and a
+    longer latency (the paper's node: GPUs with affinity to one socket, L1349-1361); each
+    queue's host memory is on a random socket (``host_socket`` [E, Q])."""
     rng = np.random.default_rng(seed)
     cpu = rng.integers(100_000, 10_000_000, size=n_kernels)
     profile = np.zeros((n_kernels, D), dtype=np.uint64)
@@ -207,8 +212,18 @@ def cost_model(seed: int, E: int, Q: int, D: int, n_kernels: int = 64, max_kerne
     s = sizes.astype(np.float64)
     h2d = (peak_h2d[:, None] * s[None, :] / (s[None, :] + half)).astype(np.float64)
     d2h = (peak_d2h[:, None] * s[None, :] / (s[None, :] + half)).astype(np.float64)
-    return dict(profile=profile, offsets=offsets, kernel_ids=kernel_ids, bytes=nbytes, source=source,
-                cached=cached, sizes=sizes, h2d_bw=h2d, d2h_bw=d2h, host_shared=1)
+    model = dict(profile=profile, offsets=offsets, kernel_ids=kernel_ids, bytes=nbytes, source=source,
+                 cached=cached, sizes=sizes, h2d_bw=h2d, d2h_bw=d2h, host_shared=1)
+    if sockets > 1:
+        far = rng.uniform(0.55, 0.8, size=(sockets, D))
+        far[0] = 1.0
+        lat = 1.0 + 2.0 * (np.arange(sockets) > 0)  # the far sockets' longer latency ...
+        model["h2d_bw"] = np.stack([far[k][:, None] * peak_h2d[:, None] * s[None, :] / (s[None, :] + half * lat[k])
+                                    for k in range(sockets)]).astype(np.float64)
+        model["d2h_bw"] = np.stack([far[k][:, None] * peak_d2h[:, None] * s[None, :] / (s[None, :] + half * lat[k])
+                                    for k in range(sockets)]).astype(np.float64)
+        model["host_socket"] = rng.integers(0, sockets, size=(E, Q)).astype(np.uint8)
+    return model
 
 
 def static_hints(K, X):

@@ -1,0 +1,42 @@
+"""A/B kernel timing of two builds of libmcl.so on one GPU (measurement only):
+
+    python scripts/ab_lib.py build/ab/libmcl_old.so build/ab/libmcl_new.so [rounds]
+
+Each round runs every library in a fresh subprocess (alternating order) and prints the
+median kernel time (CUDA events, 200 us spin hold, L2 flushed) of the single-epoch configs
+at G = 1 and of rank 0 at G = 8, and of cfg2.
+"""
+import json
+import os
+import subprocess
+import sys
+
+CHILD = r'''
+import json, os, statistics, sys
+sys.path.insert(0, os.environ["REPO"])
+import torch
+from paper_conf_cluster_ajipbf15_b200 import mcl, workloads
+mcl.load_library(os.environ["LIB"])
+flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+st = torch.cuda.Stream(); torch.cuda.set_stream(st)
+out = {}
+for name in ("cfg5", "cfg4", "cfg2"):
+    K, X = workloads.make(name); Kd, Xd = torch.from_numpy(K).cuda(), torch.from_numpy(X).cuda()
+    for G in ((1, 8) if name != "cfg2" else (1,)):
+        with mcl.Mapper(0, stream=st.cuda_stream, rank=0, world=G) as m:
+            m.set_timing(True, hold_us=200); ts = []
+            for i in range(9):
+                flush.fill_(i); m.map_queues(Kd, Xd); ts.append(m.last_kernel_time_ms()[0])
+        out[f"{name}/G{G}"] = round(statistics.median(ts[2:]), 5)
+print(json.dumps(out))
+'''
+
+libs = sys.argv[1:3]
+rounds = int(sys.argv[3]) if len(sys.argv) > 3 else 3
+repo = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+for r in range(rounds):
+    for lib in (libs if r % 2 == 0 else libs[::-1]):
+        env = dict(os.environ, REPO=repo, LIB=os.path.abspath(lib))
+        res = subprocess.run([sys.executable, "-c", CHILD], env=env, capture_output=True, text=True)
+        line = res.stdout.strip().splitlines()[-1] if res.stdout.strip() else res.stderr[-400:]
+        print(json.dumps({"round": r, "lib": os.path.basename(lib), "result": line}), flush=True)

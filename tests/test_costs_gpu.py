@@ -126,3 +126,55 @@ def test_build_costs_many_tiles_long_lists_misaligned(torch_cuda, mapper):
     assert dm["kernel_ids"].data_ptr() % 16 == 4
     Kd, Xd = mapper.build_costs(dm, 4, device_out=True)
     assert (Kd.cpu().numpy() == want_k).all() and (Xd.cpu().numpy() == want_x).all()
+
+
+@pytest.mark.parametrize("E,Q,D,S", [(60, 8, 4, 2), (9, 5, 3, 3), (400, 2, 3, 2), (5, 12, 8, 4)])
+def test_build_costs_per_socket_curves(torch_cuda, mapper, E, Q, D, S):
+    """Per (socket, device) H2D / D2H curves and each queue's host socket (PAPER.md L897-901,
+    L1349-1361; reading R19): bit-exact against oracle/costs.c, host and device buffers."""
+    m = workloads.cost_model(7 * E + S, E, Q, D, sockets=S)
+    want_k, want_x = oracle.oracle_build_costs(Q, D, m)
+    K, X = mapper.build_costs(m, D)
+    assert (K == want_k).all() and (X == want_x).all()
+    Kd, Xd = mapper.build_costs(on_device(torch_cuda, m), D, device_out=True)
+    assert (Kd.cpu().numpy() == want_k).all() and (Xd.cpu().numpy() == want_x).all()
+    # the socket matters: every queue on socket 0 gives different (never larger) X here
+    m0 = dict(m, host_socket=np.zeros((E, Q), np.uint8))
+    _, X0 = mapper.build_costs(m0, D)
+    assert (X0 == oracle.oracle_build_costs(Q, D, m0)[1]).all() and (X0 <= X).all() and (X0 < X).any()
+    # a socket axis of one with no host_socket array is the plain model
+    m1 = dict(workloads.cost_model(5, E, Q, D))
+    m1s = dict(m1, h2d_bw=m1["h2d_bw"][None], d2h_bw=m1["d2h_bw"][None])
+    assert all((a == b).all() for a, b in zip(mapper.build_costs(m1s, D), oracle.oracle_build_costs(Q, D, m1)))
+    bad = dict(m, host_socket=np.full((E, Q), S, np.uint8))
+    with pytest.raises(MclError) as e:
+        mapper.build_costs(bad, D)
+    assert e.value.status == MCL_E_INVAL
+
+
+def test_build_costs_range_is_exact(torch_cuda, mapper):
+    """A profile entry of 2^48 (even never invoked) and a kernel sum reaching 2^48 are range
+    errors, like the oracle's running-sum check; a list of 70000 invocations (the checked
+    accumulation path) sums exactly, and 70000 x 2^47 -- which would wrap a u64 -- is a range
+    error, never a small wrapped cost."""
+    from paper_conf_cluster_ajipbf15_b200.mcl import MCL_E_RANGE
+
+    D = 3
+    base = dict(bytes=np.array([[4096, 1000]], np.uint64), source=np.array([[-1, 1]], np.int32),
+                cached=None, sizes=np.array([1024, 1 << 20], np.uint64), h2d_bw=np.full((D, 2), 4.0),
+                d2h_bw=np.full((D, 2), 2.0), host_shared=0)
+    prof = np.array([[1 << 47, 1, 1], [(1 << 47) - 1, 1, 1], [3, 5, 7]], np.uint64)
+    two = dict(base, profile=prof, offsets=np.array([0, 2, 2], np.uint64), kernel_ids=np.array([0, 1], np.uint32))
+    K, _ = mapper.build_costs(two, D)
+    assert int(K[0, 0, 0]) == (1 << 48) - 1 == int(oracle.oracle_build_costs(2, D, two)[0][0, 0, 0])
+    for bad in (dict(two, kernel_ids=np.array([0, 0], np.uint32)),
+                dict(two, profile=np.vstack([prof, [[1 << 48, 0, 0]]]).astype(np.uint64)),
+                dict(two, offsets=np.array([0, 70000, 70000], np.uint64), kernel_ids=np.zeros(70000, np.uint32))):
+        with pytest.raises(MclError) as e:
+            mapper.build_costs(bad, D)
+        assert e.value.status == MCL_E_RANGE
+    long_ok = dict(two, offsets=np.array([0, 70000, 70001], np.uint64),
+                   kernel_ids=np.concatenate([np.full(70000, 2, np.uint32), [1]]).astype(np.uint32))
+    K, X = mapper.build_costs(long_ok, D)
+    wk, wx = oracle.oracle_build_costs(2, D, long_ok)
+    assert (K == wk).all() and (X == wx).all() and int(K[0, 0, 2]) == 7 * 70000

@@ -491,3 +491,27 @@ def test_default_stream_follows_torch_current_stream(torch_cuda):
             i, mp, ms = m.map_queues(Kd, Xd)
     torch.cuda.synchronize()
     assert_same((i.cpu().numpy(), mp.cpu().numpy(), ms.cpu().numpy()), want, "torch stream order")
+
+
+@pytest.mark.parametrize("Q,D", [(15, 4), (10, 8)])
+def test_large_single_epoch_ties_and_shards(torch_cuda, mapper, Q, D):
+    """Single epochs of ~1e9 mappings spread over every CTA: random, tie-heavy and all-equal
+    tables, whole and in 3 shards, equal the oracle -- the CTA winner is the minimum holder
+    with the lowest block, the rescan is the one-pass pair scan, and the CTAs merge through
+    one packed per-epoch key (atomicMin) that the last CTA decodes and resets."""
+    torch = torch_cuda
+    cases = [workloads.random_tables(900 + Q, 1, Q, D, hi=1 << 20),
+             workloads.small_int_tables(901 + Q, 1, Q, D, hi=3)]
+    eq = np.full((1, Q, D), 11, np.uint64)
+    cases.append((eq, np.zeros_like(eq)))
+    nb = D ** (Q - 3)
+    for K, X in cases:
+        want = oracle.oracle_map(K, X)
+        assert_same(run_gpu(torch, mapper, K, X), want, f"{Q}x{D}")
+        Kd, Xd = to_dev(torch, K), to_dev(torch, X)
+        for r in range(3):
+            with Mapper(0, rank=r, world=3) as m:
+                i, _, ms = m.map_queues(Kd, Xd)
+            lo, hi = (nb * r // 3) * D**3, (nb * (r + 1) // 3) * D**3
+            oi, oms, _ = oracle.oracle_map(K, X, lo=lo, hi=hi)
+            assert (int(ms[0].item()), int(i[0].item())) == (int(oms[0]), int(oi[0])), f"{Q}x{D} shard {r}"
