@@ -229,6 +229,24 @@ def test_c_oracle_matches_definitional_oracle():
     assert n > 1000
 
 
+def test_c_oracle_matches_tiny_on_10k_instances():
+    """the C oracle equals tiny.py (itertools.product + min) on 10^4
+    random cfg1-sized instances (Q <= 4, D <= 3, up to 81 mappings), a third of them with
+    costs in {0, 1, 2} (heavy ties), all in one batched oracle call."""
+    rng = np.random.default_rng(10_000)
+    n = 0
+    for Q, D in ((4, 3), (3, 3), (4, 2), (2, 3)):
+        E = 2500
+        hi = np.where(np.arange(E) % 3 == 0, 3, 1 << 30)[:, None, None]
+        K = (rng.random((E, Q, D)) * hi).astype(np.uint64)
+        X = (rng.random((E, Q, D)) * hi).astype(np.uint64)
+        ci, cm, cp = oracle.oracle_map(K, X)
+        for e in range(E):
+            assert (int(ci[e]), int(cm[e]), tuple(cp[e])) == tiny_map(K[e], X[e]), (Q, D, e)
+            n += 1
+    assert n == 10_000
+
+
 def test_error_conventions():
     K = np.zeros((1, 3, 2), np.uint64)
     with pytest.raises(oracle.OracleError) as e:
