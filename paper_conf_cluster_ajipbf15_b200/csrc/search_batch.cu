@@ -29,6 +29,26 @@
 
 namespace mcl {
 
+#ifdef MCL_TRACE
+// Measurement build only (-DMCL_TRACE): per warp and unit (<= 8 units), %globaltimer at the
+// unit's start, after its tables, after the walk and after the finish, plus the SM id.
+__device__ unsigned long long g_mcl_btrace[4096 * 4][8][4];
+__device__ unsigned int g_mcl_bsm[4096 * 4];
+__device__ __forceinline__ unsigned long long btrace_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define MCL_BTRACE(unit, slot)                                                         \
+  do {                                                                                 \
+    if (lane == 0 && gw < 4096 * 4 && (unit) < 8) g_mcl_btrace[gw][unit][slot] = btrace_ns(); \
+  } while (0)
+#else
+#define MCL_BTRACE(unit, slot) \
+  do {                         \
+  } while (0)
+#endif
+
 namespace {
 
 template <int B, int E>
@@ -167,10 +187,19 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
   };
 
   int par = 0;
+#ifdef MCL_TRACE
+  if (lane == 0 && gw < 4096 * 4) {
+    unsigned int smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    g_mcl_bsm[gw] = smid;
+    for (int u = 0; u < 8; ++u) g_mcl_btrace[gw][u][0] = 0;
+  }
+#endif
   for (uint64_t i = 0;; ++i) {
     const uint64_t e = unit_epoch(i);
     if (e >= a.E) break;
     const bool whole = i < n_whole;
+    MCL_BTRACE(i, 0);
     // ---- a1: C = K + X, range check, bound UB = sum_q max_d C (decides 32-bit loads) ----
     bool bad = false;
     if (lane < QD) {
@@ -218,6 +247,7 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
         V[t] = (d == x) ? (T)C64[q * D + x] : T(0);
       }
       __syncwarp();
+      MCL_BTRACE(i, 1);
       // ---- a2-a5: each lane walks its share in increasing order, first strict minimum ----
       T best = ~T(0);
       uint32_t best_sb = 0xffffffffu;
@@ -250,9 +280,11 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
         }
       }
       key = warp_key(best, best_sb);
+      MCL_BTRACE(i, 2);
     }
     if (whole) {
       if (!skip) finish(e, key);
+      MCL_BTRACE(i, 3);
       continue;
     }
     // a split epoch: the CTA's warps merge their keys in shared memory; warp 0 finishes
@@ -265,8 +297,19 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
       finish(e, k);
     }
     par ^= 1;  // the next split epoch writes the other buffer (one barrier in between)
+    MCL_BTRACE(i, 3);
   }
 }
+
+#ifdef MCL_TRACE
+}  // namespace mcl
+extern "C" int mcl_btrace_read(unsigned long long* out, unsigned int* sm, int nwarps) {
+  cudaError_t e = cudaMemcpyFromSymbol(out, mcl::g_mcl_btrace, (size_t)nwarps * 8 * 4 * 8);
+  if (e == cudaSuccess) e = cudaMemcpyFromSymbol(sm, mcl::g_mcl_bsm, (size_t)nwarps * 4);
+  return (int)e;
+}
+namespace mcl {
+#endif
 
 namespace {
 template <int Q, int D>
