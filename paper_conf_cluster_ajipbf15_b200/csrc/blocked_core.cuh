@@ -33,6 +33,9 @@ namespace mcl {
 #define MCL_SUPER_MAX_D 5
 #endif
 constexpr int kSuperMaxD = MCL_SUPER_MAX_D;  // super-block path for u32 and D <= this
+#ifndef MCL_CHUNK_ODOMETER
+#define MCL_CHUNK_ODOMETER 1  // chunk prefixes by odometer steps (0: full decode per chunk)
+#endif
 
 namespace {
 
@@ -307,6 +310,39 @@ __device__ __forceinline__ void walk_blocks(const WalkCtx<T, D>& w, uint64_t b0,
       }
     };
     for (; nleft && (blk % chunk) != 0; ++blk, --nleft) single(blk);
+#if MCL_CHUNK_ODOMETER
+    // The chunk prefix (queues 0..O-3) is decoded once; consecutive chunks then step an
+    // odometer over those digits (kept in shared memory), updating the prefix by one-hot
+    // deltas: one digit changes per chunk, a carry every D chunks (lanes carry at different
+    // chunks: a short divergent step instead of a full decode per chunk).
+    T base2[D];
+    if (nleft >= chunk) {
+      uint64_t ch = blk / chunk;
+#pragma unroll
+      for (int d = 0; d < D; ++d) base2[d] = B0[d];
+      for (int q = O - 3; q >= 0; --q) {
+        const uint32_t dq = (uint32_t)(ch % D);
+        ch /= D;
+        dig[q * nthr + tid] = (uint8_t)dq;
+        const T* v = V + ((size_t)q * D + dq) * D;
+#pragma unroll
+        for (int d = 0; d < D; ++d) base2[d] = add_f(base2[d], v[d], one);
+      }
+    }
+    for (bool first = true; nleft >= chunk; nleft -= chunk, blk += chunk, first = false) {
+      if (!first) {
+        for (int q = O - 3; q >= 0; --q) {  // odometer step to this chunk
+          const uint32_t old = dig[q * nthr + tid];
+          const uint32_t nw = (old + 1 == (uint32_t)D) ? 0u : old + 1;
+          dig[q * nthr + tid] = (uint8_t)nw;
+          const T* vo = V + ((size_t)q * D + old) * D;
+          const T* vn = V + ((size_t)q * D + nw) * D;
+#pragma unroll
+          for (int d = 0; d < D; ++d) base2[d] = base2[d] - vo[d] + vn[d];
+          if (nw != 0) break;
+        }
+      }
+#else
     for (; nleft >= chunk; nleft -= chunk, blk += chunk) {
       uint64_t ch = blk / chunk;
       T base2[D];
@@ -319,6 +355,7 @@ __device__ __forceinline__ void walk_blocks(const WalkCtx<T, D>& w, uint64_t b0,
 #pragma unroll
         for (int d = 0; d < D; ++d) base2[d] = add_f(base2[d], v[d], one);
       }
+#endif
       for (int y = 0; y < D; ++y) {
         T base[D], vy[D];
         load_vec<T, D>(vy, Vy + y * D);

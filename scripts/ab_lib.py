@@ -1,6 +1,6 @@
 """A/B kernel timing of two builds of libmcl.so on one GPU (measurement only):
 
-    python scripts/ab_lib.py build/ab/libmcl_old.so build/ab/libmcl_new.so [rounds]
+    python scripts/ab_lib.py build/ab/libmcl_old.so build/ab/libmcl_new.so [more.so ...] [rounds]
 
 Each round runs every library in a fresh subprocess (alternating order) and prints the
 median kernel time (CUDA events, 200 us spin hold, L2 flushed) of the single-epoch configs
@@ -20,7 +20,7 @@ mcl.load_library(os.environ["LIB"])
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 st = torch.cuda.Stream(); torch.cuda.set_stream(st)
 out = {}
-for name in ("cfg5", "cfg4", "cfg2"):
+for name in os.environ.get("AB_WORKLOADS", "cfg5,cfg4,cfg2").split(","):
     K, X = workloads.make(name); Kd, Xd = torch.from_numpy(K).cuda(), torch.from_numpy(X).cuda()
     for G in ((1, 8) if name != "cfg2" else (1,)):
         with mcl.Mapper(0, stream=st.cuda_stream, rank=0, world=G) as m:
@@ -31,8 +31,9 @@ for name in ("cfg5", "cfg4", "cfg2"):
 print(json.dumps(out))
 '''
 
-libs = sys.argv[1:3]
-rounds = int(sys.argv[3]) if len(sys.argv) > 3 else 3
+args = sys.argv[1:]
+rounds = int(args.pop()) if args and args[-1].isdigit() else 3
+libs = args
 repo = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 for r in range(rounds):
     for lib in (libs if r % 2 == 0 else libs[::-1]):

@@ -1,0 +1,16 @@
+#!/bin/bash
+# ncu --set full captures (source-correlated) of the dominant kernels, one GPU:
+#   scripts/ncu_captures.sh [cfg5 cfg4 cfg2 cfg3 costs]   -> gpurun_out/prof_<wl>.ncu-rep
+cd "${GRAFT_REPO_ROOT:-$(dirname "$0")/..}"
+mkdir -p gpurun_out
+NCU=/usr/local/cuda/bin/ncu
+for wl in ${@:-cfg5 cfg4 cfg2 cfg3 costs}; do
+  if [ "$wl" = costs ]; then
+    timeout 900 $NCU --set full --clock-control none --import-source on -k regex:build_costs -s 2 -c 1 \
+        -o gpurun_out/prof_costs -f python scripts/profile_costs.py > gpurun_out/prof_costs.log 2>&1
+  else
+    timeout 900 $NCU --set full --clock-control none --import-source on -k regex:search_ -s 2 -c 1 \
+        -o gpurun_out/prof_$wl -f python scripts/profile_run.py $wl 3 > gpurun_out/prof_$wl.log 2>&1
+  fi
+  echo "$wl rc=$?"
+done

@@ -6,11 +6,11 @@ mkdir -p gpurun_out
 NCU=/usr/local/cuda/bin/ncu
 python scripts/probe_all.py > gpurun_out/probe_ops.txt 2>&1
 for wl in cfg5 cfg4 cfg2 cfg3 cfg1; do
-  timeout 600 python bench.py --workload $wl --steps 20 --warmup 5 > gpurun_out/bench_$wl.json 2> gpurun_out/bench_$wl.err
+  timeout 600 python bench.py --workload $wl --only --steps 20 --warmup 5 > gpurun_out/bench_$wl.json 2> gpurun_out/bench_$wl.err
 done
 for wl in cfg5 cfg4 cfg2 cfg3; do
   timeout 600 $NCU --metrics gpu__time_duration.sum --clock-control none --csv \
-      --log-file gpurun_out/launches_$wl.csv python bench.py --workload $wl --steps 2 --warmup 3 --no-cpu-baseline \
+      --log-file gpurun_out/launches_$wl.csv python bench.py --workload $wl --only --steps 2 --warmup 3 --no-cpu-baseline \
       > /dev/null 2>&1
   timeout 900 $NCU --set full --clock-control none --import-source on -k regex:search_ -s 2 -c 1 \
       -o gpurun_out/prof_$wl -f python scripts/profile_run.py $wl 3 > /dev/null 2>&1
