@@ -36,14 +36,14 @@ peak = hbm_peak()
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 with Mapper(0, stream=torch.cuda.current_stream().cuda_stream) as m:
     m.set_timing(True, hold_us=200)
-    for E, Q, D in ((100_000, 8, 4), (1_000_000, 2, 3)):
-        model = workloads.cost_model(42, E, Q, D)
+    for E, Q, D, S in ((100_000, 8, 4, 1), (1_000_000, 2, 3, 1), (100_000, 8, 4, 2)):
+        model = workloads.cost_model(42, E, Q, D, sockets=S)
         dm = {k: (torch.from_numpy(np.ascontiguousarray(v)).cuda() if isinstance(v, np.ndarray) else v)
               for k, v in model.items()}
         EQ = E * Q
         nnz = int(model["kernel_ids"].shape[0])
         # ids + offsets + bytes + source + cached in, K and X out
-        alg = 4 * nnz + 8 * (EQ + 1) + 8 * EQ + 4 * EQ + 2 * EQ + 2 * 8 * D * EQ
+        alg = 4 * nnz + 8 * (EQ + 1) + 8 * EQ + 4 * EQ + 2 * EQ + 2 * 8 * D * EQ + (EQ if S > 1 else 0)
         for _ in range(3):
             m.build_costs(dm, D, device_out=True)
         ks = []
@@ -53,7 +53,7 @@ with Mapper(0, stream=torch.cuda.current_stream().cuda_stream) as m:
             m.build_costs(dm, D, device_out=True)
             ks.append(m.last_kernel_time_ms()[0])
         k = statistics.median(ks)
-        print(json.dumps({"measure": "build_costs", "lib": args.lib or "in-tree", "E": E, "Q": Q, "D": D,
+        print(json.dumps({"measure": "build_costs", "lib": args.lib or "in-tree", "E": E, "Q": Q, "D": D, "sockets": S,
                           "invocations": nnz, "kernel_ms": k, "algorithmic_bytes": alg,
                           "GB_per_s": alg / (k / 1e3) / 1e9, "frac_of_hbm": alg / (k / 1e3) / 1e9 / peak,
                           "hbm_peak_gbs": peak}), flush=True)
