@@ -62,7 +62,7 @@ KERNEL_TIMING = ("CUDA events on the mapper's stream around the search launch, i
                  "launches right after the timed steps (L2 flushed before each, as there), each preceded "
                  "by a 200 us spin kernel so the events measure device execution; the timed steps record "
                  "no library events (one timing-event record costs ~2.7 us of host time, "
-                 "scripts/host_api_costs.cu, which the step would be charged)")
+                 "scripts/archive/host_api_costs.cu, which the step would be charged)")
 KERNEL_NAMES = {"blocked_u32": "search_blocked_kernel<u32, D>",
                 "blocked_u32_lean": "search_blocked_kernel<u32, 5, lean>",
                 "blocked_u64": "search_blocked_kernel<u64, D>",
@@ -559,7 +559,7 @@ def main():
     names = [args.workload] + ([] if args.only else [n for n in ALL_CONFIGS if n != args.workload])
     # Pinned host arena for the e2e legs, allocated first, in one piece, from the CPUs of the
     # GPU's NUMA node: on the pool's VMs later / separate pinned allocations copied at 14-47
-    # instead of 53 GB/s (scripts/e2e_dbg.py), which made the e2e time bimodal by process.
+    # instead of 53 GB/s (scripts/archive/e2e_dbg.py), which made the e2e time bimodal by process.
     prev_cpus = os.sched_getaffinity(0)
     ctx.local_cpus = gpu_local_cpus(ctx.dev_index)
     if ctx.local_cpus:

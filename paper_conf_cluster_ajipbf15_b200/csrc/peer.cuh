@@ -112,8 +112,8 @@ __device__ __forceinline__ uint64_t peer_take(const PeerArgs& p, uint64_t R, uin
 // the 64-bit rerun; then the whole exchange is skipped (identical on every rank, since all
 // ranks see the same inputs). Only GPU-scope ordering is needed up to here: the other CTAs'
 // keys (written by their thread 0) are read by this GPU's last CTA alone, so an acq_rel
-// counter increment replaces fences. Measured on one B200 (scripts/collective_compare.sh,
-// scripts/peer_tail_bench.cu): a system-scope fence per CTA plus a read of the host-mapped
+// counter increment replaces fences. Measured on one B200 (scripts/archive/collective_compare.sh,
+// scripts/archive/peer_tail_bench.cu): a system-scope fence per CTA plus a read of the host-mapped
 // status word made the tail ~17 us; as written it adds ~6 us to the search kernel at
 // world = 1 -- a chain of dependent memory round trips (round counter, keys, reduction,
 // fence, signal, poll, read-back, outputs), of which the counting and one round alone are

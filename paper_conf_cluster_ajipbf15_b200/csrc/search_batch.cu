@@ -327,7 +327,7 @@ cudaError_t launch_batch_t(const BatchArgs& a, int num_sms, cudaStream_t st, int
   }
   // one resident wave of warps; whole waves of epochs take one warp each, the epochs of
   // the last partial wave one CTA each (its warps split the super-blocks)
-  // (measured, scripts/batch_waves.py: splitting pays after at least one whole wave; a
+  // (measured, scripts/archive/batch_waves.py: splitting pays after at least one whole wave; a
   // batch below one wave runs one warp per epoch)
   const uint64_t ctas = (uint64_t)num_sms * per_sm;
   BatchArgs b = a;

@@ -258,7 +258,7 @@ cudaError_t launch_small_t(const SmallArgs& a, int num_sms, cudaStream_t st, int
     return cudaGetLastError();
   }
   // tile = one epoch per thread; tiny batches (cfg1: one epoch) get a single warp.
-  // Defaults from the cfg3 sweep (scripts/sweep_small.sh, profiles/r01/sweep_small.txt):
+  // Defaults from the cfg3 sweep (scripts/archive/sweep_small.sh, profiles/r01/sweep_small.txt):
   // 128-epoch tiles, 2 stages, 4 CTAs per SM (8 tiles in flight per SM) was fastest;
   // MCL_SMALL_{THREADS,STAGES,CTAS_PER_SM} override them for tuning.
   static const int kThreads = env_int("MCL_SMALL_THREADS", 128, 32, 256);

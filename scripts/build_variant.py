@@ -1,4 +1,4 @@
-"""Build a variant of libmcl.so for A/B timing (scripts/ab_kernel.py): the listed sources
+"""Build a variant of libmcl.so for A/B timing (scripts/ab_lib.py): the listed sources
 recompiled with extra nvcc flags (e.g. -DMCL_BATCH_MINB=3), linked with the in-tree objects.
 
     python scripts/build_variant.py ab/libmcl_v1.so search_batch.cu -DMCL_BATCH_MINB=3

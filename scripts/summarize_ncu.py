@@ -63,7 +63,7 @@ def main(tag, workloads):
     traffic = json.load(open(tpath)) if os.path.exists(tpath) else {}
     lines = [f"# ncu summary ({tag})", "",
              "`ncu --set full --clock-control none --import-source on` of one launch of the search kernel "
-             "(`scripts/profile.sh`), read back with `ncu -i ... --page raw --csv`. Cold-cache, serialised: "
+             "(`scripts/ncu_captures.sh`), read back with `ncu -i ... --page raw --csv`. Cold-cache, serialised: "
              "use shares and pipe utilisation, not absolute times.", ""]
     for wl in workloads:
         rep = os.path.join(ROOT, "gpurun_out", f"prof_{wl}.ncu-rep")
