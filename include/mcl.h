@@ -82,7 +82,8 @@ mcl_status_t mcl_mapper_create(const mcl_config_t* cfg, mcl_mapper_t** out);
  *   makespan      : [E] uint64 out: its makespan, in the same unit as the costs.
  * Every pointer may be device memory (the fast path: no copies) or host memory (pageable
  * or pinned; detected with cudaPointerGetAttributes and staged through handle-owned device
- * buffers inside the call). A pointer the CUDA runtime cannot classify is MCL_E_INVAL;
+ * buffers inside the call; a small call whose buffers are pinned host memory uses them in
+ * place, zero-copy over PCIe). A pointer the CUDA runtime cannot classify is MCL_E_INVAL;
  * pageable host pointers cannot be validated and are trusted, as with any C library taking
  * host buffers. The caller owns all buffers; the library never frees them.
  * Inputs are only read; outputs are fully written on MCL_OK and unspecified on error.

@@ -154,6 +154,7 @@ struct mcl_mapper {
   int force_path = 0;
   int pipeline_chunks = 0;      // 0 auto, 1 off, n forced (mcl_set_pipeline_chunks)
   bool async_call = false;      // pipelined chunk: enqueue only (the wrapper syncs, reads flags)
+  bool zero_copy = false;       // this call may use pinned host buffers in place (small call)
   // pipelined staging: pipe[0] host->device copies, pipe[1] the searches (one stream, so
   // chunk kernels never run concurrently and share the handle's scratch safely), pipe[2]
   // device->host copies; pipe_ev = start + per-stream join, chunk_ev = per-chunk hand-offs
@@ -184,8 +185,13 @@ mcl_status_t nccl_fail(mcl_mapper* h, ncclResult_t r, const char* what) {
     if (_e != cudaSuccess) return cuda_fail(h, _e, what); \
   } while (0)
 
-// Is `p` usable in place by kernels on h->device?
-mcl_status_t classify(mcl_mapper* h, const void* p, bool* on_device) {
+// Is `p` usable in place by kernels on h->device? *dptr receives the address kernels use.
+// Pinned (page-locked, mapped) host memory is used in place -- zero-copy over PCIe -- when
+// the call is small (h->zero_copy, set per call by map_impl): one launch that reads its
+// few hundred bytes of inputs and writes its outputs over the bus instead of 2 H2D + 3 D2H
+// copies, each a separate runtime call (cfg1 host-buffer call 36 -> ~16 us). Larger pinned
+// batches and pageable memory are staged (pipelined copy engines beat PCIe zero-copy there).
+mcl_status_t classify(mcl_mapper* h, const void* p, bool* on_device, const void** dptr = nullptr) {
   cudaPointerAttributes at;
   cudaError_t e = cudaPointerGetAttributes(&at, p);
   if (e != cudaSuccess) {  // CUDA >= 11 reports unregistered host memory as success
@@ -193,6 +199,7 @@ mcl_status_t classify(mcl_mapper* h, const void* p, bool* on_device) {
     h->last_err = std::string("cannot classify a buffer pointer: ") + cudaGetErrorString(e);
     return MCL_E_INVAL;
   }
+  if (dptr) *dptr = p;
   if (at.type == cudaMemoryTypeDevice) {
     if (at.device != h->device) {
       h->last_err = "device pointer belongs to another CUDA device";
@@ -201,8 +208,11 @@ mcl_status_t classify(mcl_mapper* h, const void* p, bool* on_device) {
     *on_device = true;
   } else if (at.type == cudaMemoryTypeManaged) {
     *on_device = true;
+  } else if (at.type == cudaMemoryTypeHost && h->zero_copy && at.devicePointer) {
+    *on_device = true;  // pinned host memory, small call: zero-copy
+    if (dptr) *dptr = at.devicePointer;
   } else {
-    *on_device = false;  // pageable or pinned host memory: staged
+    *on_device = false;  // pageable or (large call) pinned host memory: staged
   }
   return MCL_OK;
 }
@@ -414,9 +424,9 @@ namespace {
 
 // Stage a host buffer of `bytes` into `buf` (device pointers are used in place).
 mcl_status_t stage_in(mcl_mapper* h, DevBuf& buf, const void* src, size_t bytes, bool on_device,
-                      const void** out) {
+                      const void** out, const void* dsrc = nullptr) {
   if (on_device) {
-    *out = src;
+    *out = dsrc ? dsrc : src;
     return MCL_OK;
   }
   MCL_CUDA(h, buf.ensure(bytes), "cudaMalloc(staging)");
@@ -431,9 +441,10 @@ mcl_status_t classify_stage_in(mcl_mapper* h, DevBuf& buf, const void* src, size
   *out = nullptr;
   if (!src) return MCL_OK;
   bool on = false;
-  mcl_status_t st = classify(h, src, &on);
+  const void* d = nullptr;
+  mcl_status_t st = classify(h, src, &on, &d);
   if (st != MCL_OK) return st;
-  return stage_in(h, buf, src, bytes, on, out);
+  return stage_in(h, buf, src, bytes, on, out, d);
 }
 
 // Argument checks shared by the entry points: Q in [1, 32], D in [1, 16], and an epoch
@@ -472,13 +483,14 @@ mcl_status_t stage_outputs(mcl_mapper* h, uint64_t epochs, uint32_t Q, uint64_t*
   o->user_ms = makespan;
   o->user_map = mapping;
   bool di = true, dm = true, dmap = true;
+  const void *pi = index, *pm = makespan, *pmap = mapping;
   mcl_status_t st;
-  if (index && (st = classify(h, index, &di)) != MCL_OK) return st;
-  if ((st = classify(h, makespan, &dm)) != MCL_OK) return st;
-  if (mapping && (st = classify(h, mapping, &dmap)) != MCL_OK) return st;
-  o->idx = index;
-  o->ms = makespan;
-  o->map = mapping;
+  if (index && (st = classify(h, index, &di, &pi)) != MCL_OK) return st;
+  if ((st = classify(h, makespan, &dm, &pm)) != MCL_OK) return st;
+  if (mapping && (st = classify(h, mapping, &dmap, &pmap)) != MCL_OK) return st;
+  o->idx = (uint64_t*)pi;
+  o->ms = (uint64_t*)pm;
+  o->map = (uint8_t*)pmap;
   if (!di) {
     MCL_CUDA(h, h->out_idx.ensure(epochs * 8), "cudaMalloc(staging)");
     o->idx = (uint64_t*)h->out_idx.p;
@@ -687,6 +699,15 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
     return MCL_E_INVAL;
   }
   DeviceGuard g(h->device);
+  // small calls use pinned host buffers in place (zero-copy, see classify)
+  static const int kZeroCopyMax = mcl::env_int("MCL_ZERO_COPY_MAX", 64 << 10, 0, 1 << 30);
+  h->zero_copy = !h->async_call && h->pipeline_chunks <= 1 &&  // a forced pipeline is staged
+                 (uint64_t)epochs * ((uint64_t)Q * D * 16 + 16 + Q + (base_load ? D * 8 : 0) +
+                                     (eligible ? Q * 2 : 0)) <= (uint64_t)kZeroCopyMax;
+  struct ZeroCopyReset {  // the flag holds for this call only
+    mcl_mapper* h;
+    ~ZeroCopyReset() { h->zero_copy = false; }
+  } zc_reset{h};
   // With a communicator or imported peer slabs the call is collective (a 1-rank
   // communicator / slab set exercises the same exchange on a single GPU). The fused peer
   // exchange (NEXT-2) takes precedence over NCCL for the calls its slabs can hold.

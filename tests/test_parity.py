@@ -515,3 +515,33 @@ def test_large_single_epoch_ties_and_shards(torch_cuda, mapper, Q, D):
             lo, hi = (nb * r // 3) * D**3, (nb * (r + 1) // 3) * D**3
             oi, oms, _ = oracle.oracle_map(K, X, lo=lo, hi=hi)
             assert (int(ms[0].item()), int(i[0].item())) == (int(oms[0]), int(oi[0])), f"{Q}x{D} shard {r}"
+
+
+def test_small_pinned_calls_zero_copy(torch_cuda, mapper):
+    """Small calls whose buffers are all pinned host memory run the kernels on them in place
+    (zero-copy over PCIe, no staging copies): cfg1 decisions, a small batch, a constrained
+    call with pinned base loads and masks, and a pinned call too large for zero-copy (staged)
+    -- all equal the oracle."""
+    torch = torch_cuda
+
+    def pinned(a):
+        return torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
+
+    def outs(E, Q):
+        return (torch.empty(E, dtype=torch.uint64).pin_memory(), torch.empty((E, Q), dtype=torch.uint8).pin_memory(),
+                torch.empty(E, dtype=torch.uint64).pin_memory())
+
+    for name in workloads.NPB_RATIO:
+        K, X = workloads.cfg1_npb(name)
+        i, mp, ms = outs(1, 4)
+        mapper.map_queues_into(pinned(K), pinned(X), i, mp, ms)
+        assert_same((i.numpy(), mp.numpy(), ms.numpy()), oracle.oracle_map(K, X), name)
+    for (E, Q, D) in ((40, 6, 4), (3, 8, 4), (2000, 8, 4)):  # the last one is staged
+        K, X = workloads.random_tables(E + Q, E, Q, D)
+        i, mp, ms = outs(E, Q)
+        mapper.map_queues_into(pinned(K), pinned(X), i, mp, ms)
+        assert_same((i.numpy(), mp.numpy(), ms.numpy()), oracle.oracle_map(K, X), f"{E}x{Q}x{D}")
+    K, X = workloads.random_tables(77, 8, 7, 4)
+    base, elig = workloads.constraints(77, 8, 7, 4)
+    gi, gmp, gms = mapper.map_queues_constrained(pinned(K), pinned(X), pinned(base), pinned(elig))
+    assert_same((gi.numpy(), gmp.numpy(), gms.numpy()), oracle.oracle_map_constrained(K, X, base, elig), "constrained")
