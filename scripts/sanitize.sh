@@ -22,3 +22,9 @@ timeout 900 $CS --tool memcheck --error-exitcode 9 python -m pytest tests/test_p
 echo "memcheck pipeline rc=$? $(grep -E 'ERROR SUMMARY' gpurun_out/sanitize_memcheck_pipeline.log | tail -1) $(grep -E 'passed|failed' gpurun_out/sanitize_memcheck_pipeline.log | tail -1)"
 timeout 900 $CS --tool racecheck --error-exitcode 9 python -m pytest tests/test_pipeline_gpu.py -m gpu -q -p no:cacheprovider -k "share_scratch or chunks_cfg2" > gpurun_out/sanitize_racecheck_pipeline.log 2>&1
 echo "racecheck pipeline rc=$? $(grep -E 'RACECHECK SUMMARY' gpurun_out/sanitize_racecheck_pipeline.log | tail -1) $(grep -E 'passed|failed' gpurun_out/sanitize_racecheck_pipeline.log | tail -1)"
+# round-2 paths: mixed-radix constrained kernel, packed-key merge, static policy, sockets,
+# zero-copy small calls
+for tool in memcheck racecheck synccheck; do
+  timeout 1200 $CS --tool $tool --error-exitcode 9 python scripts/sanitize_cases.py > gpurun_out/sanitize_${tool}_r02.log 2>&1
+  echo "$tool r02 cases rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY' gpurun_out/sanitize_${tool}_r02.log | tail -1)"
+done

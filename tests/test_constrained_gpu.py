@@ -9,6 +9,7 @@ import oracle
 from conftest import cuda_available
 from paper_conf_cluster_ajipbf15_b200 import workloads
 from paper_conf_cluster_ajipbf15_b200.mcl import MCL_E_INVAL, MCL_E_RANGE, Mapper, MclError
+from shard_ranges import mixed_shard_ranges
 
 pytestmark = pytest.mark.gpu
 
@@ -73,42 +74,6 @@ def test_constrained_all_paths(torch_cuda, mapper, Q, D):
                 continue  # the mixed-radix kernel serves calls with eligible masks
             w = want if (b is base and el is elig) else oracle.oracle_map_constrained(K, X, b, el)
             check(run(torch_cuda, mapper, K, X, b, el, p), w, f"Q={Q} D={D} path={p}")
-
-
-def mixed_shard_ranges(elig_row, Q, D, G, wide=False):
-    """Full-index ranges [lo, hi) of the G shards of a masked single-epoch call
-    (include/mcl.h: the feasible enumeration cut into contiguous pieces). The mixed-radix
-    kernel's reduced space: pinned queues (one eligible device) leave it; the other queues
-    keep their order; blocks are the digits of all but the last three of them, each over
-    its eligible devices (for u32 with D <= 5 the last of those over all D devices); shard r
-    takes blocks [nb r / G, nb (r + 1) / G). A block's first leaf (inner digits 0) bounds
-    its full indices from below, so every feasible mapping of shard r lies in
-    [first(block lo), first(block hi))."""
-    full = (1 << D) - 1
-    masks = [(int(m) & full) if int(m) else full for m in elig_row]
-    devs = [[d for d in range(D) if (m >> d) & 1] for m in masks]
-    w = [D ** (Q - 1 - q) for q in range(Q)]
-    pinned = [q for q in range(Q) if len(devs[q]) == 1]
-    free = [q for q in range(Q) if len(devs[q]) != 1]
-    O = max(0, len(free) - 3)
-    outer = free[:O]
-    lists = [devs[q] for q in outer]
-    if not wide and D <= 5 and O >= 1:
-        lists[-1] = list(range(D))
-    nb = int(np.prod([len(x) for x in lists])) if lists else 1
-    pin_idx = sum(devs[q][0] * w[q] for q in pinned)
-
-    def first(b):
-        if b >= nb:
-            return D**Q
-        f = pin_idx
-        for p in range(O - 1, -1, -1):
-            r = len(lists[p])
-            f += lists[p][b % r] * w[outer[p]]
-            b //= r
-        return f
-
-    return [(first(nb * r // G), first(nb * (r + 1) // G)) for r in range(G)]
 
 
 def test_mixed_shard_ranges_helper():
