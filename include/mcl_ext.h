@@ -64,9 +64,11 @@ mcl_status_t mcl_force_path(mcl_mapper_t* h, int path);
    per SM), 1 = off, n > 1 = exactly min(n, epochs) chunks. With three or more chunks the
    first and the last hold half as many epochs as the others (a short first copy before the
    first search, a short search after the last copy). mcl_last_launch_info's info[7] is the
-   number of chunks of a pipelined call (0 otherwise). Small calls whose buffers are all
-   pinned host memory skip staging altogether (the kernels use them in place, zero-copy;
-   MCL_ZERO_COPY_MAX bytes, default 64 KiB) unless n > 1 forces the pipeline.
+   number of chunks of a pipelined call (0 otherwise). Calls whose buffers are pinned host
+   memory skip staging altogether when they are small (MCL_ZERO_COPY_MAX bytes, default
+   64 KiB) or run the warp-per-epoch batch kernel (which reads each epoch's costs one epoch
+   ahead, so PCIe reads overlap the search): the kernels use them in place, zero-copy --
+   unless n > 1 forces the pipeline.
    Errors: MCL_E_INVAL (NULL h, n < 0). */
 mcl_status_t mcl_set_pipeline_chunks(mcl_mapper_t* h, int chunks);
 

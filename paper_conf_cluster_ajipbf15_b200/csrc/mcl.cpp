@@ -699,11 +699,19 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
     return MCL_E_INVAL;
   }
   DeviceGuard g(h->device);
-  // small calls use pinned host buffers in place (zero-copy, see classify)
+  // Pinned host buffers are used in place (zero-copy, see classify) by small calls, and by
+  // the warp-per-epoch batch kernel, which loads each epoch's costs one epoch ahead -- its
+  // PCIe reads then overlap the search (cfg2 from pinned buffers: 0.142 ms zero-copy vs
+  // 0.183 ms with pipelined staging; cfg3's thread-per-epoch kernel is PCIe-bound either
+  // way, 1.94 vs 1.91 ms, and keeps the pipeline; profiles/r02/e2e_study.jsonl).
   static const int kZeroCopyMax = mcl::env_int("MCL_ZERO_COPY_MAX", 64 << 10, 0, 1 << 30);
+  const bool batch_path = !base_load && !eligible && h->comm == nullptr && !h->peer_ready &&
+                          h->world <= 1 && mcl::batch_supported(Q, D) &&
+                          epochs >= (uint64_t)h->num_sms * 4 && (h->force_path == 0 || h->force_path == 7);
   h->zero_copy = !h->async_call && h->pipeline_chunks <= 1 &&  // a forced pipeline is staged
-                 (uint64_t)epochs * ((uint64_t)Q * D * 16 + 16 + Q + (base_load ? D * 8 : 0) +
-                                     (eligible ? Q * 2 : 0)) <= (uint64_t)kZeroCopyMax;
+                 (batch_path ||
+                  (uint64_t)epochs * ((uint64_t)Q * D * 16 + 16 + Q + (base_load ? D * 8 : 0) +
+                                      (eligible ? Q * 2 : 0)) <= (uint64_t)kZeroCopyMax);
   struct ZeroCopyReset {  // the flag holds for this call only
     mcl_mapper* h;
     ~ZeroCopyReset() { h->zero_copy = false; }

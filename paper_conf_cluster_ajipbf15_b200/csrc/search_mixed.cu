@@ -189,6 +189,7 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1) searc
   __shared__ MixedTab mt;
   __shared__ uint32_t s_status;
   __shared__ uint64_t s_ub, s_feas;
+  __shared__ uint64_t s_ubr;  // bound of the reduced problem (decides u32 vs u64)
   __shared__ uint64_t s_base[D];
   __shared__ __align__(16) T base0[D];
   __shared__ uint64_t s_gmin;
@@ -295,11 +296,11 @@ __global__ void __launch_bounds__(256, (sizeof(T) == 4 && D <= 5) ? 2 : 1) searc
         // bound of every leaf the kernel forms: max base' + sum of the reduced rows' maxima
         uint64_t bm = 0;
         for (uint32_t d = 0; d < D; ++d) bm = max(bm, s_base[d]);
-        s_ub = bm + rm;
+        s_ubr = bm + rm;  // not s_ub: every thread reads s_ub above, with no barrier between
       }
     }
     __syncthreads();
-    if (sizeof(T) == 4 && s_ub >= 0xffffffffull) {  // UB < 2^32 - 1 for 32-bit loads
+    if (sizeof(T) == 4 && s_ubr >= 0xffffffffull) {  // UB < 2^32 - 1 for 32-bit loads
       if (tid == 0 && part == 0) raise_flag(a.flags, kFlagNeedU64);
       abandoned = true;
       continue;

@@ -84,19 +84,23 @@ def test_pipelined_small_kernel_and_pageable(torch_cuda, mapper):
 
 
 def test_pipelined_auto_matches_unpipelined(torch_cuda, mapper):
-    """The automatic chunking of a full cfg2 batch (4 chunks of one wave or more) and the
-    unpipelined staged call return identical outputs; no mapping output (NULL) works."""
+    """The automatic chunking of a full cfg2 batch from pageable buffers (4 chunks of one
+    wave or more), the unpipelined staged call, and the zero-copy call from pinned buffers
+    (the warp-per-epoch kernel reads them in place) return identical outputs; no mapping
+    output (NULL) works."""
     K, X = workloads.cfg2()
-    got_auto = host_call(torch_cuda, mapper, K, X)
+    got_auto = host_call(torch_cuda, mapper, K, X, pinned=False)
     assert mapper.launch_info()["chunks"] > 1
     mapper.set_pipeline_chunks(1)
     try:
-        got_off = host_call(torch_cuda, mapper, K, X)
+        got_off = host_call(torch_cuda, mapper, K, X, pinned=False)
         assert mapper.launch_info()["chunks"] == 0
     finally:
         mapper.set_pipeline_chunks(0)
-    for a, b in zip(got_auto, got_off):
-        assert (a == b).all()
+    got_zc = host_call(torch_cuda, mapper, K, X, pinned=True)
+    assert mapper.launch_info()["chunks"] == 0 and mapper.launch_info()["path"] == "batch_u32"
+    for a, b, c in zip(got_auto, got_off, got_zc):
+        assert (a == b).all() and (a == c).all()
     check(got_auto, oracle.oracle_map(K, X), "cfg2 auto")
     gi, _, gms = host_call(torch_cuda, mapper, K, X, with_mapping=False)
     assert (gi == got_auto[0]).all() and (gms == got_auto[2]).all()
