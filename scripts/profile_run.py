@@ -12,10 +12,20 @@ reps = int(sys.argv[2]) if len(sys.argv) > 2 else 3
 kw = {}
 if len(sys.argv) > 3:  # optional epochs override for batched configs (sanitizer runs)
     kw["E"] = int(sys.argv[3])
-K, X = workloads.make(name, **kw)
+constrained = name.endswith("c")  # e.g. cfg5c: cfg5 with 3 pinned + 3 masked queues (NEXT-3)
+K, X = workloads.make(name.rstrip("c"), **kw)
 Kd, Xd = torch.from_numpy(K).cuda(), torch.from_numpy(X).cuda()
+if constrained:
+    base, elig = workloads.constraints(77, *K.shape)
+    elig[:] = 0
+    elig[:, [1, 5, 10]] = [1 << 3, 1 << 0, 1 << 6]
+    elig[:, [2, 7, 11]] = [0b00110110, 0b11000001, 0b0111]
+    Bd, Ed = torch.from_numpy(base).cuda(), torch.from_numpy(elig).cuda()
 with Mapper(0) as m:
     for _ in range(reps):
-        idx, mp, ms = m.map_queues(Kd, Xd)
+        if constrained:
+            idx, mp, ms = m.map_queues_constrained(Kd, Xd, Bd, Ed)
+        else:
+            idx, mp, ms = m.map_queues(Kd, Xd)
     torch.cuda.synchronize()
     print(name, m.launch_info(), int(idx[0]), int(ms[0]))

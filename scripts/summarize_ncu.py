@@ -35,6 +35,8 @@ METRICS = [
     ("sm__throughput.avg.pct_of_peak_sustained_elapsed", "SM throughput % peak"),
 ]
 MAPPINGS = {"cfg1": 81, "cfg2": 10_000 * 4**8, "cfg3": 10**6 * 9, "cfg4": 4**16, "cfg5": 8**12}
+# cfg5c (3 pinned + 3 masked queues, NEXT-3): thread instructions per FEASIBLE mapping
+MAPPINGS["cfg5c"] = 9_437_184
 
 
 def raw(rep):
@@ -92,4 +94,4 @@ def main(tag, workloads):
 
 
 if __name__ == "__main__":
-    main(sys.argv[1], sys.argv[2:] or ["cfg5", "cfg4", "cfg2", "cfg3", "costs"])
+    main(sys.argv[1], sys.argv[2:] or ["cfg5", "cfg4", "cfg2", "cfg3", "costs", "cfg5c"])
