@@ -323,3 +323,17 @@ def test_static_policy_baseline(torch_cuda, mapper):
         mapper.static_mappings(np.full((1, Q), 3, np.uint8), score)  # hint >= classes
     with pytest.raises(MclError):
         mapper.static_mappings(hints[:1], score, np.full((1, Q), 1 << 15, np.uint16))  # no device
+
+
+@pytest.mark.parametrize("D", [6, 7, 8])
+def test_mixed_radix_u64_wide_devices(torch_cuda, mapper, D):
+    """64-bit loads on the mixed-radix kernel for D = 6..8 (the builds with register
+    spills): base loads near 2^40 force the rerun; every epoch equals the oracle."""
+    torch = torch_cuda
+    Q = 6
+    K, X = workloads.random_tables(90 + D, 12, Q, D, hi=1 << 20)
+    base, elig = random_constraints(91 + D, 12, Q, D, pin_frac=0.3)
+    big = base + np.uint64(1 << 40)
+    want = oracle.oracle_map_constrained(K, X, big, elig)
+    check(run(torch, mapper, K, X, big, elig), want, f"u64 D={D}")
+    assert mapper.launch_info()["path"] == "mixed_u64"

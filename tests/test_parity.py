@@ -415,6 +415,16 @@ def test_nccl_single_rank_collective_path(torch_cuda):
             got = m.map_queues(to_dev(torch, K), to_dev(torch, X))
             assert m.launch_info()["two_step"]
             assert_same(tuple(t.cpu().numpy() for t in got), oracle.oracle_map(K, X), "two-step")
+            # masked calls (mixed-radix kernel) through the same sequence, device and pinned
+            K, X = workloads.cfg4(seed=5, Q=11)
+            base, elig = workloads.constraints(12, 1, 11, 4)
+            want = oracle.oracle_map_constrained(K, X, base, elig)
+            got = m.map_queues_constrained(to_dev(torch, K), to_dev(torch, X), to_dev(torch, base), to_dev(torch, elig))
+            assert m.launch_info()["allreduce"] and m.launch_info()["path"] == "mixed_u32"
+            assert_same(tuple(t.cpu().numpy() for t in got), want, "constrained nccl")
+            pin = [torch.from_numpy(a).pin_memory() for a in (K, X, base, elig)]
+            got = m.map_queues_constrained(*pin)
+            assert_same(tuple(t.numpy() for t in got), want, "constrained nccl pinned")
     finally:
         mcl.mcl_comm_destroy(comm)
 

@@ -96,6 +96,18 @@ def test_fused_exchange_errors(torch_cuda):
         K, X = workloads.cfg1_npb("FT")
         i, mp, ms = m.map_queues(K, X)
         assert int(i[0]) == int(oracle.oracle_map(K, X)[0][0])
+        # pinned host buffers of a small call are used in place (zero-copy) by the search
+        # kernel and its in-kernel exchange / decode
+        import torch
+
+        Kp, Xp = torch.from_numpy(K).pin_memory(), torch.from_numpy(X).pin_memory()
+        ip = torch.empty(1, dtype=torch.uint64).pin_memory()
+        mp_ = torch.empty((1, 4), dtype=torch.uint8).pin_memory()
+        msp = torch.empty(1, dtype=torch.uint64).pin_memory()
+        m.map_queues_into(Kp, Xp, ip, mp_, msp)
+        want = oracle.oracle_map(K, X)
+        assert m.launch_info()["fused_exchange"]
+        assert int(ip[0]) == int(want[0][0]) and int(msp[0]) == int(want[1][0]) and (mp_.numpy() == want[2]).all()
 
 
 def _free_port():
