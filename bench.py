@@ -87,6 +87,8 @@ def parse(argv=None):
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="CPU-oracle sample budget (headline)")
     p.add_argument("--config-cpu-seconds", type=float, default=2.5,
                    help="CPU-oracle sample budget per other config and thread count")
+    p.add_argument("--ref-step-seconds", type=float, default=None,
+                   help="reference arm: oracle seconds per step (default: ~150 s over all steps, 2-20 s each)")
     p.add_argument("--collective", default="auto", choices=["auto", "fused", "nccl"],
                    help="cross-GPU combine of a sharded single-epoch search: fused = in-kernel "
                         "exchange over peer memory (NEXT-2), nccl = ncclAllReduce + decode kernel; "
@@ -253,7 +255,7 @@ def reference_arm(args, rank):
     K, X, w = workload(args.workload)
     threads = oracle.default_threads()
     total = args.steps + args.warmup
-    per_step = max(2.0, min(20.0, 150.0 / max(1, total)))
+    per_step = args.ref_step_seconds or max(2.0, min(20.0, 150.0 / max(1, total)))
     rate, _, _, _ = oracle_sample(K, X, w, 1.0, threads)  # calibration
     n = max(1 << 20, int(rate * per_step))
     tiny = w["E"] == 1 and w["N"] < (1 << 16)
