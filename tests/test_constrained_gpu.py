@@ -337,3 +337,15 @@ def test_mixed_radix_u64_wide_devices(torch_cuda, mapper, D):
     want = oracle.oracle_map_constrained(K, X, big, elig)
     check(run(torch, mapper, K, X, big, elig), want, f"u64 D={D}")
     assert mapper.launch_info()["path"] == "mixed_u64"
+
+
+def test_mixed_radix_batches_beyond_one_wave(torch_cuda, mapper):
+    """Batches larger than one wave of CTAs (whole-CTA epochs, then the tail epochs split over
+    several CTAs merged through scratch) on the mixed-radix kernel == the oracle."""
+    torch = torch_cuda
+    E, Q, D = 700, 7, 4
+    K, X = workloads.random_tables(123, E, Q, D, hi=1 << 18)
+    base, elig = random_constraints(124, E, Q, D, pin_frac=0.3)
+    want = oracle.oracle_map_constrained(K, X, base, elig)
+    check(run(torch, mapper, K, X, base, elig), want, "mixed E=700")
+    assert mapper.launch_info()["path"] == "mixed_u32"

@@ -134,6 +134,13 @@ def _rank(rank, world, port, q):
                 i, mp, ms = m.map_queues(dev(torch, K), dev(torch, X))
                 out.append((name, i.cpu().numpy(), ms.cpu().numpy(), mp.cpu().numpy(),
                             m.launch_info()["fused_exchange"]))
+            # masked calls: each rank searches its piece of the FEASIBLE enumeration
+            # (mixed-radix kernel) and the fused exchange combines them
+            Kc, Xc = workloads.cfg4(seed=6, Q=11)
+            bc, ec = workloads.constraints(21, 1, 11, 4)
+            i, mp, ms = m.map_queues_constrained(dev(torch, Kc), dev(torch, Xc), dev(torch, bc), dev(torch, ec))
+            out.append(("constrained", i.cpu().numpy(), ms.cpu().numpy(), mp.cpu().numpy(),
+                        m.launch_info()["fused_exchange"] and m.launch_info()["path"] == "mixed_u32"))
             # more epochs than the slabs hold and no communicator: an error, never this
             # rank's shard-local argmin presented as the global result
             K, X = workloads.small_int_tables(8, 64, 7, 3, hi=4)
@@ -167,6 +174,9 @@ def test_fused_exchange_two_ranks_one_gpu(torch_cuda):
         pytest.skip(f"CUDA IPC between two processes on one device unavailable: {errs[0]}")
     assert not errs, errs
     want = {name: oracle.oracle_map(K, X) for name, K, X in _cases() if K.shape[0] <= 8}
+    Kc, Xc = workloads.cfg4(seed=6, Q=11)
+    bc, ec = workloads.constraints(21, 1, 11, 4)
+    want["constrained"] = oracle.oracle_map_constrained(Kc, Xc, bc, ec)
     from paper_conf_cluster_ajipbf15_b200.mcl import MCL_E_INVAL
 
     for rank, out, _ in res:
