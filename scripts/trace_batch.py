@@ -58,7 +58,13 @@ for w in range(nw):
 ends = np.array(ends) / 1e3
 span = ends.max()
 hist = [int((ends > x).sum()) for x in np.arange(0, span + 5, 5)]
+by_unit = {}
+for u in range(5):
+    w = [(t[x, u, 2] - t[x, u, 1]) / 1e3 for x in range(nw) if valid[x, u] and t[x, u, 2] > 0]
+    if w:
+        by_unit[u] = [float(np.percentile(w, 10)), float(np.median(w)), float(np.percentile(w, 90))]
 print(json.dumps({
+    "walk_us_by_unit_p10_p50_p90": by_unit,
     "E": E, "env": {k: v for k, v in os.environ.items() if k.startswith("MCL_")}, "warps": nw, "kernel_span_us": float(span), "first_start_spread_us": float(np.max(starts) / 1e3),
     "setup_us_median": float(np.median(setup) / 1e3), "walk_us_median": float(np.median(walk) / 1e3),
     "walk_us_p10_p90": [float(np.percentile(walk, 10) / 1e3), float(np.percentile(walk, 90) / 1e3)],
