@@ -5,6 +5,11 @@
  * 100 ns on either GPU; EP goes to the GPUs): optimum (1, 1, 2, 2),
  * index 44, makespan 200. Epoch 1 is case F ("BT-like", [100, 350, 350] per queue; mostly
  * CPU, L1800-1807): (0, 0, 0, 1), index 1, makespan 350.
+ * Then, on epoch 0: queue 0 pinned to the CPU (a SCHED_OFF queue, L838-845): the CPU carries
+ * 2000 ns whatever the others do, so the optimum is 2000 and its lowest index keeps the other
+ * queues off the CPU: (0, 1, 1, 1), index 13. And the SCHED_AUTO_STATIC policy (L1088-1116)
+ * with every queue hinted compute-bound and a device profile favouring the GPUs equally sends
+ * all four to GPU0 -- makespan 400, twice the optimum.
  *
  *   gcc -O2 -I include examples/map_queues.c -L paper_conf_cluster_ajipbf15_b200 -lmcl \
  *       -Wl,-rpath,$PWD/paper_conf_cluster_ajipbf15_b200 -o /tmp/map_queues
@@ -50,6 +55,24 @@ int main(void) {
     printf("\n");
     ok &= index[e] == want_index[e] && makespan[e] == want_ms[e];
   }
+  /* constrained: queue 0 pinned to the CPU (one-bit eligible mask), the others free */
+  uint16_t elig[Q] = {0x1, 0, 0, 0};
+  mcl_constraints_t cons = {NULL, elig};
+  uint64_t ci, cms;
+  uint8_t cmap[Q];
+  st = mcl_map_queues_constrained(h, Q, D, 1, &K[0][0][0], &X[0][0][0], &cons, &ci, cmap, &cms);
+  printf("pinned queue 0: %s index %llu makespan %llu mapping %u %u %u %u\n", mcl_status_string(st),
+         (unsigned long long)ci, (unsigned long long)cms, cmap[0], cmap[1], cmap[2], cmap[3]);
+  ok &= st == MCL_OK && ci == 13 && cms == 2000;
+  /* static hint policy vs the optimum: every queue compute-bound; class cost CPU 4, GPUs 1 */
+  uint8_t hints[Q] = {0, 0, 0, 0}, smap[Q];
+  const uint64_t score[1][D] = {{4, 1, 1}};
+  uint64_t sms;
+  st = mcl_static_mappings(h, Q, D, 1, hints, 1, &score[0][0], NULL, smap);
+  if (st == MCL_OK) st = mcl_score_mappings(h, Q, D, 1, &K[0][0][0], &X[0][0][0], NULL, smap, &sms);
+  printf("static policy: %s mapping %u %u %u %u makespan %llu\n", mcl_status_string(st), smap[0], smap[1],
+         smap[2], smap[3], (unsigned long long)sms);
+  ok &= st == MCL_OK && sms == 400 && smap[0] == 1 && smap[3] == 1;
   /* an entry >= 2^48 is a range error, reported, not silently wrapped */
   K[1][2][1] = (uint64_t)1 << 48;
   st = mcl_map_queues(h, Q, D, E, &K[0][0][0], &X[0][0][0], index, NULL, makespan);

@@ -1,6 +1,7 @@
 """The C ABI from plain C: examples/map_queues.c compiles against include/mcl.h and
 libmcl.so alone (CPU test), and on a GPU returns the hand-solved optima of DESIGN.md
-Appendix A cases E and F and reports a 2^48 entry as MCL_E_RANGE (GPU test)."""
+Appendix A cases E and F, the hand-solved constrained optimum with a pinned queue, the static
+policy's mapping and makespan, and reports a 2^48 entry as MCL_E_RANGE (GPU test)."""
 from __future__ import annotations
 
 import os
@@ -37,5 +38,7 @@ def test_c_example_runs(tmp_path):
     assert r.returncode == 0, r.stdout + r.stderr
     assert "epoch 0: index 44 makespan 200 mapping 1 1 2 2" in r.stdout
     assert "epoch 1: index 1 makespan 350 mapping 0 0 0 1" in r.stdout
+    assert "pinned queue 0: MCL_OK: success index 13 makespan 2000 mapping 0 1 1 1" in r.stdout
+    assert "static policy: MCL_OK: success mapping 1 1 1 1 makespan 400" in r.stdout
     assert "entry 2^48: MCL_E_RANGE" in r.stdout
     assert r.stdout.strip().endswith("OK")
