@@ -307,6 +307,7 @@ class Ctx:
         self.dist = None
         self.comm = None
         self.arena = None
+        self.fused_failed = False  # the fused exchange failed once: NCCL for the rest of the run
 
 
 def max_over_ranks(ctx, values):
@@ -420,17 +421,37 @@ def measure(ctx, name):
     mapper = Mapper(dev_index, stream=stream.cuda_stream, nccl_comm=comm,
                     rank=rank if sharded else 0, world=world if sharded else 1)
     combine = "nccl" if comm else "none"
-    if sharded and args.collective != "nccl":
-        # fused in-kernel exchange over NVLink peer memory (agreed by all ranks)
+    if sharded and args.collective != "nccl" and not ctx.fused_failed:
+        # fused in-kernel exchange over NVLink peer memory, validated by one sharded call
+        # against the same call's answer on a single GPU; all ranks agree (gloo) -- if any
+        # rank cannot map the slabs or the exchange fails, every rank falls back to an NCCL
+        # communicator instead of failing the run
+        ok = 1
         try:
-            mapper.connect_peers(max_epochs=1, timeout_ms=60_000)
-            ok = 1
+            mapper.connect_peers(max_epochs=1, timeout_ms=20_000)
+            Kv, Xv = Kd[:1], Xd[:1]
+            vi, _, vm = mapper.map_queues(Kv, Xv, with_mapping=False)
+            with Mapper(dev_index, stream=stream.cuda_stream) as solo:
+                si, _, sm = solo.map_queues(Kv, Xv, with_mapping=False)
+            ok = int(bool((vi == si).all() and (vm == sm).all()))
         except Exception as exc:  # pragma: no cover
             print(f"[bench] fused exchange unavailable ({exc})", file=sys.stderr)
             ok = 0
         if -max_over_ranks(ctx, [-ok])[0] < 1:  # min over ranks
-            raise SystemExit("[bench] fused exchange unavailable on some rank; rerun with --collective nccl")
-        combine = "fused"
+            print("[bench] fused exchange unusable on some rank: NCCL communicator instead", file=sys.stderr)
+            ctx.fused_failed = True
+            mapper.close()
+        else:
+            combine = "fused"
+    if sharded and combine == "none":  # --collective nccl, or the fused exchange's fallback
+        if ctx.comm is None:
+            obj = [mcl.mcl_comm_unique_id() if rank == 0 else None]
+            ctx.dist.broadcast_object_list(obj, src=0)
+            ctx.comm = mcl.mcl_comm_init(dev_index, world, rank, obj[0])
+        if mapper.handle:
+            mapper.close()
+        mapper = Mapper(dev_index, stream=stream.cuda_stream, nccl_comm=ctx.comm, rank=rank, world=world)
+        combine = "nccl"
     mapper.set_timing(False)
 
     for _ in range(max(3, args.warmup)):
