@@ -4,21 +4,24 @@
 // a = Q-3, b = Q-2, c = Q-1 (digits i, j, k) vary inside a block, the outer Q-3 digits are
 // fixed and give the prefix load vector P[d] (queues on one device
 // serialise, devices run concurrently). With M = max_d P[d] and every cost >= 0, the
-// makespan of leaf (i, j, k) is max(M, load of each device the inner queues touch), which
-// the compiler-unrolled leaf table below forms with ONE integer max per mapping:
+// makespan of leaf (i, j, k) is max(M, v) with v the largest load of the devices the inner
+// queues touch, which the compiler-unrolled leaf table below forms with at most ONE integer
+// max per mapping:
 //
-//   i, j, k distinct : max3(P_i+A_i, P_j+B_j, max(M, P_k+C_k))
-//   i == j != k      : max (P_i+A_i+B_i, max(M, P_k+C_k))
-//   i == k != j      : max3(P_i+A_i+C_i, P_j+B_j, M)
-//   j == k != i      : max3(P_i+A_i, P_j+B_j+C_j, M)
-//   i == j == k      : max (M, P_i+A_i+B_i+C_i)
+//   i, j, k distinct : v = max3(P_i+A_i, P_j+B_j, P_k+C_k)
+//   i == j != k      : v = max (P_i+A_i+B_i, P_k+C_k)
+//   i == k != j      : v = max (P_i+A_i+C_i, P_j+B_j)
+//   j == k != i      : v = max (P_i+A_i, P_j+B_j+C_j)
+//   i == j == k      : v = P_i+A_i+B_i+C_i            (no instruction)
 //
 // (A, B, C = the composed cost rows C[q][.] = K + X of queues a, b, c.)
-// Every leaf's makespan is formed explicitly in a register; the argmin is folded with the
-// sm_100a three-input minimum (VIMNMX3: two mappings per ALU instruction), so the floor is
-// 1.5 ALU instructions per mapping. The block minimum is compared
-// with the thread's running best (strict <, blocks visited in increasing index order);
-// only the best block (or super-block) is re-scanned at the end for the lowest leaf index.
+// Because max(M, .) is non-decreasing, the block minimum of the makespans is max(M, min v):
+// M is applied once per block, not per leaf. The minimum is folded with the sm_100a
+// three-input minimum (VIMNMX3: two leaves per ALU instruction), so the floor is
+// 1.5 - 1/D^2 ALU instructions per mapping. The block minimum is
+// compared with the thread's running best (strict <, blocks visited in increasing index
+// order); only the best block (or super-block) is re-scanned at the end for the lowest
+// leaf index, from the definition.
 //
 // The outer digits walk an odometer: digit x (queue Q-4) is the block loop, the digits of
 // queues 0..Q-5 live in shared memory and update the base load vector by one-hot vectors
@@ -90,10 +93,35 @@ __device__ __forceinline__ T max_of(const T (&P)[D]) {
   return M;
 }
 
-// Enumerate the D^3 leaves of one block in increasing index order, calling f(leaf, ms).
-// M = max_d P[d] (prefix makespan).
+#ifndef MCL_LEAF_M_AFTER
+#define MCL_LEAF_M_AFTER 1  // apply the prefix makespan M once per block (0: in every leaf)
+#endif
+
+// Enumerate the D^3 leaves of one block in increasing index order, calling f(leaf, v).
+// M = max_d P[d] (prefix makespan). With MCL_LEAF_M_AFTER, v is the maximum load of the
+// devices the leaf's three inner queues touch, and the leaf's makespan is max(M, v); as
+// max(M, .) is non-decreasing, min over the leaves of max(M, v) = max(M, min v), so the
+// block applies M once to its minimum instead of once per leaf (no M in the leaf table:
+// D fewer maxima per block for the max(M, C_k) terms, and the D diagonal leaves i == j == k
+// need none at all). Otherwise v is the makespan itself.
 template <typename T, int D, typename F>
 __device__ __forceinline__ void for_each_leaf(const Sums<T, D>& s, T M, F&& f) {
+#if MCL_LEAF_M_AFTER
+#pragma unroll
+  for (int i = 0; i < D; ++i)
+#pragma unroll
+    for (int j = 0; j < D; ++j)
+#pragma unroll
+      for (int k = 0; k < D; ++k) {
+        T v;
+        if (i != j && i != k && j != k) v = max3(s.a[i], s.b[j], s.c[k]);
+        else if (i == j && j != k) v = max2(s.ab[i], s.c[k]);
+        else if (i == k && i != j) v = max2(s.ac[i], s.b[j]);
+        else if (j == k && i != j) v = max2(s.a[i], s.bc[j]);
+        else v = s.abc[i];
+        f((i * D + j) * D + k, v);
+      }
+#else
   T PCM[D];
 #pragma unroll
   for (int d = 0; d < D; ++d) PCM[d] = max2(M, s.c[d]);
@@ -111,6 +139,7 @@ __device__ __forceinline__ void for_each_leaf(const Sums<T, D>& s, T M, F&& f) {
         else v = max2(M, s.abc[i]);
         f((i * D + j) * D + k, v);
       }
+#endif
 }
 
 // Fold one block's leaves into a running 4-way minimum, two leaves per three-input min.
@@ -142,7 +171,8 @@ __device__ __forceinline__ T block_eval(const Sums<T, D>& s, T M) {
   T acc[4] = {kMax, kMax, kMax, kMax};
   T pend = kMax;
   block_fold<T, D>(s, M, 0, acc, pend);
-  return fold_result<T>(acc, pend, D * D * D);
+  const T g = fold_result<T>(acc, pend, D * D * D);
+  return MCL_LEAF_M_AFTER ? max2(M, g) : g;
 }
 
 template <typename T, int D>
@@ -165,6 +195,7 @@ __device__ __forceinline__ T superblock_eval(const T (&base)[D], const T* __rest
   constexpr int kLeaves = D * D * D;
   T acc[4] = {kMax, kMax, kMax, kMax};
   T pend = kMax;
+  T r = kMax;  // MCL_LEAF_M_AFTER: minimum over the blocks of max(M_x, block minimum)
   Sums<T, D> sb;
   make_sums<T, D>(sb, base, in, one);
   const T Mb = max_of<T, D>(base);
@@ -180,9 +211,17 @@ __device__ __forceinline__ T superblock_eval(const T (&base)[D], const T* __rest
     s.bc[x] = add_f(sb.bc[x], cx, one);
     s.abc[x] = add_f(sb.abc[x], cx, one);
     const T M = max2(Mb, add_f(base[x], cx, one));
+#if MCL_LEAF_M_AFTER
+    // each block's leaves fold on their own (its M applies to its minimum only)
+    T bacc[4] = {kMax, kMax, kMax, kMax};
+    T bpend = kMax;
+    block_fold<T, D>(s, M, 0, bacc, bpend);
+    r = min2(r, max2(M, fold_result<T>(bacc, bpend, kLeaves)));
+#else
     block_fold<T, D>(s, M, x * kLeaves, acc, pend);
+#endif
   }
-  return fold_result<T>(acc, pend, D * kLeaves);
+  return MCL_LEAF_M_AFTER ? r : fold_result<T>(acc, pend, D * kLeaves);
 }
 
 template <typename T, int D>
