@@ -27,8 +27,8 @@ Rank 0 prints one JSON line. `value` is whole-job mappings/s from CUDA events ov
 K timed steps (L2 flushed between steps, outside the events), max over ranks; `e2e` is the
 same metric through the C ABI with pinned host buffers (H2D + D2H inside the timed region;
 batched workloads stage in pipelined chunks, `e2e.pipelined_chunks`); `roofline` is the
-dominant kernel's algorithmic rate against its roofline: `frac` on the leaf table's floor of
-1.5 - 1/D^2 ALU lane-instructions per mapping (SS7) and `frac_survey` on SURVEY SS8(d)'s 2
+dominant kernel's algorithmic rate against its roofline: `frac` on the 1.5 ALU
+lane-instructions per mapping floor (SS7) and `frac_survey` on SURVEY SS8(d)'s 2
 integer ops per mapping, both against the derived ALU peak (the probe-measured rates beside
 them); `cpu_baseline` is the CPU oracle timed on a bounded sample of the workload on the
 host's cores (plus one thread for cfg1-3). `--impl reference` times the oracle instead (this
@@ -52,11 +52,7 @@ sys.path.insert(0, ROOT)
 METRIC = "queue->device mappings scored/sec"
 UNIT = "mappings/s"
 ALU_LANES_PER_CLK_SM = 64       # B200 ALU pipe: 16 lanes x 4 SMSPs per SM per clock (measured: probe)
-def alu_instr_per_mapping(D):
-    """The leaf table's floor (SS7): one max per leaf except the D diagonal leaves of
-    a D^3 block (none), plus 1/2 VIMNMX3 to fold it: 1.5 - 1/D^2 ALU lane-instructions per
-    mapping (1.5 before round 2's once-per-block prefix maximum)."""
-    return 1.5 - 1.0 / (D * D)
+ALU_INSTR_PER_MAPPING = 1.5     # floor: 1 VIMNMX forms the makespan + 1/2 VIMNMX3 folds it
 SURVEY_OPS_PER_MAPPING = 2      # SURVEY SS8(d): one max forms the makespan, one min folds it
 L2_FLUSH_BYTES = 256 << 20      # > 126 MB L2
 HOLD_US = 200                   # spin ahead of each kernel-duration launch (> host launch latency)
@@ -336,8 +332,7 @@ def roofline(w, info, kern_ms, sms, max_mhz, world, mcl, dev_index):
         per_launch = w["E"] * w["N"] if is_replicated(w) else w["N"] / world
         mps = per_launch / (kern_ms / 1e3)
         peak = ALU_LANES_PER_CLK_SM * sms * max_mhz * 1e6 / 1e12
-        floor = alu_instr_per_mapping(w["D"])
-        achieved = floor * mps / 1e12
+        achieved = ALU_INSTR_PER_MAPPING * mps / 1e12
         survey = SURVEY_OPS_PER_MAPPING * mps / 1e12
         roof = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tops/s",
                 "frac": achieved / peak,
@@ -345,8 +340,8 @@ def roofline(w, info, kern_ms, sms, max_mhz, world, mcl, dev_index):
                 "traffic": traffic_from_profiles(w["name"]),
                 "kernel": KERNEL_NAMES.get(info["path"], info["path"]), "kernel_ms": kern_ms,
                 "kernel_timing": KERNEL_TIMING,
-                "algorithmic": f"frac: {floor:.4g} ALU lane-instructions per mapping (the leaf-table floor "
-                               f"1.5 - 1/D^2 with the 3-input VIMNMX3 fold, DESIGN.md SS7); frac_survey: "
+                "algorithmic": f"frac: {ALU_INSTR_PER_MAPPING} ALU lane-instructions per mapping (the floor "
+                               f"with the 3-input VIMNMX3 fold, DESIGN.md SS7); frac_survey: "
                                f"{SURVEY_OPS_PER_MAPPING} integer ops per mapping (SURVEY SS8(d)); x "
                                f"{per_launch:.4g} mappings per launch",
                 "peak_basis": f"derived: {ALU_LANES_PER_CLK_SM} ALU lanes/clk/SM x {sms} SMs x "

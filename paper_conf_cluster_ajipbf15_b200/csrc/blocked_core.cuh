@@ -4,24 +4,22 @@
 // a = Q-3, b = Q-2, c = Q-1 (digits i, j, k) vary inside a block, the outer Q-3 digits are
 // fixed and give the prefix load vector P[d] (queues on one device
 // serialise, devices run concurrently). With M = max_d P[d] and every cost >= 0, the
-// makespan of leaf (i, j, k) is max(M, v) with v the largest load of the devices the inner
-// queues touch, which the compiler-unrolled leaf table below forms with at most ONE integer
-// max per mapping:
+// makespan of leaf (i, j, k) is max(M, load of each device the inner queues touch), which
+// the compiler-unrolled leaf table below forms with ONE integer max per mapping:
 //
-//   i, j, k distinct : v = max3(P_i+A_i, P_j+B_j, P_k+C_k)
-//   i == j != k      : v = max (P_i+A_i+B_i, P_k+C_k)
-//   i == k != j      : v = max (P_i+A_i+C_i, P_j+B_j)
-//   j == k != i      : v = max (P_i+A_i, P_j+B_j+C_j)
-//   i == j == k      : v = P_i+A_i+B_i+C_i            (no instruction)
+//   i, j, k distinct : max3(P_i+A_i, P_j+B_j, max(M, P_k+C_k))
+//   i == j != k      : max (P_i+A_i+B_i, max(M, P_k+C_k))
+//   i == k != j      : max3(P_i+A_i+C_i, P_j+B_j, M)
+//   j == k != i      : max3(P_i+A_i, P_j+B_j+C_j, M)
+//   i == j == k      : max (M, P_i+A_i+B_i+C_i)
 //
 // (A, B, C = the composed cost rows C[q][.] = K + X of queues a, b, c.)
-// Because max(M, .) is non-decreasing, the block minimum of the makespans is max(M, min v):
-// M is applied once per block, not per leaf. The minimum is folded with the sm_100a
-// three-input minimum (VIMNMX3: two leaves per ALU instruction), so the floor is
-// 1.5 - 1/D^2 ALU instructions per mapping. The block minimum is
-// compared with the thread's running best (strict <, blocks visited in increasing index
-// order); only the best block (or super-block) is re-scanned at the end for the lowest
-// leaf index, from the definition.
+// Every leaf's makespan is formed explicitly in a register (a mapping counts
+// as scored only then); the argmin is folded with the sm_100a three-input minimum (VIMNMX3:
+// two mappings per ALU instruction), so the floor is 1.5 ALU instructions per mapping
+// (DESIGN.md "Roofline"). The block minimum is compared with the thread's running best
+// (strict <, blocks visited in increasing index order); only the best block (or
+// super-block) is re-scanned at the end for the lowest leaf index.
 //
 // The outer digits walk an odometer: digit x (queue Q-4) is the block loop, the digits of
 // queues 0..Q-5 live in shared memory and update the base load vector by one-hot vectors
@@ -94,16 +92,17 @@ __device__ __forceinline__ T max_of(const T (&P)[D]) {
 }
 
 #ifndef MCL_LEAF_M_AFTER
-#define MCL_LEAF_M_AFTER 1  // apply the prefix makespan M once per block (0: in every leaf)
+#define MCL_LEAF_M_AFTER 0  // 1: apply the prefix makespan M once per block, not in each leaf
 #endif
 
-// Enumerate the D^3 leaves of one block in increasing index order, calling f(leaf, v).
-// M = max_d P[d] (prefix makespan). With MCL_LEAF_M_AFTER, v is the maximum load of the
-// devices the leaf's three inner queues touch, and the leaf's makespan is max(M, v); as
-// max(M, .) is non-decreasing, min over the leaves of max(M, v) = max(M, min v), so the
-// block applies M once to its minimum instead of once per leaf (no M in the leaf table:
-// D fewer maxima per block for the max(M, C_k) terms, and the D diagonal leaves i == j == k
-// need none at all). Otherwise v is the makespan itself.
+// Enumerate the D^3 leaves of one block in increasing index order, calling f(leaf, v), v =
+// the leaf's makespan. M = max_d P[d] (prefix makespan).
+// MCL_LEAF_M_AFTER (measurement option, not built by default): v is only the maximum load
+// of the devices the leaf's three inner queues touch (makespan = max(M, v)); as max(M, .)
+// is non-decreasing, min over the leaves of max(M, v) = max(M, min v), so the block applies
+// M once to its minimum (D fewer maxima per block, and the D diagonal leaves need none).
+// Same results, 1.4-9 % faster (SS7), but the leaves' makespans are then not
+// formed in registers, which SURVEY SS8(d) requires of a "scored" mapping.
 template <typename T, int D, typename F>
 __device__ __forceinline__ void for_each_leaf(const Sums<T, D>& s, T M, F&& f) {
 #if MCL_LEAF_M_AFTER

@@ -48,12 +48,11 @@ def test_roofline_bookkeeping():
     mps = 8**12 / 6e-3
     peak = 64 * 148 * 1965e6 / 1e12
     assert r["bound"] == "alu" and abs(r["peak"] - peak) < 1e-9
-    floor = 1.5 - 1 / 64  # the leaf table's floor at D = 8: 1.5 - 1/D^2 per mapping
-    assert abs(r["frac"] - floor * mps / 1e12 / peak) < 1e-12
+    assert abs(r["frac"] - 1.5 * mps / 1e12 / peak) < 1e-12
     assert abs(r["frac_survey"] - 2 * mps / 1e12 / peak) < 1e-12
     # sharded: per launch is this rank's share of the index space
     r8 = bench.roofline(w, {"path": "blocked_u32"}, 0.75, 148, 1965, 8, FakeMcl, 0)
-    assert abs(r8["achieved"] - floor * 8**12 / 8 / 0.75e-3 / 1e12) < 1e-9
+    assert abs(r8["achieved"] - 1.5 * 8**12 / 8 / 0.75e-3 / 1e12) < 1e-9
     # batched HBM-bound kernel: algorithmic bytes per epoch = 2*Q*D*8 in + 8 + 8 + Q out
     w3 = dict(name="cfg3", E=10**6, Q=2, D=3, N=9)
     r3 = bench.roofline(w3, {"path": "small_batched"}, 0.02, 148, 1965, 1, FakeMcl, 0)
