@@ -9,7 +9,8 @@
  * 2000 ns whatever the others do, so the optimum is 2000 and its lowest index keeps the other
  * queues off the CPU: (0, 1, 1, 1), index 13. And the SCHED_AUTO_STATIC policy (L1088-1116)
  * with every queue hinted compute-bound and a device profile favouring the GPUs equally sends
- * all four to GPU0 -- makespan 400, twice the optimum.
+ * all four to GPU0 -- makespan 400, twice the optimum. Last, the resident mapper answers the
+ * same decisions without a launch per call.
  *
  *   gcc -O2 -I include examples/map_queues.c -L paper_conf_cluster_ajipbf15_b200 -lmcl \
  *       -Wl,-rpath,$PWD/paper_conf_cluster_ajipbf15_b200 -o /tmp/map_queues
@@ -73,6 +74,20 @@ int main(void) {
   printf("static policy: %s mapping %u %u %u %u makespan %llu\n", mcl_status_string(st), smap[0], smap[1],
          smap[2], smap[3], (unsigned long long)sms);
   ok &= st == MCL_OK && sms == 400 && smap[0] == 1 && smap[3] == 1;
+  /* the resident mapper: one warp stays on the GPU and serves decisions from a pinned host
+     mailbox (no launch per call); the same two epochs, then 1000 single decisions */
+  st = mcl_resident_start(h, Q, D, E, 0);
+  uint64_t ri[E], rms[E];
+  uint8_t rmap[E][Q];
+  if (st == MCL_OK) st = mcl_resident_map(h, E, &K[0][0][0], &X[0][0][0], ri, &rmap[0][0], rms);
+  int rok = st == MCL_OK && ri[0] == 44 && rms[0] == 200 && ri[1] == 1 && rms[1] == 350;
+  for (int i = 0; i < 1000 && st == MCL_OK; ++i) {
+    st = mcl_resident_map(h, 1, &K[i & 1][0][0], &X[i & 1][0][0], ri, &rmap[0][0], rms);
+    rok &= st == MCL_OK && ri[0] == want_index[i & 1] && rms[0] == want_ms[i & 1];
+  }
+  if (mcl_resident_stop(h) != MCL_OK) rok = 0;
+  printf("resident: %s %s\n", mcl_status_string(st), rok ? "agrees" : "differs");
+  ok &= rok;
   /* an entry >= 2^48 is a range error, reported, not silently wrapped */
   K[1][2][1] = (uint64_t)1 << 48;
   st = mcl_map_queues(h, Q, D, E, &K[0][0][0], &X[0][0][0], index, NULL, makespan);

@@ -287,6 +287,34 @@ mcl_status_t mcl_static_mappings(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64
                                  const uint64_t* device_score, const uint16_t* eligible,
                                  uint8_t* mappings);
 
+/*
+ * Resident mapper: low-latency online decisions (cfg1-sized searches). The paper's mapper
+ * runs at every scheduling epoch on the application's critical path;
+ * a launch per decision costs a launch, its ramp and a stream synchronisation (~15 us).
+ * mcl_resident_start leaves ONE warp resident on the handle's device, polling a mailbox
+ * in pinned, device-mapped host memory; mcl_resident_map writes the inputs and a request
+ * number into it and spins until the warp publishes the answer (no launch, no copy engine,
+ * no stream synchronisation per call). Same definition and outputs as mcl_map_queues.
+ *   Q, D        : fixed per start; D^Q <= 4096, Q <= 16, D <= 16.
+ *   max_epochs  : epochs per mcl_resident_map call, 1..64.
+ *   idle_ms     : the warp exits after this long without a request (0 = 100 ms); the next
+ *                 mcl_resident_map relaunches it (one launch, then resident again).
+ * mcl_resident_map: cost_kernel / cost_xfer [epochs][Q][D] and the outputs ([epochs],
+ *   [epochs][Q] or NULL, [epochs]) are HOST pointers (pageable or pinned; copied through the
+ *   mailbox); epochs <= max_epochs. Synchronous. One call at a time per handle.
+ * While the warp is resident, device-wide synchronisation (cudaDeviceSynchronize,
+ * torch.cuda.synchronize) waits for it to exit (at most idle_ms): call mcl_resident_stop
+ * first. mcl_resident_stop (and mcl_mapper_destroy) stop the warp and free the mailbox.
+ * Errors: MCL_E_INVAL (shape, epochs, device pointers, not started), MCL_E_RANGE (an entry
+ * >= 2^48), MCL_E_NOMEM, MCL_E_CUDA (launch failure, or no answer within 2 s).
+ */
+mcl_status_t mcl_resident_start(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint32_t max_epochs,
+                                uint32_t idle_ms);
+mcl_status_t mcl_resident_map(mcl_mapper_t* h, uint64_t epochs, const uint64_t* cost_kernel,
+                              const uint64_t* cost_xfer, uint64_t* mapping_index,
+                              uint8_t* mapping, uint64_t* makespan);
+mcl_status_t mcl_resident_stop(mcl_mapper_t* h);
+
 /* Destroy a handle (NULL-safe). Frees the handle's scratch; never the caller's buffers and
    never the NCCL communicator (its owner, e.g. the torch process group, keeps it). */
 void mcl_mapper_destroy(mcl_mapper_t* h);

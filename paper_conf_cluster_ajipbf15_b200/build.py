@@ -20,7 +20,7 @@ LIB = os.path.join(PKG, "libmcl.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 SOURCES = ["search_blocked.cu", "search_mixed.cu", "search_batch.cu", "search_flat.cu", "search_generic.cu", "search_small.cu",
-           "search_bnb.cu", "costs.cu", "reduce.cu", "score.cu", "probe.cu", "mcl.cpp"]
+           "search_bnb.cu", "resident.cu", "costs.cu", "reduce.cu", "score.cu", "probe.cu", "mcl.cpp"]
 HEADERS = ["common.cuh", "kernels.h", "blocked_core.cuh", "peer.cuh"]
 
 

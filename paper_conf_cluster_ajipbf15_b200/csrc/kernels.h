@@ -276,6 +276,39 @@ cudaError_t launch_decode_pair(const uint64_t* gms, const uint64_t* gidx, uint64
                                cudaStream_t st);
 cudaError_t launch_extract_ms(const uint64_t* pair, uint64_t E, uint64_t* ms, cudaStream_t st);
 
+// Resident mapper (resident.cu): one warp serving decisions from a mailbox in pinned,
+// device-mapped host memory. Control words each on their own 64-byte line; the data
+// arrays follow the header in the same allocation (ResidentArgs holds their device aliases).
+struct ResidentBox {
+  uint64_t req;          // host -> device, written after the inputs: request number (bits
+                         // 0-31) | epochs (bits 32-47) | stop (bit 63)
+  uint32_t pad0[14];
+  uint32_t done_seq;     // device -> host: number of the last request served
+  uint32_t status;       // kFlag* of that request
+  uint32_t alive;        // 1 while the warp runs
+  uint32_t exit_reason;  // 1 stop, 2 idle timeout
+  uint32_t pad1[2];
+  uint64_t trace[5];     // -DMCL_RESIDENT_TRACE builds: %globaltimer at request seen, inputs
+                         // read, scored, results published
+  uint32_t pad2[16];
+};
+static_assert(sizeof(ResidentBox) == 192, "three 64-byte lines");
+constexpr uint32_t kResidentMaxMappings = 4096;  // D^Q per epoch (12 index bits)
+constexpr uint32_t kResidentMaxQ = 16, kResidentMaxD = 16;
+struct ResidentArgs {
+  ResidentBox* box;           // device alias of the mailbox
+  const uint64_t* K;          // [cap][Q][D] device aliases of the mailbox arrays
+  const uint64_t* X;
+  uint64_t* index;            // [cap]
+  uint64_t* makespan;         // [cap]
+  uint8_t* mapping;           // [cap][Q]
+  uint32_t Q, D, N, cap;
+  uint32_t seq0;              // request number already served when the warp starts
+  uint64_t idle_ns;
+};
+size_t resident_smem_bytes(uint32_t Q, uint32_t D, uint32_t cap);
+cudaError_t launch_resident(const ResidentArgs& a, cudaStream_t st);
+
 // ALU throughput probe (probe.cu), SURVEY N7.
 cudaError_t probe_alu(int op, int sms, cudaStream_t st, double* lane_ops_per_s,
                       double* lane_ops_per_clk_sm, double* eff_mhz);

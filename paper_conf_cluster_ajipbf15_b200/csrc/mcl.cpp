@@ -11,6 +11,7 @@
 #include <dlfcn.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -164,6 +165,13 @@ struct mcl_mapper {
   cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
   int64_t info[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   std::string last_err;
+  // resident mapper (mcl_resident_*): mailbox in pinned, mapped host memory, the warp's
+  // own stream, its launch arguments (device aliases) and the last request number
+  unsigned char* res_mem = nullptr;
+  cudaStream_t res_stream = nullptr;
+  mcl::ResidentArgs res_args{};
+  uint32_t res_seq = 0;
+  bool res_started = false;
 };
 
 namespace {
@@ -348,6 +356,7 @@ mcl_status_t mcl_mapper_create(const mcl_config_t* cfg, mcl_mapper_t** out) {
 
 void mcl_mapper_destroy(mcl_mapper_t* h) {
   if (!h) return;
+  mcl_resident_stop(h);
   {
     DeviceGuard g(h->device);
     if (h->stream) cudaStreamSynchronize(h->stream);
@@ -1475,6 +1484,192 @@ mcl_status_t mcl_comm_destroy(void* comm) {
   if (!comm) return MCL_OK;
   if (!nccl().ok) return MCL_E_NCCL;
   return nccl().CommDestroy((ncclComm_t)comm) == ncclSuccess ? MCL_OK : MCL_E_NCCL;
+}
+
+}  // extern "C"
+
+// ---------------------------------------------------------------- resident mapper ------
+namespace {
+
+mcl::ResidentBox* res_box(mcl_mapper* h) { return reinterpret_cast<mcl::ResidentBox*>(h->res_mem); }
+
+// (Re)launch the resident warp; it serves the requests numbered after seq0. `alive` is set
+// here, before the launch, so 0 is only ever seen after a warp has exited.
+mcl_status_t resident_launch(mcl_mapper* h, uint32_t seq0) {
+  mcl::ResidentBox* box = res_box(h);
+  // no stop bit; the number of the last request (a relaunch for a pending request passes
+  // seq0 = its number - 1, so the new warp serves it)
+  __atomic_store_n(&box->req, __atomic_load_n(&box->req, __ATOMIC_RELAXED) & ~(1ull << 63), __ATOMIC_RELEASE);
+  __atomic_store_n(&box->alive, 1u, __ATOMIC_RELEASE);  // the warp clears it when it exits
+  h->res_args.seq0 = seq0;
+  MCL_CUDA(h, mcl::launch_resident(h->res_args, h->res_stream), "resident launch");
+  return MCL_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+mcl_status_t mcl_resident_start(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint32_t max_epochs,
+                                uint32_t idle_ms) {
+  if (!h) return MCL_E_INVAL;
+  if (h->res_started) {
+    h->last_err = "resident mapper already started on this handle";
+    return MCL_E_INVAL;
+  }
+  uint64_t N = 0;
+  if (Q < 1 || D < 1 || Q > mcl::kResidentMaxQ || D > mcl::kResidentMaxD || max_epochs < 1 ||
+      max_epochs > 64 || mul_overflow_pow(D, Q, mcl::kResidentMaxMappings, &N)) {
+    h->last_err = "resident mapper: needs D^Q <= 4096, Q <= 16, D <= 16, 1 <= max_epochs <= 64";
+    return MCL_E_INVAL;
+  }
+  DeviceGuard g(h->device);
+  const size_t qd = (size_t)max_epochs * Q * D;
+  const size_t off_k = sizeof(mcl::ResidentBox), off_x = off_k + qd * 8, off_i = off_x + qd * 8,
+               off_m = off_i + (size_t)max_epochs * 8, off_p = off_m + (size_t)max_epochs * 8,
+               bytes = off_p + (size_t)max_epochs * Q;
+  if (cudaHostAlloc((void**)&h->res_mem, bytes, cudaHostAllocMapped) != cudaSuccess) {
+    cudaGetLastError();
+    h->res_mem = nullptr;
+    h->last_err = "cudaHostAlloc(resident mailbox) failed";
+    return MCL_E_NOMEM;
+  }
+  std::memset(h->res_mem, 0, bytes);
+  unsigned char* dev = nullptr;
+  cudaError_t e = cudaHostGetDevicePointer((void**)&dev, h->res_mem, 0);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->res_stream, cudaStreamNonBlocking);
+  if (e != cudaSuccess) {
+    cudaFreeHost(h->res_mem);
+    h->res_mem = nullptr;
+    return cuda_fail(h, e, "resident mailbox / stream");
+  }
+  mcl::ResidentArgs& a = h->res_args;
+  a.box = reinterpret_cast<mcl::ResidentBox*>(dev);
+  a.K = reinterpret_cast<const uint64_t*>(dev + off_k);
+  a.X = reinterpret_cast<const uint64_t*>(dev + off_x);
+  a.index = reinterpret_cast<uint64_t*>(dev + off_i);
+  a.makespan = reinterpret_cast<uint64_t*>(dev + off_m);
+  a.mapping = dev + off_p;
+  a.Q = Q;
+  a.D = D;
+  a.N = (uint32_t)N;
+  a.cap = max_epochs;
+  a.idle_ns = (uint64_t)(idle_ms ? idle_ms : 100) * 1000000ull;
+  h->res_seq = 0;
+  h->res_started = true;
+  const mcl_status_t st = resident_launch(h, 0);
+  if (st != MCL_OK) mcl_resident_stop(h);
+  return st;
+}
+
+mcl_status_t mcl_resident_map(mcl_mapper_t* h, uint64_t epochs, const uint64_t* cost_kernel,
+                              const uint64_t* cost_xfer, uint64_t* mapping_index,
+                              uint8_t* mapping, uint64_t* makespan) {
+  if (!h) return MCL_E_INVAL;
+  if (!h->res_started) {
+    h->last_err = "resident mapper not started (mcl_resident_start)";
+    return MCL_E_INVAL;
+  }
+  if (epochs == 0) return MCL_OK;
+  mcl::ResidentArgs& a = h->res_args;
+  if (epochs > a.cap || !cost_kernel || !cost_xfer || !mapping_index || !makespan) {
+    h->last_err = "resident mapper: epochs above max_epochs or a NULL buffer";
+    return MCL_E_INVAL;
+  }
+  for (const void* p : {(const void*)cost_kernel, (const void*)cost_xfer, (const void*)mapping_index,
+                        (const void*)makespan, (const void*)mapping}) {
+    if (!p) continue;
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+      cudaGetLastError();
+      h->last_err = "resident mapper: cannot classify a buffer pointer";
+      return MCL_E_INVAL;
+    }
+    if (at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged) {
+      h->last_err = "resident mapper: buffers must be host memory";
+      return MCL_E_INVAL;
+    }
+  }
+  mcl::ResidentBox* box = res_box(h);
+  if (!__atomic_load_n(&box->alive, __ATOMIC_ACQUIRE)) {  // idle exit: relaunch
+    DeviceGuard g(h->device);
+    const cudaError_t e = cudaStreamQuery(h->res_stream);  // the exited kernel is gone
+    if (e != cudaSuccess && e != cudaErrorNotReady) return cuda_fail(h, e, "resident kernel");
+    cudaGetLastError();
+    const mcl_status_t st = resident_launch(h, h->res_seq);
+    if (st != MCL_OK) return st;
+  }
+  const size_t qd = (size_t)epochs * a.Q * a.D;
+  unsigned char* base = h->res_mem;
+  const size_t off_k = sizeof(mcl::ResidentBox), off_x = off_k + (size_t)a.cap * a.Q * a.D * 8,
+               off_i = off_x + (size_t)a.cap * a.Q * a.D * 8, off_m = off_i + (size_t)a.cap * 8,
+               off_p = off_m + (size_t)a.cap * 8;
+  std::memcpy(base + off_k, cost_kernel, qd * 8);
+  std::memcpy(base + off_x, cost_xfer, qd * 8);
+  const uint32_t seq = ++h->res_seq;
+  // inputs before the request word (x86 stores are ordered; release for the compiler)
+  __atomic_store_n(&box->req, ((uint64_t)epochs << 32) | seq, __ATOMIC_RELEASE);
+  const auto t0 = std::chrono::steady_clock::now();
+  for (uint32_t spin = 1;; ++spin) {
+    if (__atomic_load_n(&box->done_seq, __ATOMIC_ACQUIRE) == seq) break;
+    if ((spin & 1023u) == 0) {
+      const bool dead = !__atomic_load_n(&box->alive, __ATOMIC_ACQUIRE);
+      if (dead || std::chrono::steady_clock::now() - t0 > std::chrono::seconds(2)) {
+        if (dead && __atomic_load_n(&box->done_seq, __ATOMIC_ACQUIRE) == seq) break;
+        DeviceGuard g(h->device);
+        const cudaError_t e = cudaStreamQuery(h->res_stream);
+        h->last_err = dead ? "resident warp exited before answering"
+                           : "resident warp did not answer within 2 s";
+        if (e != cudaSuccess && e != cudaErrorNotReady) return cuda_fail(h, e, "resident kernel");
+        if (!dead) return MCL_E_CUDA;
+        // it exited idle between the alive check and the request: a new warp serves it
+        const mcl_status_t st = resident_launch(h, seq - 1);
+        if (st != MCL_OK) return st;
+      }
+    }
+  }
+  const uint32_t status = __atomic_load_n(&box->status, __ATOMIC_RELAXED);
+  if (status & mcl::kFlagRange) {
+    h->last_err = "a cost entry >= 2^48";
+    return MCL_E_RANGE;
+  }
+  if (status) {
+    h->last_err = "resident mapper: bad request";
+    return MCL_E_INVAL;
+  }
+  std::memcpy(mapping_index, base + off_i, epochs * 8);
+  std::memcpy(makespan, base + off_m, epochs * 8);
+  if (mapping) std::memcpy(mapping, base + off_p, epochs * a.Q);
+  return MCL_OK;
+}
+
+#ifdef MCL_RESIDENT_TRACE
+// measurement builds only: the resident warp's timestamps of its last request
+int mcl_resident_trace(mcl_mapper_t* h, uint64_t out[4]) {
+  if (!h || !h->res_mem) return -1;
+  for (int i = 0; i < 3; ++i) out[i] = __atomic_load_n(&res_box(h)->trace[i], __ATOMIC_RELAXED);
+  out[3] = out[2];
+  return 0;
+}
+#endif
+
+mcl_status_t mcl_resident_stop(mcl_mapper_t* h) {
+  if (!h) return MCL_E_INVAL;
+  if (!h->res_mem) return MCL_OK;
+  DeviceGuard g(h->device);
+  mcl::ResidentBox* box = res_box(h);
+  __atomic_store_n(&box->req, __atomic_load_n(&box->req, __ATOMIC_RELAXED) | (1ull << 63), __ATOMIC_RELEASE);
+  cudaError_t e = cudaSuccess;
+  if (h->res_stream) {
+    e = cudaStreamSynchronize(h->res_stream);
+    cudaStreamDestroy(h->res_stream);
+    h->res_stream = nullptr;
+  }
+  cudaFreeHost(h->res_mem);
+  h->res_mem = nullptr;
+  h->res_started = false;
+  if (e != cudaSuccess) return cuda_fail(h, e, "resident kernel");
+  return MCL_OK;
 }
 
 }  // extern "C"

@@ -1,0 +1,245 @@
+// resident.cu -- a resident mapper for online decisions (cfg1-sized searches).
+//
+// The paper's mapper runs at every scheduling epoch, inside the runtime's scheduler thread,
+// and its decision is on the application's critical path (the search
+// must stay "negligible"). A launch per decision costs a kernel launch, the launch ramp and
+// a stream synchronisation (~15 us per call, SS12), far more than scoring 81
+// mappings. Here ONE warp stays resident on the GPU and serves decisions from a mailbox in
+// pinned, device-mapped host memory: the host writes an epoch batch's K and X and then a
+// request number; the warp (polling the request number over PCIe) reads the inputs in
+// place, scores every mapping (the same definition as every other path: C = K + X,
+// PAPER.md L2106-2118; loads per device, makespan = max over devices, L1048-1052; argmin
+// with the lowest index on ties), writes index / makespan / mapping digits back into the
+// mailbox and publishes the request number as done. No launch, no copy engine, no stream
+// synchronisation per decision.
+//
+// Shape: any Q <= 16, D <= 16 with D^Q <= 4096 (one warp; lane l scores mappings l, l + 32,
+// ... in increasing order keeping its first strict minimum, then five shuffle rounds of the
+// lexicographic (makespan, index) minimum). The warp exits when the host sets `stop`, or
+// after `idle_ns` without a request (the host relaunches it on demand).
+#include "common.cuh"
+#include "kernels.h"
+
+namespace mcl {
+
+namespace {
+
+__device__ __forceinline__ uint64_t ld_acquire_sys64(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_sys(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t ld_relaxed_sys64(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint64_t now_ns() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+// Lowest-index minimum makespan of one epoch (C = [Q][D] composed costs in shared memory),
+// by the 32 lanes: lane l scores m = l, l + 32, ... in increasing order (strict <), then
+// five shuffle rounds of the lexicographic (makespan, index) minimum. QT, DT > 0: shape
+// fixed at compile time (digits by constant division, loads in registers by static
+// selects); 0: runtime shape (loads in this lane's shared-memory row).
+template <int QT, int DT>
+__device__ __forceinline__ void score_epoch(const uint64_t* C, uint32_t Qr, uint32_t Dr, uint32_t N,
+                                            uint64_t* sL, uint64_t& best_ms, uint32_t& best_m) {
+  const int lane = threadIdx.x & 31;
+  uint64_t bms = ~0ull;
+  uint32_t bm = 0xffffffffu;
+  if constexpr (QT > 0) {
+    uint64_t c[QT][DT];
+#pragma unroll
+    for (int q = 0; q < QT; ++q)
+#pragma unroll
+      for (int d = 0; d < DT; ++d) c[q][d] = C[q * DT + d];
+    for (uint32_t m = lane; m < N; m += 32) {
+      uint64_t L[DT];
+#pragma unroll
+      for (int d = 0; d < DT; ++d) L[d] = 0;
+      uint32_t rest = m;
+#pragma unroll
+      for (int q = QT - 1; q >= 0; --q) {  // queue 0 is the most significant digit
+        const uint32_t dq = rest % DT;
+        rest /= DT;
+#pragma unroll
+        for (int d = 0; d < DT; ++d) L[d] += (dq == (uint32_t)d) ? c[q][d] : 0;  // a3
+      }
+      uint64_t ms = L[0];
+#pragma unroll
+      for (int d = 1; d < DT; ++d) ms = max(ms, L[d]);  // a4
+      if (ms < bms) {  // a5: strict, so the lane keeps its lowest index of a tie
+        bms = ms;
+        bm = m;
+      }
+    }
+  } else {
+    for (uint32_t m = lane; m < N; m += 32) {
+      for (uint32_t d = 0; d < Dr; ++d) sL[d] = 0;
+      uint32_t rest = m;
+      for (int q = (int)Qr - 1; q >= 0; --q) {
+        const uint32_t dq = rest % Dr;
+        rest /= Dr;
+        sL[dq] += C[q * Dr + dq];
+      }
+      uint64_t ms = 0;
+      for (uint32_t d = 0; d < Dr; ++d) ms = max(ms, sL[d]);
+      if (ms < bms) {
+        bms = ms;
+        bm = m;
+      }
+    }
+  }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) {  // lexicographic (makespan, index) minimum
+    const uint64_t oms = __shfl_xor_sync(0xffffffffu, bms, off);
+    const uint32_t om = __shfl_xor_sync(0xffffffffu, bm, off);
+    if (oms < bms || (oms == bms && om < bm)) {
+      bms = oms;
+      bm = om;
+    }
+  }
+  best_ms = bms;
+  best_m = bm;
+}
+
+}  // namespace
+
+template <int QT, int DT>
+__global__ void __launch_bounds__(32) resident_kernel(ResidentArgs a) {
+  extern __shared__ __align__(16) uint64_t s_res[];
+  const int lane = threadIdx.x;
+  const uint32_t Q = QT > 0 ? QT : a.Q, D = DT > 0 ? DT : a.D, N = a.N, QD = Q * D;
+  uint64_t* sC = s_res;                                   // [cap][Q][D] composed costs
+  uint64_t* sL = s_res + (size_t)a.cap * QD + lane * 16;  // generic shapes: this lane's loads
+  ResidentBox* box = a.box;
+  uint32_t last = a.seq0;
+  uint64_t t_idle = now_ns();
+  for (;;) {
+    // ---- wait for a request: lane 0 polls one word (number, epochs, stop) over PCIe ----
+    uint64_t req = 0;
+    uint32_t quit = 0;
+    if (lane == 0) {
+      // one acquire load of the request word at a time: measured, several relaxed loads
+      // in flight (4 or 8, staggered) or a pause between polls only add latency
+      // (SS7, resident mapper)
+      for (;;) {
+        req = ld_acquire_sys64(&box->req);
+        if (req >> 63) {
+          quit = 1;
+          break;
+        }
+        if ((uint32_t)req != last) break;
+        if (now_ns() - t_idle > a.idle_ns) {
+          quit = 2;
+          break;
+        }
+      }
+    }
+    quit = __shfl_sync(0xffffffffu, quit, 0);
+    req = __shfl_sync(0xffffffffu, req, 0);
+    if (quit) {
+      if (lane == 0) {
+        box->exit_reason = quit;
+        st_release_sys(&box->alive, 0u);
+      }
+      return;
+    }
+    const uint32_t seq = (uint32_t)req, E = (uint32_t)(req >> 32) & 0xffffu;
+    last = seq;
+#ifdef MCL_RESIDENT_TRACE
+    const uint64_t tr0 = now_ns();
+#endif
+    // ---- inputs, read in place from host memory after the acquire (a1: C = K + X) ----
+    uint32_t status = 0;
+    if (E > a.cap) status |= kFlagBadModel;
+    const uint32_t n = (E <= a.cap ? E : 0u) * QD;
+    bool bad = false;
+    for (uint32_t i0 = lane; i0 < n; i0 += 4 * 32) {  // 8 loads in flight per lane (PCIe)
+      uint64_t k[4], x[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const uint32_t i = i0 + 32 * u;
+        k[u] = i < n ? ld_relaxed_sys64(a.K + i) : 0;
+        x[u] = i < n ? ld_relaxed_sys64(a.X + i) : 0;
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const uint32_t i = i0 + 32 * u;
+        bad |= (k[u] >= kEntryLimit) | (x[u] >= kEntryLimit);
+        if (i < n) sC[i] = k[u] + x[u];
+      }
+    }
+    if (__any_sync(0xffffffffu, bad)) status |= kFlagRange;
+    __syncwarp();
+#ifdef MCL_RESIDENT_TRACE
+    const uint64_t tr1 = now_ns();
+#endif
+    if (status == 0) {
+      for (uint32_t e = 0; e < E; ++e) {
+        uint64_t ms;
+        uint32_t idx;
+        score_epoch<QT, DT>(sC + (size_t)e * QD, Q, D, N, sL, ms, idx);
+        if (lane == 0) {
+          a.index[e] = idx;
+          a.makespan[e] = ms;
+        }
+        if (lane < (int)Q) {  // a7: digits of the index, queue 0 most significant
+          uint32_t rest = idx;
+          for (int q = (int)Q - 1; q > lane; --q) rest /= D;
+          a.mapping[(size_t)e * Q + lane] = (uint8_t)(rest % D);
+        }
+      }
+    }
+    if (lane == 0) box->status = status;
+    // every lane's result stores, then lane 0's release of the request number: the warp
+    // barrier orders them before it, and a release at system scope is cumulative, so the
+    // host's acquire of done_seq sees all of them
+    __syncwarp();
+    if (lane == 0) {
+#ifdef MCL_RESIDENT_TRACE
+      box->trace[0] = tr0;
+      box->trace[1] = tr1;
+      box->trace[2] = now_ns();
+#endif
+      st_release_sys(&box->done_seq, seq);
+    }
+    t_idle = now_ns();
+  }
+}
+
+size_t resident_smem_bytes(uint32_t Q, uint32_t D, uint32_t cap) {
+  return ((size_t)cap * Q * D + 32 * 16) * sizeof(uint64_t);
+}
+
+cudaError_t launch_resident(const ResidentArgs& a, cudaStream_t st) {
+  const size_t smem = resident_smem_bytes(a.Q, a.D, a.cap);
+  void (*k)(ResidentArgs) = resident_kernel<0, 0>;
+  switch (a.Q * 100 + a.D) {  // compile-time shapes of small decisions (cfg1: 4 x 3)
+#define MCL_RES_CASE(QQ, DD) \
+  case QQ * 100 + DD: k = resident_kernel<QQ, DD>; break;
+    MCL_RES_CASE(2, 2) MCL_RES_CASE(2, 3) MCL_RES_CASE(2, 4) MCL_RES_CASE(3, 2) MCL_RES_CASE(3, 3)
+    MCL_RES_CASE(3, 4) MCL_RES_CASE(4, 2) MCL_RES_CASE(4, 3) MCL_RES_CASE(4, 4) MCL_RES_CASE(5, 3)
+    MCL_RES_CASE(5, 4) MCL_RES_CASE(6, 3) MCL_RES_CASE(6, 4) MCL_RES_CASE(8, 2) MCL_RES_CASE(8, 3)
+#undef MCL_RES_CASE
+    default: break;
+  }
+  // the compile-time shapes need at most 64 x 8 x 4 entries + the lane rows (20 KB, under
+  // the default 48 KB); only the generic kernel may need the larger opt-in
+  if (k == resident_kernel<0, 0>) {
+    static SmemAttrCache cache;
+    cudaError_t err = ensure_smem(k, smem, cache);
+    if (err != cudaSuccess) return err;
+  }
+  k<<<1, 32, smem, st>>>(a);
+  return cudaGetLastError();
+}
+
+}  // namespace mcl

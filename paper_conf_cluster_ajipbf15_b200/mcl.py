@@ -30,6 +30,7 @@ EXPORTED = [
     "mcl_map_queues_constrained", "mcl_score_mappings", "mcl_map_queues_pruned",
     "mcl_build_costs", "mcl_map_from_profiles",
     "mcl_peer_export", "mcl_peer_import", "mcl_static_mappings",
+    "mcl_resident_start", "mcl_resident_map", "mcl_resident_stop",
 ]
 
 
@@ -113,6 +114,9 @@ def load_library(path: str | None = None) -> ctypes.CDLL:
         "mcl_peer_export": (i32, [vp, u64, ctypes.c_char_p]),
         "mcl_peer_import": (i32, [vp, ctypes.c_char_p, u32]),
         "mcl_static_mappings": (i32, [vp, u32, u32, u64, vp, u32, vp, vp, vp]),
+        "mcl_resident_start": (i32, [vp, u32, u32, u32, u32]),
+        "mcl_resident_map": (i32, [vp, u64, vp, vp, vp, vp, vp]),
+        "mcl_resident_stop": (i32, [vp]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -514,6 +518,72 @@ class Mapper:
         if st != MCL_OK:
             raise MclError(st, "mcl_static_mappings", mcl_last_error_string(self.handle))
         return out
+
+    def resident_start(self, Q: int, D: int, max_epochs: int = 1, idle_ms: int = 0) -> None:
+        """Leave one warp resident for low-latency decisions (include/mcl.h
+        mcl_resident_start): D^Q <= 4096, max_epochs <= 64 per resident_map call. While it is
+        resident, device-wide synchronisation waits for it (up to idle_ms): stop it first."""
+        st = load_library().mcl_resident_start(self.handle, Q, D, max_epochs, idle_ms)
+        if st != MCL_OK:
+            raise MclError(st, "mcl_resident_start", mcl_last_error_string(self.handle))
+        self._resident = (int(Q), int(D), int(max_epochs))
+        self._res_fn = load_library().mcl_resident_map
+        self._res_cache = None
+
+    def resident_map(self, K, X, out=None):
+        """One decision batch through the resident warp. K, X: HOST arrays [E, Q, D] (or
+        [Q, D]) uint64 (numpy, or CPU torch tensors); returns (index [E], mapping [E, Q],
+        makespan [E]) numpy arrays, or fills ``out`` = (index, mapping, makespan)."""
+        Q, D, cap = getattr(self, "_resident", (0, 0, 0))
+        if not Q:
+            raise MclError(-1, "mcl_resident_map", "resident mapper not started")
+        if K.ndim == 2:
+            K, X = K[None], X[None]
+        E = int(K.shape[0])
+        if out is None:
+            out = (np.empty(E, np.uint64), np.empty((E, Q), np.uint8), np.empty(E, np.uint64))
+        idx, mp, ms = out
+        c = self._res_cache
+        if (c is not None and K is c[0] and X is c[1] and idx is c[2] and mp is c[3] and ms is c[4]
+                and K.shape == c[5]):
+            # the same five arrays as the previous call (kept alive by the cache, so their
+            # addresses are still theirs): a decision is a few microseconds, and building an
+            # address from a numpy array costs ~1.5 us each
+            st = self._res_fn(self.handle, E, *c[6])
+        elif (type(K) is np.ndarray and type(X) is np.ndarray and type(idx) is np.ndarray
+                and type(ms) is np.ndarray and type(mp) is np.ndarray):
+            want = (E, Q, D)
+            if (K.shape != want or X.shape != want or idx.shape != (E,) or ms.shape != (E,)
+                    or mp.shape != (E, Q)):
+                raise ValueError(f"resident_map: expected K, X {want}, outputs ({E},), ({E}, {Q}), ({E},)")
+            for a, dt in ((K, np.uint64), (X, np.uint64), (idx, np.uint64), (ms, np.uint64), (mp, np.uint8)):
+                if a.dtype != dt or not a.flags.c_contiguous:
+                    raise TypeError(f"expected C-contiguous {np.dtype(dt)} arrays")
+            ptrs = tuple(a.ctypes.data for a in (K, X, idx, mp, ms))
+            self._res_cache = (K, X, idx, mp, ms, K.shape, ptrs)
+            st = self._res_fn(self.handle, E, *ptrs)
+        else:
+            _check("K", K, (E, Q, D))
+            _check("X", X, (E, Q, D))
+            _check("index", idx, (E,))
+            _check("mapping", mp, (E, Q))
+            _check("makespan", ms, (E,))
+            pk, _k = _ptr_and_keepalive(K, np.uint64)
+            px, _x = _ptr_and_keepalive(X, np.uint64)
+            pi, _i = _ptr_and_keepalive(idx, np.uint64)
+            pm, _m = _ptr_and_keepalive(ms, np.uint64)
+            pmap = _ptr_and_keepalive(mp, np.uint8)[0] if mp is not None else None
+            st = self._res_fn(self.handle, E, pk, px, pi, pmap, pm)
+        if st != MCL_OK:
+            raise MclError(st, "mcl_resident_map", mcl_last_error_string(self.handle))
+        return idx, mp, ms
+
+    def resident_stop(self) -> None:
+        st = load_library().mcl_resident_stop(self.handle)
+        self._resident = (0, 0, 0)
+        self._res_cache = None
+        if st != MCL_OK:
+            raise MclError(st, "mcl_resident_stop", mcl_last_error_string(self.handle))
 
     @staticmethod
     def _alloc_outputs(K, E, Q, with_mapping):

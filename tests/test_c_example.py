@@ -40,5 +40,6 @@ def test_c_example_runs(tmp_path):
     assert "epoch 1: index 1 makespan 350 mapping 0 0 0 1" in r.stdout
     assert "pinned queue 0: MCL_OK: success index 13 makespan 2000 mapping 0 1 1 1" in r.stdout
     assert "static policy: MCL_OK: success mapping 1 1 1 1 makespan 400" in r.stdout
+    assert "resident: MCL_OK: success agrees" in r.stdout
     assert "entry 2^48: MCL_E_RANGE" in r.stdout
     assert r.stdout.strip().endswith("OK")
