@@ -531,7 +531,7 @@ def measure(ctx, name):
             res_s = (time.perf_counter() - t0) / (e2e_steps * 10)
         finally:
             mapper.resident_stop()
-        e2e_s = min(e2e_s, res_s)
+        e2e_s = res_s  # the call a user makes for a single decision
     mapper.close()
 
     total_ms, kern_mean, e2e_s, e2e_launch_s = max_over_ranks(ctx, [total_ms, kern_mean, e2e_s, e2e_launch_s])
@@ -563,7 +563,7 @@ def measure(ctx, name):
         "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": K.nbytes + X.nbytes,
                 "d2h_bytes_per_step": E * (8 + 8 + Q), "ms_per_step": e2e_s * 1e3,
                 "api": ("mcl_resident_map (resident warp; inputs read in place over PCIe, results "
-                        "written back to the pinned mailbox)" if res_s is not None and e2e_s == res_s
+                        "written back to the pinned mailbox)" if res_s is not None
                         else "mcl_map_queues on pinned host buffers"),
                 "pipelined_chunks": e2e_chunks,
                 "host_buffers": "one pinned arena allocated at start-up on the GPU's NUMA node"
