@@ -283,8 +283,8 @@ struct ResidentBox {
   uint64_t req;          // host -> device, written after the inputs: request number (bits
                          // 0-31) | epochs (bits 32-47) | stop (bit 63)
   uint32_t pad0[14];
-  uint32_t done_seq;     // device -> host: number of the last request served
-  uint32_t status;       // kFlag* of that request
+  uint32_t done_seq;     // (unused: every result record carries its request's tag)
+  uint32_t status;       // (unused)
   uint32_t alive;        // 1 while the warp runs
   uint32_t exit_reason;  // 1 stop, 2 idle timeout
   uint32_t pad1[2];
@@ -295,13 +295,18 @@ struct ResidentBox {
 static_assert(sizeof(ResidentBox) == 192, "three 64-byte lines");
 constexpr uint32_t kResidentMaxMappings = 4096;  // D^Q per epoch (12 index bits)
 constexpr uint32_t kResidentMaxQ = 16, kResidentMaxD = 16;
+// Result record of one epoch, three u64 words each written whole by one store (single-copy
+// atomic at system scope), each tagged with the request number so the host accepts a
+// record only when all three words are this request's -- no fence before a done flag:
+//   w0 = seq << 32 | status << 16 | index (< 4096)
+//   w1 = (seq mod 2^11) << 53 | makespan (< 2^53)
+//   w2 = seq << 32 | digits (queue q's device in bits [q*b, q*b + b), b = bits of D - 1)
+constexpr int kResidentRecWords = 3;
 struct ResidentArgs {
   ResidentBox* box;           // device alias of the mailbox
   const uint64_t* K;          // [cap][Q][D] device aliases of the mailbox arrays
   const uint64_t* X;
-  uint64_t* index;            // [cap]
-  uint64_t* makespan;         // [cap]
-  uint8_t* mapping;           // [cap][Q]
+  uint64_t* rec;              // [cap][3] result records
   uint32_t Q, D, N, cap;
   uint32_t seq0;              // request number already served when the warp starts
   uint64_t idle_ns;

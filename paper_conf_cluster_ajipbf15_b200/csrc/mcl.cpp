@@ -1525,9 +1525,8 @@ mcl_status_t mcl_resident_start(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint32_
   }
   DeviceGuard g(h->device);
   const size_t qd = (size_t)max_epochs * Q * D;
-  const size_t off_k = sizeof(mcl::ResidentBox), off_x = off_k + qd * 8, off_i = off_x + qd * 8,
-               off_m = off_i + (size_t)max_epochs * 8, off_p = off_m + (size_t)max_epochs * 8,
-               bytes = off_p + (size_t)max_epochs * Q;
+  const size_t off_k = sizeof(mcl::ResidentBox), off_x = off_k + qd * 8, off_r = off_x + qd * 8,
+               bytes = off_r + (size_t)max_epochs * mcl::kResidentRecWords * 8;
   if (cudaHostAlloc((void**)&h->res_mem, bytes, cudaHostAllocMapped) != cudaSuccess) {
     cudaGetLastError();
     h->res_mem = nullptr;
@@ -1547,9 +1546,7 @@ mcl_status_t mcl_resident_start(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint32_
   a.box = reinterpret_cast<mcl::ResidentBox*>(dev);
   a.K = reinterpret_cast<const uint64_t*>(dev + off_k);
   a.X = reinterpret_cast<const uint64_t*>(dev + off_x);
-  a.index = reinterpret_cast<uint64_t*>(dev + off_i);
-  a.makespan = reinterpret_cast<uint64_t*>(dev + off_m);
-  a.mapping = dev + off_p;
+  a.rec = reinterpret_cast<uint64_t*>(dev + off_r);
   a.Q = Q;
   a.D = D;
   a.N = (uint32_t)N;
@@ -1602,20 +1599,35 @@ mcl_status_t mcl_resident_map(mcl_mapper_t* h, uint64_t epochs, const uint64_t* 
   const size_t qd = (size_t)epochs * a.Q * a.D;
   unsigned char* base = h->res_mem;
   const size_t off_k = sizeof(mcl::ResidentBox), off_x = off_k + (size_t)a.cap * a.Q * a.D * 8,
-               off_i = off_x + (size_t)a.cap * a.Q * a.D * 8, off_m = off_i + (size_t)a.cap * 8,
-               off_p = off_m + (size_t)a.cap * 8;
+               off_r = off_x + (size_t)a.cap * a.Q * a.D * 8;
   std::memcpy(base + off_k, cost_kernel, qd * 8);
   std::memcpy(base + off_x, cost_xfer, qd * 8);
   const uint32_t seq = ++h->res_seq;
   // inputs before the request word (x86 stores are ordered; release for the compiler)
   __atomic_store_n(&box->req, ((uint64_t)epochs << 32) | seq, __ATOMIC_RELEASE);
+  // The answer: one three-word record per epoch, each word tagged with this request's
+  // number (kernels.h, ResidentArgs); a failed request answers with its status in epoch 0.
+  const uint64_t* rec = reinterpret_cast<const uint64_t*>(base + off_r);
+  auto ready = [&](uint64_t e) {
+    const uint64_t w0 = __atomic_load_n(rec + 3 * e, __ATOMIC_ACQUIRE);
+    const uint64_t w1 = __atomic_load_n(rec + 3 * e + 1, __ATOMIC_ACQUIRE);
+    const uint64_t w2 = __atomic_load_n(rec + 3 * e + 2, __ATOMIC_ACQUIRE);
+    return (uint32_t)(w0 >> 32) == seq && (w1 >> 53) == (seq & 0x7ffu) && (uint32_t)(w2 >> 32) == seq;
+  };
+  auto answered = [&]() {
+    if (!ready(0)) return false;
+    if ((__atomic_load_n(rec, __ATOMIC_RELAXED) >> 16) & 0xffffu) return true;  // an error
+    for (uint64_t e = 1; e < epochs; ++e)
+      if (!ready(e)) return false;
+    return true;
+  };
   const auto t0 = std::chrono::steady_clock::now();
   for (uint32_t spin = 1;; ++spin) {
-    if (__atomic_load_n(&box->done_seq, __ATOMIC_ACQUIRE) == seq) break;
+    if (answered()) break;
     if ((spin & 1023u) == 0) {
       const bool dead = !__atomic_load_n(&box->alive, __ATOMIC_ACQUIRE);
       if (dead || std::chrono::steady_clock::now() - t0 > std::chrono::seconds(2)) {
-        if (dead && __atomic_load_n(&box->done_seq, __ATOMIC_ACQUIRE) == seq) break;
+        if (dead && answered()) break;
         DeviceGuard g(h->device);
         const cudaError_t e = cudaStreamQuery(h->res_stream);
         h->last_err = dead ? "resident warp exited before answering"
@@ -1628,7 +1640,7 @@ mcl_status_t mcl_resident_map(mcl_mapper_t* h, uint64_t epochs, const uint64_t* 
       }
     }
   }
-  const uint32_t status = __atomic_load_n(&box->status, __ATOMIC_RELAXED);
+  const uint32_t status = (uint32_t)(rec[0] >> 16) & 0xffffu;
   if (status & mcl::kFlagRange) {
     h->last_err = "a cost entry >= 2^48";
     return MCL_E_RANGE;
@@ -1637,9 +1649,16 @@ mcl_status_t mcl_resident_map(mcl_mapper_t* h, uint64_t epochs, const uint64_t* 
     h->last_err = "resident mapper: bad request";
     return MCL_E_INVAL;
   }
-  std::memcpy(mapping_index, base + off_i, epochs * 8);
-  std::memcpy(makespan, base + off_m, epochs * 8);
-  if (mapping) std::memcpy(mapping, base + off_p, epochs * a.Q);
+  const uint32_t b = a.D <= 1 ? 0u : 32u - (uint32_t)__builtin_clz(a.D - 1);
+  const uint32_t dmask = (1u << b) - 1u;
+  for (uint64_t e = 0; e < epochs; ++e) {
+    mapping_index[e] = rec[3 * e] & 0xffffu;
+    makespan[e] = rec[3 * e + 1] & ((1ull << 53) - 1);
+    if (mapping) {  // the kernel's digits, unpacked into one byte per queue
+      const uint32_t packed = (uint32_t)rec[3 * e + 2];
+      for (uint32_t q = 0; q < a.Q; ++q) mapping[e * a.Q + q] = (uint8_t)((packed >> (q * b)) & dmask);
+    }
+  }
   return MCL_OK;
 }
 
@@ -1647,8 +1666,7 @@ mcl_status_t mcl_resident_map(mcl_mapper_t* h, uint64_t epochs, const uint64_t* 
 // measurement builds only: the resident warp's timestamps of its last request
 int mcl_resident_trace(mcl_mapper_t* h, uint64_t out[4]) {
   if (!h || !h->res_mem) return -1;
-  for (int i = 0; i < 3; ++i) out[i] = __atomic_load_n(&res_box(h)->trace[i], __ATOMIC_RELAXED);
-  out[3] = out[2];
+  for (int i = 0; i < 4; ++i) out[i] = __atomic_load_n(&res_box(h)->trace[i], __ATOMIC_RELAXED);
   return 0;
 }
 #endif

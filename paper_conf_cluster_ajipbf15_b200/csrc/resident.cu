@@ -37,6 +37,9 @@ __device__ __forceinline__ uint64_t ld_relaxed_sys64(const uint64_t* p) {
   asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ void st_relaxed_sys64(uint64_t* p, uint64_t v) {
+  asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
 __device__ __forceinline__ uint64_t now_ns() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -128,8 +131,8 @@ __global__ void __launch_bounds__(32) resident_kernel(ResidentArgs a) {
     uint32_t quit = 0;
     if (lane == 0) {
       // one acquire load of the request word at a time: measured, several relaxed loads
-      // in flight (4 or 8, staggered) or a pause between polls only add latency
-      // (SS7, resident mapper)
+      // in flight (4 or 8, staggered), a pause between polls, or polling tagged inputs
+      // together with the request word only add latency (SS7, resident mapper)
       for (;;) {
         req = ld_acquire_sys64(&box->req);
         if (req >> 63) {
@@ -159,7 +162,7 @@ __global__ void __launch_bounds__(32) resident_kernel(ResidentArgs a) {
 #endif
     // ---- inputs, read in place from host memory after the acquire (a1: C = K + X) ----
     uint32_t status = 0;
-    if (E > a.cap) status |= kFlagBadModel;
+    if (E > a.cap || E == 0) status |= kFlagBadModel;
     const uint32_t n = (E <= a.cap ? E : 0u) * QD;
     bool bad = false;
     for (uint32_t i0 = lane; i0 < n; i0 += 4 * 32) {  // 8 loads in flight per lane (PCIe)
@@ -182,35 +185,34 @@ __global__ void __launch_bounds__(32) resident_kernel(ResidentArgs a) {
 #ifdef MCL_RESIDENT_TRACE
     const uint64_t tr1 = now_ns();
 #endif
-    if (status == 0) {
-      for (uint32_t e = 0; e < E; ++e) {
-        uint64_t ms;
-        uint32_t idx;
-        score_epoch<QT, DT>(sC + (size_t)e * QD, Q, D, N, sL, ms, idx);
-        if (lane == 0) {
-          a.index[e] = idx;
-          a.makespan[e] = ms;
+    // digit width b: the smallest b with D <= 2^b (0 for D = 1); Q * b <= 16 here
+    const uint32_t b = D <= 1 ? 0u : 32u - __clz(D - 1);
+    for (uint32_t e = 0; e < (status == 0 ? E : 1u); ++e) {
+      uint64_t ms = 0;
+      uint32_t idx = 0;
+      if (status == 0) score_epoch<QT, DT>(sC + (size_t)e * QD, Q, D, N, sL, ms, idx);
+      uint64_t* rec = a.rec + (size_t)e * kResidentRecWords;
+      if (lane == 0) {
+        st_relaxed_sys64(rec + 0, ((uint64_t)seq << 32) | ((uint64_t)status << 16) | idx);
+      } else if (lane == 1) {
+        st_relaxed_sys64(rec + 1, ((uint64_t)(seq & 0x7ffu) << 53) | ms);
+      } else if (lane == 2) {  // a7: digits of the index, queue 0 most significant
+        uint32_t rest = idx, packed = 0;
+        for (int q = (int)Q - 1; q >= 0; --q) {
+          packed |= (rest % D) << (q * b);
+          rest /= D;
         }
-        if (lane < (int)Q) {  // a7: digits of the index, queue 0 most significant
-          uint32_t rest = idx;
-          for (int q = (int)Q - 1; q > lane; --q) rest /= D;
-          a.mapping[(size_t)e * Q + lane] = (uint8_t)(rest % D);
-        }
+        st_relaxed_sys64(rec + 2, ((uint64_t)seq << 32) | packed);
       }
     }
-    if (lane == 0) box->status = status;
-    // every lane's result stores, then lane 0's release of the request number: the warp
-    // barrier orders them before it, and a release at system scope is cumulative, so the
-    // host's acquire of done_seq sees all of them
-    __syncwarp();
-    if (lane == 0) {
 #ifdef MCL_RESIDENT_TRACE
+    if (lane == 0) {
       box->trace[0] = tr0;
       box->trace[1] = tr1;
       box->trace[2] = now_ns();
-#endif
-      st_release_sys(&box->done_seq, seq);
+      box->trace[3] = box->trace[2];
     }
+#endif
     t_idle = now_ns();
   }
 }

@@ -5,7 +5,7 @@ three public ways of calling the mapper (measurement only; prints one JSON line 
   launch_dev   : mcl_map_queues with device-resident buffers (launch + sync per call)
 Wall-clock per call from Python (ctypes), median of rounds of 500 calls, results checked.
 
-    python scripts/resident_latency.py [calls]
+    python scripts/resident_latency.py [calls] [--lib path/to/libmcl.so]
 """
 import json
 import os
@@ -18,9 +18,14 @@ sys.path.insert(0, ROOT)
 import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
-from paper_conf_cluster_ajipbf15_b200 import Mapper, workloads  # noqa: E402
+from paper_conf_cluster_ajipbf15_b200 import Mapper, mcl, workloads  # noqa: E402
 
-calls = int(sys.argv[1]) if len(sys.argv) > 1 else 500
+argv = sys.argv[1:]
+if "--lib" in argv:
+    i = argv.index("--lib")
+    mcl.load_library(os.path.abspath(argv[i + 1]))
+    del argv[i:i + 2]
+calls = int(argv[0]) if argv else 500
 K, X = workloads.make("cfg1")
 Kp, Xp = torch.from_numpy(K).pin_memory(), torch.from_numpy(X).pin_memory()
 Kd, Xd = Kp.cuda(), Xp.cuda()
@@ -49,7 +54,7 @@ with Mapper(0) as m:
         m.resident_map(Kn, Xn, out=r_out)
         assert r_out[0][0] == ref[0][0] and r_out[2][0] == ref[2][0] and (r_out[1] == ref[1]).all()
         med, best = per_call(lambda: m.resident_map(Kn, Xn, out=r_out))
-        out.append({"measure": "cfg1 decision latency", "path": "resident", "us_per_call_median": med,
+        out.append({"measure": "cfg1 decision latency", "path": "resident", "lib": os.path.basename(mcl.LIB_PATH if not "--lib" in sys.argv else sys.argv[sys.argv.index("--lib") + 1]), "us_per_call_median": med,
                     "us_per_call_best_round": best})
     finally:
         m.resident_stop()

@@ -51,6 +51,6 @@ with mcl.Mapper(0) as m:
     empty = (time.perf_counter() - t0) / 1000 * 1e6
 med = [statistics.median(c) for c in zip(*rows)]
 print(json.dumps({"measure": "resident phases (us, median of 2900 calls)", "host_call": med[0],
-                  "inputs_read": med[1], "score": med[2], "fence_system": med[3],
+                  "inputs_read": med[1], "score": med[2], "release_store": med[3],
                   "unaccounted (poll + done + host)": med[0] - sum(med[1:]),
                   "bare_ctypes_call": statistics.median(raw), "ctypes_noop_call": empty}))

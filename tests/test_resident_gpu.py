@@ -134,3 +134,17 @@ def test_resident_errors(torch_cuda):
                 m.resident_start(4, 3)  # already started
         finally:
             m.resident_stop()
+
+
+def test_resident_close_without_stop(torch_cuda):
+    """Closing the handle while the warp is resident stops it (mcl_mapper_destroy); device-
+    wide synchronisation afterwards returns at once."""
+    torch = torch_cuda
+    K, X = workloads.random_tables(13, 2, 4, 3, hi=1 << 16)
+    m = Mapper(0)
+    m.resident_start(4, 3, max_epochs=2, idle_ms=60000)
+    check(m.resident_map(K, X), K, X, "before close")
+    m.close()
+    t0 = time.perf_counter()
+    torch.cuda.synchronize()
+    assert time.perf_counter() - t0 < 5.0
