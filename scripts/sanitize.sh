@@ -28,3 +28,8 @@ for tool in memcheck racecheck synccheck; do
   timeout 1200 $CS --tool $tool --error-exitcode 9 python scripts/sanitize_cases.py > gpurun_out/sanitize_${tool}_r02.log 2>&1
   echo "$tool r02 cases rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY' gpurun_out/sanitize_${tool}_r02.log | tail -1)"
 done
+# resident mapper (one warp polling a pinned host mailbox; tagged result records)
+timeout 600 $CS --tool memcheck --error-exitcode 9 python -m pytest tests/test_resident_gpu.py -m gpu -q -p no:cacheprovider -k "errors or 4-3 or back_to_back" > gpurun_out/sanitize_memcheck_resident.log 2>&1
+echo "memcheck resident rc=$? $(grep -E 'ERROR SUMMARY' gpurun_out/sanitize_memcheck_resident.log | tail -1) $(grep -E 'passed|failed' gpurun_out/sanitize_memcheck_resident.log | tail -1)"
+timeout 600 $CS --tool racecheck --error-exitcode 9 python -m pytest tests/test_resident_gpu.py -m gpu -q -p no:cacheprovider -k "4-3" > gpurun_out/sanitize_racecheck_resident.log 2>&1
+echo "racecheck resident rc=$? $(grep -E 'RACECHECK SUMMARY' gpurun_out/sanitize_racecheck_resident.log | tail -1) $(grep -E 'passed|failed' gpurun_out/sanitize_racecheck_resident.log | tail -1)"
