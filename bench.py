@@ -516,7 +516,9 @@ def measure(ctx, name):
     # ---- decision-sized searches: the same through the resident mapper (mcl_resident_*,
     # one warp left on the GPU serving a pinned host mailbox; no launch per call) ----
     e2e_launch_s, res_s = e2e_s, None
-    if resident_eligible(w) and not sharded:
+    if resident_eligible(w) and not sharded and not os.environ.get("MCL_BENCH_NO_RESIDENT"):
+        # (MCL_BENCH_NO_RESIDENT=1 under profilers that serialise launches: a resident
+        # kernel then only returns after its idle timeout)
         Kn, Xn = Kh.numpy(), Xh.numpy()
         outs = (ih.numpy(), ph.numpy(), mh.numpy())
         mapper.resident_start(Q, D, max_epochs=E)

@@ -5,7 +5,7 @@ cd "${GRAFT_REPO_ROOT:-$(dirname "$0")/..}"
 mkdir -p gpurun_out
 NCU=/usr/local/cuda/bin/ncu
 # launch list of the default bench command (every config): cold-cache, serialised per launch
-timeout 900 $NCU --metrics gpu__time_duration.sum --clock-control none --csv \
+MCL_BENCH_NO_RESIDENT=1 timeout 900 $NCU --metrics gpu__time_duration.sum --clock-control none --csv \
     --log-file gpurun_out/launches_default.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline \
     > gpurun_out/launches_default.log 2>&1
 echo "launch list rc=$?"
