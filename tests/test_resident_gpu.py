@@ -148,3 +148,24 @@ def test_resident_close_without_stop(torch_cuda):
     t0 = time.perf_counter()
     torch.cuda.synchronize()
     assert time.perf_counter() - t0 < 5.0
+
+
+def test_resident_beside_searches(torch_cuda):
+    """A resident warp and the handle's ordinary searches at the same time: decisions through
+    the mailbox between (and during) full-GPU searches on the handle's stream, all exact."""
+    torch = torch_cuda
+    Kb, Xb = workloads.random_tables(21, 1, 10, 6, hi=1 << 20)  # 6^10 = 6e7 mappings
+    want_b = oracle.oracle_map(Kb, Xb)
+    Ks, Xs = workloads.random_tables(22, 50, 4, 3, hi=1 << 16)
+    want_s = oracle.oracle_map(Ks, Xs)
+    Kd, Xd = torch.from_numpy(Kb).cuda(), torch.from_numpy(Xb).cuda()
+    with Mapper(0) as m, Mapper(0) as r:
+        r.resident_start(4, 3)
+        try:
+            for e in range(Ks.shape[0]):
+                gi, gmp, gms = m.map_queues(Kd, Xd)
+                assert int(gi[0]) == want_b[0][0] and int(gms[0]) == want_b[1][0]
+                ri, rmp, rms = r.resident_map(Ks[e], Xs[e])
+                assert ri[0] == want_s[0][e] and rms[0] == want_s[1][e] and (rmp[0] == want_s[2][e]).all()
+        finally:
+            r.resident_stop()
