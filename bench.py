@@ -563,7 +563,9 @@ def measure(ctx, name):
         "clocks": clocks,
         "gpu_launches": launches,
         "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": K.nbytes + X.nbytes,
-                "d2h_bytes_per_step": E * (8 + 8 + Q), "ms_per_step": e2e_s * 1e3,
+                # resident: one three-word record per epoch (kernels.h ResidentArgs)
+                "d2h_bytes_per_step": E * 24 if res_s is not None else E * (8 + 8 + Q),
+                "ms_per_step": e2e_s * 1e3,
                 "api": ("mcl_resident_map (resident warp; inputs read in place over PCIe, results "
                         "written back to the pinned mailbox)" if res_s is not None
                         else "mcl_map_queues on pinned host buffers"),
