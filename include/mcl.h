@@ -334,7 +334,8 @@ const char* mcl_last_error_string(const mcl_mapper_t* h);
  *             5 = register-blocked u32 over a flattened (epoch, block) space,
  *             6 = branch and bound (mcl_map_queues_pruned), 7 = warp-per-epoch batched u32,
  *             8 = register-blocked u32, one-CTA-per-SM build (single epochs, D = 5),
- *             9 / 10 = mixed-radix constrained search over the feasible mappings, u32 / u64)
+ *             9 / 10 = mixed-radix constrained search over the feasible mappings, u32 / u64,
+ *             11 = the same, one warp per epoch, for batches of constrained epochs)
  *   info[1] = number of kernels launched by the call, info[2] = CTAs of the main kernel,
  *   info[3] = threads per CTA, info[4] = 1 if an NCCL all-reduce ran, 2 if the fused peer
  *   exchange ran, info[5] = index bits of the packed key, info[6] = 1 if the two-step

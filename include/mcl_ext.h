@@ -50,8 +50,10 @@ mcl_status_t mcl_probe_int_rate(int device, int op, double* lane_ops_per_s,
    epoch batched kernel (unconstrained single-GPU batches of the shapes it is instantiated
    for; chosen automatically from one full wave of epochs), 8 = mixed-radix constrained
    kernel (calls with eligible-device masks, 2 <= D <= 8, Q >= 3; the automatic choice for
-   them -- force 1 for the INF-masked full-space blocked kernel instead). A path that does
-   not support (Q, D) or the handle's sharding makes the call fail with MCL_E_INVAL. */
+   them -- force 1 for the INF-masked full-space blocked kernel instead), 9 = its warp-per-
+   epoch form for batches (single GPU, at most 2^16 reduced blocks per epoch; chosen
+   automatically from four epochs per SM). A path that does not support (Q, D) or the
+   handle's sharding makes the call fail with MCL_E_INVAL. */
 mcl_status_t mcl_force_path(mcl_mapper_t* h, int path);
 
 /* Pipelined staging of host-resident batches. When every cost table and output of an

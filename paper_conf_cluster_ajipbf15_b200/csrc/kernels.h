@@ -133,6 +133,9 @@ cudaError_t launch_blocked(const BlockedArgs& a, bool wide, dim3 grid, int threa
 // memory layout as the blocked kernel (rlo / rhi unused: the shard is a.rank / a.world of
 // each epoch's reduced block space).
 int mixed_ctas_per_sm(uint32_t D, bool wide, int threads, size_t smem);
+// Batches of constrained epochs, one warp per epoch (u32 loads only; kFlagNeedU64 -> the
+// 64-bit CTA kernel). grid_out: CTAs of kMixedWarps warps.
+cudaError_t launch_mixed_warp(const BlockedArgs& a, int num_sms, cudaStream_t st, int* grid_out);
 cudaError_t launch_mixed(const BlockedArgs& a, bool wide, dim3 grid, int threads, size_t smem,
                          cudaStream_t st);
 

@@ -408,7 +408,7 @@ mcl_status_t mcl_set_pipeline_chunks(mcl_mapper_t* h, int chunks) {
 }
 
 mcl_status_t mcl_force_path(mcl_mapper_t* h, int path) {
-  if (!h || path < 0 || path > 8) return MCL_E_INVAL;
+  if (!h || path < 0 || path > 9) return MCL_E_INVAL;
   h->force_path = path;
   return MCL_OK;
 }
@@ -813,15 +813,19 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
   const bool batch_ok = !shard_mode && !multi && !constrained && mcl::batch_supported(Q, D);
   // eligible-device masks: the mixed-radix kernel enumerates the feasible mappings only
   const bool mixed_ok = eligible != nullptr && mcl::blocked_supported(Q, D);
+  // batches of small constrained epochs: one warp per epoch (at most 2^16 reduced blocks of
+  // D^3 leaves per epoch, one resident wave of CTAs filled)
+  const bool mixed_warp_ok = mixed_ok && !shard_mode && !multi && N / ((uint64_t)D * D * D) <= (1ull << 16);
   if (!shard_mode && !multi && !constrained && mcl::small_supported(Q, D)) path = 4;
   else if (batch_ok && epochs >= (uint64_t)h->num_sms * 4) path = 7;
+  else if (mixed_warp_ok && epochs >= (uint64_t)h->num_sms * 4) path = 11;
   else if (mixed_ok) path = 9;
   else if (mcl::blocked_supported(Q, D)) path = 1;
   else path = 3;
   if (h->force_path && h->force_path != 6) {  // 6 only affects mcl_map_queues_pruned
     const int f = h->force_path;
     const bool ok = (f == 3) || ((f == 1 || f == 2) && mcl::blocked_supported(Q, D)) ||
-                    (f == 8 && mixed_ok) ||
+                    (f == 8 && mixed_ok) || (f == 9 && mixed_warp_ok) ||
                     (f == 7 && batch_ok) ||
                     (f == 5 && epochs > 1 && !shard_mode && !multi && !constrained &&
                      mcl::flat_supported(Q, D, mcl::index_bits_host(N))) ||
@@ -830,7 +834,9 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
       h->last_err = "forced kernel path does not support this shape / sharding";
       return MCL_E_INVAL;
     }
-    path = (f == 5) ? 1 : (f == 8 ? 9 : f);  // 5 = the flattened form of the blocked u32 kernel
+    // 5 = the flattened form of the blocked u32 kernel; 8 / 9 = the mixed-radix CTA / warp
+    // kernels (paths 9 / 11)
+    path = (f == 5) ? 1 : (f == 8 ? 9 : (f == 9 ? 11 : f));
   }
 
   int nlaunch = 0;
@@ -872,6 +878,16 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
       grid.x = gx;
       threads = 32;
       path = 5;
+    } else if (path == 11) {
+      mcl::BlockedArgs a{};
+      a.Q = Q; a.D = D; a.E = epochs; a.K = K; a.X = X;
+      a.out = out; a.ibits = ibits; a.flags = h->flags_dev; a.one = 1;
+      a.base = Bd; a.elig = Ed;
+      a.world = 1;
+      int gx = 0;
+      MCL_CUDA(h, mcl::launch_mixed_warp(a, h->num_sms, s, &gx), "search_mixed_warp launch");
+      grid.x = gx;
+      threads = 128;
     } else if (path == 9 || path == 10) {
       // constrained: mixed-radix search of the feasible mappings (search_mixed.cu); the
       // shard is taken per epoch on the device from the reduced block count
@@ -1019,11 +1035,11 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
       h->info[6] = (flags & mcl::kFlagTwoStep) ? 1 : 0;
     }
     if (flags & mcl::kFlagNeedU64) {  // some epoch's bound needs 64-bit loads: rerun the wide kernel
-      if (path != 1 && path != 5 && path != 7 && path != 9) {
+      if (path != 1 && path != 5 && path != 7 && path != 9 && path != 11) {
         h->last_err = "internal: 64-bit request from a 64-bit kernel";
         return MCL_E_CUDA;
       }
-      path = (path == 9) ? 10 : 2;
+      path = (path == 9 || path == 11) ? 10 : 2;
       continue;
     }
     if (use_nccl && (flags & mcl::kFlagNoPack)) {  // key does not pack: two-step lexicographic all-reduce

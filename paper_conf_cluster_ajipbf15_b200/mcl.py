@@ -18,7 +18,8 @@ LIB_PATH = os.path.join(_HERE, "libmcl.so")
 
 MCL_OK, MCL_E_INVAL, MCL_E_RANGE, MCL_E_CUDA, MCL_E_NCCL, MCL_E_NOMEM = 0, -1, -2, -3, -4, -5
 PATH_NAMES = {1: "blocked_u32", 2: "blocked_u64", 3: "generic", 4: "small_batched", 5: "flat_u32",
-              6: "pruned", 7: "batch_u32", 8: "blocked_u32_lean", 9: "mixed_u32", 10: "mixed_u64"}
+              6: "pruned", 7: "batch_u32", 8: "blocked_u32_lean", 9: "mixed_u32", 10: "mixed_u64",
+              11: "mixed_warp_u32"}
 
 # Every symbol the headers declare (tests check the library exports all of them).
 EXPORTED = [
@@ -648,7 +649,8 @@ class Mapper:
         """Testing aid: 0 auto, 1 blocked u32 (CTA per epoch), 2 blocked u64, 3 generic,
         4 small batched, 5 flattened batched blocked u32, 6 branch-and-bound kernel in
         map_queues_pruned even for small index spaces, 7 warp-per-epoch batched kernel,
-        8 mixed-radix constrained kernel (the default for calls with eligible masks)."""
+        8 mixed-radix constrained kernel (the default for calls with eligible masks), 9 its
+        warp-per-epoch form (the default for batches of them)."""
         st = load_library().mcl_force_path(self.handle, path)
         if st != MCL_OK:
             raise MclError(st, "mcl_force_path")

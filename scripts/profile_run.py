@@ -17,9 +17,11 @@ K, X = workloads.make(name.rstrip("c"), **kw)
 Kd, Xd = torch.from_numpy(K).cuda(), torch.from_numpy(X).cuda()
 if constrained:
     base, elig = workloads.constraints(77, *K.shape)
-    elig[:] = 0
-    elig[:, [1, 5, 10]] = [1 << 3, 1 << 0, 1 << 6]
-    elig[:, [2, 7, 11]] = [0b00110110, 0b11000001, 0b0111]
+    if K.shape[1] == 12:  # cfg5c: 3 pinned + 3 masked queues
+        elig[:] = 0
+        elig[:, [1, 5, 10]] = [1 << 3, 1 << 0, 1 << 6]
+        elig[:, [2, 7, 11]] = [0b00110110, 0b11000001, 0b0111]
+    # else (e.g. cfg2c): 25 % pinned + 25 % masked queues per epoch (workloads.constraints)
     Bd, Ed = torch.from_numpy(base).cuda(), torch.from_numpy(elig).cuda()
 with Mapper(0) as m:
     for _ in range(reps):

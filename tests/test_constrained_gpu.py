@@ -347,5 +347,66 @@ def test_mixed_radix_batches_beyond_one_wave(torch_cuda, mapper):
     K, X = workloads.random_tables(123, E, Q, D, hi=1 << 18)
     base, elig = random_constraints(124, E, Q, D, pin_frac=0.3)
     want = oracle.oracle_map_constrained(K, X, base, elig)
-    check(run(torch, mapper, K, X, base, elig), want, "mixed E=700")
+    check(run(torch, mapper, K, X, base, elig, 8), want, "mixed E=700")
     assert mapper.launch_info()["path"] == "mixed_u32"
+
+
+# ------------------------------- mixed radix, one warp per epoch (batched constrained) ----
+@pytest.mark.parametrize("Q,D", [(3, 2), (4, 3), (5, 4), (6, 5), (7, 3), (6, 6), (5, 7), (5, 8), (8, 4), (9, 3)])
+def test_mixed_warp_random_and_ties(torch_cuda, mapper, Q, D):
+    """The warp-per-epoch mixed-radix kernel (forced, path 9) == the constrained oracle,
+    bit-exact, on random and tie-heavy tables with pins, masks, bits >= D and zero masks."""
+    torch = torch_cuda
+    E = 70
+    for seed, maker in ((Q * 100 + D + 5, workloads.random_tables), (Q * 100 + D + 6, workloads.small_int_tables)):
+        K, X = maker(seed, E, Q, D)
+        base, elig = random_constraints(seed + 9, E, Q, D, pin_frac=0.35)
+        elig[::5, 0] = np.where(elig[::5, 0] != 0, elig[::5, 0] | np.uint16(1 << 15), 0)
+        elig[1::7, :] = 0
+        for b in (base, None):
+            want = oracle.oracle_map_constrained(K, X, b, elig)
+            check(run(torch, mapper, K, X, b, elig, 9), want, f"warp Q={Q} D={D} {maker.__name__}")
+            assert mapper.launch_info()["path"] == "mixed_warp_u32"
+
+
+@pytest.mark.parametrize("Q,D", [(4, 3), (6, 4), (9, 5), (8, 8)])
+def test_mixed_warp_pins_everywhere(torch_cuda, mapper, Q, D):
+    """Every pinned-queue count on the warp kernel, including all queues pinned."""
+    torch = torch_cuda
+    rng = np.random.default_rng(Q * D + 1)
+    K, X = workloads.random_tables(Q + D + 1, Q + 1, Q, D, hi=1 << 16)
+    base = rng.integers(0, 1 << 16, size=(Q + 1, D), dtype=np.uint64)
+    elig = np.zeros((Q + 1, Q), np.uint16)
+    for e in range(Q + 1):
+        pin = rng.permutation(Q)[:e]
+        elig[e, pin] = (1 << rng.integers(0, D, size=e)).astype(np.uint16)
+    want = oracle.oracle_map_constrained(K, X, base, elig)
+    check(run(torch, mapper, K, X, base, elig, 9), want, f"warp pins Q={Q} D={D}")
+
+
+def test_mixed_warp_auto_batch_u64_and_errors(torch_cuda, mapper):
+    """A cfg2-shaped constrained batch (8 x 4, 25 % pinned + 25 % masked) takes the warp
+    kernel automatically; an epoch whose bound needs 64 bits reruns the call on the 64-bit
+    CTA kernel; input errors raise as on every path."""
+    torch = torch_cuda
+    E, Q, D = 1000, 8, 4
+    K, X = workloads.random_tables(131, E, Q, D, hi=1 << 18)
+    base, elig = workloads.constraints(132, E, Q, D, pin_frac=0.25, mask_frac=0.25)
+    want = oracle.oracle_map_constrained(K, X, base, elig)
+    check(run(torch, mapper, K, X, base, elig), want, "auto warp")
+    assert mapper.launch_info()["path"] == "mixed_warp_u32"
+    big = base.copy()
+    big[E // 2] += np.uint64(1 << 40)  # one epoch over 2^32: the whole call reruns wide
+    want_big = oracle.oracle_map_constrained(K, X, big, elig)
+    check(run(torch, mapper, K, X, big, elig), want_big, "auto warp -> u64")
+    assert mapper.launch_info()["path"] == "mixed_u64"
+    Kr = K.copy()
+    Kr[E - 1, 3, 2] = 1 << 48
+    with pytest.raises(MclError) as e:
+        run(torch, mapper, Kr, X, base, elig)
+    assert e.value.status == MCL_E_RANGE
+    bad = elig.copy()
+    bad[7, 2] = 1 << 5  # no eligible device below D
+    with pytest.raises(MclError) as e:
+        run(torch, mapper, K, X, base, bad)
+    assert e.value.status == MCL_E_INVAL
