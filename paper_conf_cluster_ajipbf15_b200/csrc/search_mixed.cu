@@ -38,10 +38,24 @@ struct MixedTab {
   uint64_t nb;               // blocks of D^3 leaves = prod_{p < O} radix[p]
   uint64_t pin_idx;          // sum over pinned queues of d_q * D^(Q-1-q)
   uint8_t radix[kMaxQueues];
+  uint32_t rmul[kMaxQueues];             // ceil(2^20 / radix[p]): division of indices < 2^16
   uint8_t dev[kMaxQueues][kMaxDevices];  // digit -> device of reduced queue p
   uint64_t w[kMaxQueues];                // D^(Q-1-q) of reduced queue p (0 = virtual)
   int8_t orig[kMaxQueues];               // original queue of reduced queue p (-1 = virtual)
 };
+
+// q = x / radix[p] and x - q * radix[p]. Block indices of the warp kernel (I = 32 bits) are
+// below 2^16 and radices at most 16, so q = (x * ceil(2^20 / r)) >> 20 exactly (the error
+// x * (m r - 2^20) / (r 2^20) < 2^16 * 16 / (r 2^20) <= 1 / r); 64-bit indices divide.
+template <typename I>
+__device__ __forceinline__ I div_radix(I x, const MixedTab& mt, int p, uint32_t* rem) {
+  const uint32_t r = mt.radix[p];
+  I q;
+  if constexpr (sizeof(I) == 4) q = (I)(((uint64_t)x * mt.rmul[p]) >> 20);
+  else q = x / r;
+  *rem = (uint32_t)(x - q * r);
+  return q;
+}
 
 // Decode reduced block `blk` into its outer digits (radix[p], p = O-1 fastest) and return
 // the prefix load vector base0 + sum_p V[p][t_p]; optionally the full-index part of the
@@ -54,9 +68,8 @@ __device__ __forceinline__ void mixed_prefix(T (&P)[D], I blk, const MixedTab& m
   for (int d = 0; d < D; ++d) P[d] = B0[d];
   uint64_t f = 0;
   for (int p = (int)mt.O - 1; p >= 0; --p) {
-    const uint32_t r = mt.radix[p];
-    const uint32_t t = (uint32_t)(blk % r);
-    blk /= r;
+    uint32_t t;
+    blk = div_radix<I>(blk, mt, p, &t);
     f += (uint64_t)mt.dev[p][t] * mt.w[p];
     const T* v = V + ((size_t)p * D + t) * D;
 #pragma unroll
@@ -70,9 +83,9 @@ template <int D, typename I = uint64_t>
 __device__ __forceinline__ uint64_t mixed_full_index(I blk, uint32_t leaf, const MixedTab& mt) {
   uint64_t f = mt.pin_idx;
   for (int p = (int)mt.O - 1; p >= 0; --p) {
-    const uint32_t r = mt.radix[p];
-    f += (uint64_t)mt.dev[p][blk % r] * mt.w[p];
-    blk /= r;
+    uint32_t t;
+    blk = div_radix<I>(blk, mt, p, &t);
+    f += (uint64_t)mt.dev[p][t] * mt.w[p];
   }
   const uint32_t i = leaf / (D * D), j = (leaf / D) % D, k = leaf % D;
   return f + i * mt.w[mt.O] + j * mt.w[mt.O + 1] + k * mt.w[mt.O + 2];
@@ -136,7 +149,10 @@ __device__ __forceinline__ void mixed_build(MixedTab& mt, const uint64_t* C64, u
       for (uint32_t d = 0; d < D; ++d) mt.dev[mt.O - 1][d] = (uint8_t)d;
     }
     uint64_t nb = 1;
-    for (uint32_t p = 0; p < mt.O; ++p) nb *= mt.radix[p];
+    for (uint32_t p = 0; p < mt.O; ++p) {
+      nb *= mt.radix[p];
+      mt.rmul[p] = ((1u << 20) + mt.radix[p] - 1u) / mt.radix[p];
+    }
     mt.nb = nb;
     mt.pin_idx = pin;
     // bound of every leaf the kernel forms: max base' + sum of the reduced rows' maxima
@@ -209,14 +225,13 @@ __device__ __forceinline__ void walk_mixed(const MixedTab& mt, const T* __restri
   const T* Vx = V + (size_t)(O - 1) * D * D;
   const T* c4 = in + 7 * D;
   const uint32_t rx = mt.radix[O - 1];
-  uint32_t x = (uint32_t)(b0 % rx);
-  I hi = b0 / rx;
+  uint32_t x;
+  I hi = div_radix<I>(b0, mt, O - 1, &x);
   T base[D];
   load_vec<T, D>(base, B0);
   for (int p = O - 2; p >= 0; --p) {
-    const uint32_t r = mt.radix[p];
-    const uint32_t t = (uint32_t)(hi % r);
-    hi /= r;
+    uint32_t t;
+    hi = div_radix<I>(hi, mt, p, &t);
     dig[p * nthr + tid] = (uint8_t)t;
     const T* v = V + ((size_t)p * D + t) * D;
 #pragma unroll
@@ -530,7 +545,17 @@ __global__ void __launch_bounds__(32 * kMixedWarps, D <= 5 ? 4 : 2) search_mixed
       const T bt = (T)(key >> 32);
       c = Cand{(uint64_t)bt, mixed_span_first_warp<T, D, uint32_t>(bb, span, mt, V, base0, in, bt, one)};
     }
-    if (lane == 0) write_epoch(a.out, e, Q, D, a.ibits, c, a.flags, feas);
+    // a7: outputs, digits of the index in parallel (queue q on lane q, D a constant)
+    if (c.ms != kNone && c.ms > feas) c = Cand{kNone, kNone};
+    if (lane == 0) {
+      a.out.index[e] = c.idx;
+      a.out.makespan[e] = c.ms;
+    }
+    if (a.out.mapping && (uint32_t)lane < Q) {
+      uint64_t rest = c.idx;
+      for (uint32_t q = Q - 1; q > (uint32_t)lane; --q) rest /= D;
+      a.out.mapping[e * Q + lane] = (c.idx == kNone) ? 0xFF : (uint8_t)(rest % D);
+    }
     __syncwarp();  // the tables are rebuilt for the next epoch
   }
 }
