@@ -1,5 +1,6 @@
 """Small runs of the round-2 paths for compute-sanitizer (memcheck / racecheck / synccheck):
-the mixed-radix constrained kernel (single epoch spread over CTAs, batched, sharded, u64),
+the mixed-radix constrained kernels (single epoch spread over CTAs, batched, one warp per
+epoch, sharded, u64),
 the blocked kernel's packed-key merge of a split epoch, the static policy and scoring
 kernels, per-socket cost tables, and zero-copy small calls on pinned host buffers.
 
@@ -28,6 +29,13 @@ with Mapper(0) as m:
     base, elig = workloads.constraints(2, 24, 8, 4)
     m.map_queues_constrained(dev(K), dev(X), dev(base), dev(elig))
     m.map_queues_constrained(dev(K), dev(X), dev(base + np.uint64(1 << 40)), dev(elig))
+    # the warp-per-epoch mixed-radix kernel (forced; a batch of 40 epochs), and its u64 rerun
+    K, X = workloads.cfg2(E=40, seed=8)
+    base, elig = workloads.constraints(9, 40, 8, 4)
+    m.force_path(9)
+    m.map_queues_constrained(dev(K), dev(X), dev(base), dev(elig))
+    m.map_queues_constrained(dev(K), dev(X), dev(base + np.uint64(1 << 40)), dev(elig))
+    m.force_path(0)
     # blocked kernel, one epoch over every CTA (packed-key merge, pair rescan)
     K, X = workloads.cfg4(seed=4, Q=11)
     m.map_queues(dev(K), dev(X))
