@@ -9,9 +9,10 @@
 // request number; the warp (polling the request number over PCIe) reads the inputs in
 // place, scores every mapping (the same definition as every other path: C = K + X,
 // PAPER.md L2106-2118; loads per device, makespan = max over devices, L1048-1052; argmin
-// with the lowest index on ties), writes index / makespan / mapping digits back into the
-// mailbox and publishes the request number as done. No launch, no copy engine, no stream
-// synchronisation per decision.
+// with the lowest index on ties) and answers with one record per epoch of three words
+// (index, makespan, packed digits), each stored whole and tagged with the request number,
+// so the host accepts the answer without a fence or a separate done flag (kernels.h,
+// ResidentArgs). No launch, no copy engine, no stream synchronisation per decision.
 //
 // Shape: any Q <= 16, D <= 16 with D^Q <= 4096 (one warp; lane l scores mappings l, l + 32,
 // ... in increasing order keeping its first strict minimum, then five shuffle rounds of the
