@@ -352,7 +352,8 @@ def test_mixed_radix_batches_beyond_one_wave(torch_cuda, mapper):
 
 
 # ------------------------------- mixed radix, one warp per epoch (batched constrained) ----
-@pytest.mark.parametrize("Q,D", [(3, 2), (4, 3), (5, 4), (6, 5), (7, 3), (6, 6), (5, 7), (5, 8), (8, 4), (9, 3)])
+@pytest.mark.parametrize("Q,D", [(3, 2), (4, 3), (5, 4), (6, 5), (7, 3), (6, 6), (5, 7), (5, 8), (8, 4), (9, 3),
+                                 (12, 3), (10, 4), (18, 2)])
 def test_mixed_warp_random_and_ties(torch_cuda, mapper, Q, D):
     """The warp-per-epoch mixed-radix kernel (forced, path 9) == the constrained oracle,
     bit-exact, on random and tie-heavy tables with pins, masks, bits >= D and zero masks."""
