@@ -131,11 +131,12 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
     for (int d = 0; d < D; ++d) b[d] = add_f(b2[d], row[d], one);
   };
   // a warp's lexicographic minimum of (makespan << 32 | super-block)
+  // (two 32-bit warp reductions, REDUX: the minimum makespan, then the lowest super-block
+  // among the lanes holding it -- the same key as a 64-bit shuffle tree, in fewer steps)
   auto warp_key = [&](T best, uint32_t best_sb) {
-    uint64_t key = ((uint64_t)best << 32) | best_sb;
-#pragma unroll
-    for (int off = 16; off > 0; off >>= 1) key = min(key, __shfl_xor_sync(0xffffffffu, key, off));
-    return key;
+    const uint32_t g = __reduce_min_sync(0xffffffffu, (uint32_t)best);
+    const uint32_t sb = __reduce_min_sync(0xffffffffu, (uint32_t)best == g ? best_sb : 0xffffffffu);
+    return ((uint64_t)g << 32) | sb;
   };
   // The lowest leaf inside the winning super-block, then the outputs (a5, a7). Leaf
   // (x, i, j, k) of the super-block has offset ((x * D + i) * D + j) * D + k: lane
