@@ -68,8 +68,9 @@ KERNEL_NAMES = {"blocked_u32": "search_blocked_kernel<u32, D>",
                 "blocked_u64": "search_blocked_kernel<u64, D>",
                 "generic": "search_generic_kernel", "flat_u32": "search_flat_kernel<u32, D>",
                 "small_batched": "search_small_kernel<Q, D> / search_tiny_kernel<Q, D>",
-                "batch_u32": "search_batch_kernel<Q, D>"}
-ALU_PATHS = ("blocked_u32", "blocked_u32_lean", "blocked_u64", "generic", "flat_u32", "batch_u32")
+                "batch_u32": "search_batch_kernel<Q, D>",
+                "batch_pool_u32": "search_pool_kernel<Q, D>"}
+ALU_PATHS = ("blocked_u32", "blocked_u32_lean", "blocked_u64", "generic", "flat_u32", "batch_u32", "batch_pool_u32")
 
 
 def parse(argv=None):

@@ -335,7 +335,8 @@ const char* mcl_last_error_string(const mcl_mapper_t* h);
  *             6 = branch and bound (mcl_map_queues_pruned), 7 = warp-per-epoch batched u32,
  *             8 = register-blocked u32, one-CTA-per-SM build (single epochs, D = 5),
  *             9 / 10 = mixed-radix constrained search over the feasible mappings, u32 / u64,
- *             11 = the same, one warp per epoch, for batches of constrained epochs)
+ *             11 = the same, one warp per epoch, for batches of constrained epochs,
+ *             12 = batched u32 with one 16-warp CTA per SM sharing its epochs in parts)
  *   info[1] = number of kernels launched by the call, info[2] = CTAs of the main kernel,
  *   info[3] = threads per CTA, info[4] = 1 if an NCCL all-reduce ran, 2 if the fused peer
  *   exchange ran, info[5] = index bits of the packed key, info[6] = 1 if the two-step

@@ -250,7 +250,8 @@ struct BatchArgs {
   uint64_t e_full;    // set by launch_batch: epochs searched by one warp (whole waves)
 };
 bool batch_supported(uint32_t Q, uint32_t D);
-cudaError_t launch_batch(const BatchArgs& a, int num_sms, cudaStream_t st, int* grid_out);
+// *pooled = true when the SM-pooled form ran (one 16-warp CTA per SM, sub-epoch parts)
+cudaError_t launch_batch(const BatchArgs& a, int num_sms, cudaStream_t st, int* grid_out, bool* pooled);
 
 // Small batched search (search_small.cu): one thread per epoch, tiles staged in shared
 // memory by cp.async.bulk (TMA bulk copy). Instantiated for a few (Q, D) shapes.

@@ -846,13 +846,14 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
     dim3 grid(1, 1, 1);
     int threads = 0;
     bool lean_ran = false;  // the one-CTA-per-SM build of the blocked kernel (reported as path 8)
+    bool pool_ran = false;  // the SM-pooled batch kernel (reported as path 12)
     if (h->timing) MCL_CUDA(h, record_start(h, s), "cudaEventRecord(start)");
     if (path == 7) {
       mcl::BatchArgs a{Q, D, epochs, K, X, o_idx, o_ms, o_map, h->flags_dev, 1u};
       int gx = 0;
-      MCL_CUDA(h, mcl::launch_batch(a, h->num_sms, s, &gx), "search_batch launch");
+      MCL_CUDA(h, mcl::launch_batch(a, h->num_sms, s, &gx, &pool_ran), "search_batch launch");
       grid.x = gx;
-      threads = 128;
+      threads = pool_ran ? 512 : 128;
     } else if (path == 4) {
       mcl::SmallArgs a{Q, D, epochs, K, X, o_idx, o_ms, o_map, h->flags_dev};
       int gx = 0;
@@ -1007,7 +1008,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
     }
     ++nlaunch;
     if (h->timing) MCL_CUDA(h, cudaEventRecord(h->ev[1], s), "cudaEventRecord");
-    h->info[0] = lean_ran ? 8 : path;
+    h->info[0] = lean_ran ? 8 : (pool_ran ? 12 : path);
     h->info[2] = (int64_t)grid.x * grid.y;
     h->info[3] = threads;
     h->info[4] = 0;

@@ -24,6 +24,7 @@
 // (R6): chunk = digits of queues 0..Q-6, y = queue Q-5, x = queue Q-4, leaf =
 // queues Q-3..Q-1.
 #include <algorithm>
+#include <type_traits>
 
 #include "blocked_core.cuh"
 
@@ -34,6 +35,7 @@ namespace mcl {
 // unit's start, after its tables, after the walk and after the finish, plus the SM id.
 __device__ unsigned long long g_mcl_btrace[4096 * 4][8][4];
 __device__ unsigned int g_mcl_bsm[4096 * 4];
+__device__ unsigned long long g_mcl_ptrace[1024][4];  // SM-pooled kernel, per CTA
 __device__ __forceinline__ unsigned long long btrace_ns() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -302,6 +304,317 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
   }
 }
 
+// ---------------------------------------------------------------------------------------
+// SM-pooled form (default for batches): one CTA of 16 warps per SM shares its epochs at
+// sub-epoch granularity. Why: with a warp per epoch the SMSP's oldest-first warp scheduler
+// starves the younger warps, so the four warps of an SMSP finish their (equal) work at
+// ~35 / 47 / 60 / 74 us and the last ~15 us run one warp per SMSP at ~64-81 % ALU
+// (SS7, profiles/r02/batch_study.md). Here a favoured warp simply claims more
+// work: the CTA's epochs (blockIdx.x, + gridDim.x, ...: a static, monotone ordinal -> epoch
+// map, no global atomics) are cut into PARTS of 32 * kSbLane super-blocks, and the 16 warps
+// claim (ordinal, part) pairs from one shared counter. Each epoch's tables (inner sums and
+// one-hot outer rows, built once per epoch by the warp that claimed part 0 of the epoch
+// kPoolAhead ordinals earlier) live in a ring of kPoolSlots shared-memory slots; a part's
+// warp key (makespan << 32 | super-block) is merged by a shared 64-bit atomicMin, and the
+// warp completing an epoch's last part re-scans the winning super-block, writes the
+// outputs and frees the slot. The lexicographic minimum over parts is the epoch's lowest
+// super-block holding the minimum (every lane walks its super-blocks in increasing order
+// with strict <), so the result is the same as the warp-per-epoch kernel's.
+#ifndef MCL_BATCH_POOL
+#define MCL_BATCH_POOL 1  // 0: warp-per-epoch kernel for every batch (A/B builds)
+#endif
+namespace {
+constexpr int kPoolWarps = 16;
+constexpr int kPoolSlots = 16;
+constexpr int kPoolAhead = 4;  // epochs prepared ahead of the claims (PCIe reads when zero-copy)
+#ifndef MCL_POOL_SBL
+#define MCL_POOL_SBL 2u  // super-blocks per lane in one part (when it divides D)
+#endif
+// CTA-scope acquire/release fence for the shared-memory hand-offs between warps (lighter
+// than __threadfence_block's sequentially consistent MEMBAR.SC.CTA)
+__device__ __forceinline__ void fence_cta() { asm volatile("fence.acq_rel.cta;" ::: "memory"); }
+#ifndef MCL_POOL_TAIL
+#define MCL_POOL_TAIL 2  // last ordinals of each CTA cut into single-super-block parts
+#endif
+#ifndef MCL_POOL_UNROLL
+#define MCL_POOL_UNROLL 1  // unroll of a lane's super-block loop within a part
+#endif
+constexpr int kPoolTail = MCL_POOL_TAIL;
+constexpr int kPoolUnroll = MCL_POOL_UNROLL;
+#ifndef MCL_POOL_MIN_PER_SM
+#define MCL_POOL_MIN_PER_SM 2
+#endif
+constexpr int kPoolMinPerSm = MCL_POOL_MIN_PER_SM;  // smaller batches: warp per epoch
+}  // namespace
+
+template <int Q, int D>
+__global__ void __launch_bounds__(32 * kPoolWarps, 1) search_pool_kernel(BatchArgs a) {
+  using T = uint32_t;
+  constexpr int QD = Q * D;
+  constexpr uint32_t kChunks = (uint32_t)IPow<D, Q - 5>::v;
+  constexpr uint32_t kSb = kChunks * D;                       // super-blocks per epoch
+  constexpr uint32_t kSbLane = (D % MCL_POOL_SBL == 0) ? MCL_POOL_SBL : 1u;  // super-blocks per lane and part
+  constexpr uint32_t kPartSb = 32u * kSbLane;
+  constexpr uint32_t kParts = (kSb + kPartSb - 1) / kPartSb;  // parts per epoch
+  constexpr uint32_t kParts1 = (kSb + 31u) / 32u;             // the same, one super-block per lane
+  constexpr int kVN = (Q - 4) * D * D;
+  static_assert(QD <= 64, "two cost entries per lane");
+  static_assert(D * D <= 32, "finish: one lane per (x, i) pair of a super-block");
+  static_assert(D % kSbLane == 0, "a lane's super-blocks share one chunk");
+  struct Slot {
+    uint64_t C64[QD];
+    T in[8 * D];
+    T V[kVN];
+  };
+  __shared__ __align__(16) Slot s_slot[kPoolSlots];
+  __shared__ unsigned long long s_key[kPoolSlots];
+  __shared__ uint32_t s_cnt[kPoolSlots];
+  __shared__ int s_ready[kPoolSlots];  // ordinal whose tables the slot holds
+  __shared__ int s_done[kPoolSlots];   // last ordinal finished in the slot
+  __shared__ uint32_t s_skip[kPoolSlots];
+  __shared__ uint32_t s_next;
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const uint32_t one = a.one;
+  const uint64_t G = gridDim.x, b = blockIdx.x;
+#ifdef MCL_TRACE
+  // per CTA: entry, first part claimed with its tables ready, first failed claim, last exit
+  __shared__ uint32_t s_exit, s_first;
+  if (threadIdx.x == 0 && b < 1024) {
+    s_exit = 0;
+    s_first = 0;
+    g_mcl_ptrace[b][0] = btrace_ns();
+  }
+#endif
+  const uint32_t n_ord = a.E > b ? (uint32_t)((a.E - b + G - 1) / G) : 0u;
+  const uint32_t n_big = n_ord > (uint32_t)kPoolTail ? n_ord - (uint32_t)kPoolTail : 0u;
+  const uint32_t t_big = n_big * kParts;
+  const uint32_t total = t_big + (n_ord - n_big) * kParts1;
+  if (threadIdx.x < kPoolSlots) {
+    s_key[threadIdx.x] = ~0ull;
+    s_cnt[threadIdx.x] = 0;
+    s_ready[threadIdx.x] = -1;
+    s_done[threadIdx.x] = (int)threadIdx.x - kPoolSlots;
+  }
+  if (threadIdx.x == 0) s_next = 0;
+  __syncthreads();
+
+  // ---- a1 + tables of ordinal n, by one whole warp ----
+  auto prepare = [&](uint32_t n) {
+    const int si = (int)(n % kPoolSlots);
+    Slot& S = s_slot[si];
+    const uint64_t e = b + (uint64_t)n * G;
+    const uint64_t* Ke = a.K + e * QD;
+    const uint64_t* Xe = a.X + e * QD;
+    uint64_t k0 = 0, x0 = 0, k1 = 0, x1 = 0;
+    if (lane < QD) { k0 = Ke[lane]; x0 = Xe[lane]; }
+    if (lane + 32 < QD) { k1 = Ke[lane + 32]; x1 = Xe[lane + 32]; }
+    if (lane == 0) {  // the slot's previous occupant (ordinal n - kPoolSlots) is finished
+      while (*(volatile int*)&s_done[si] != (int)n - kPoolSlots) __nanosleep(64);
+    }
+    __syncwarp();
+    bool bad = false;
+    if (lane < QD) {
+      bad |= (k0 >= kEntryLimit) | (x0 >= kEntryLimit);
+      S.C64[lane] = k0 + x0;
+    }
+    if (lane + 32 < QD) {
+      bad |= (k1 >= kEntryLimit) | (x1 >= kEntryLimit);
+      S.C64[lane + 32] = k1 + x1;
+    }
+    __syncwarp();
+    uint64_t row = 0;
+    if (lane < Q) {
+#pragma unroll
+      for (int d = 0; d < D; ++d) row = max(row, S.C64[lane * D + d]);
+    }
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) row += __shfl_xor_sync(0xffffffffu, row, off);
+    const bool anybad = __any_sync(0xffffffffu, bad);
+    const bool skip = anybad || row >= 0xffffffffull;  // 32-bit loads need UB < 2^32 - 1
+    if (skip && lane == 0) raise_flag(a.flags, anybad ? kFlagRange : kFlagNeedU64);
+    if (!skip) {
+      if (lane < D) {
+        const T A = (T)S.C64[(Q - 3) * D + lane], B = (T)S.C64[(Q - 2) * D + lane],
+                Cc = (T)S.C64[(Q - 1) * D + lane];
+        S.in[0 * D + lane] = A;
+        S.in[1 * D + lane] = B;
+        S.in[2 * D + lane] = Cc;
+        S.in[3 * D + lane] = A + B;
+        S.in[4 * D + lane] = A + Cc;
+        S.in[5 * D + lane] = B + Cc;
+        S.in[6 * D + lane] = A + B + Cc;
+        S.in[7 * D + lane] = (T)S.C64[(Q - 4) * D + lane];
+      }
+      for (int t = lane; t < kVN; t += 32) {
+        const int q = t / (D * D), x = (t / D) % D, d = t % D;
+        S.V[t] = (d == x) ? (T)S.C64[q * D + x] : T(0);
+      }
+    }
+    if (lane == 0) s_skip[si] = skip ? 1u : 0u;
+    __syncwarp();
+    fence_cta();
+    if (lane == 0) *(volatile int*)&s_ready[si] = (int)n;
+  };
+
+  auto chunk_base = [&](const T* V, uint32_t c, T (&bv)[D]) {
+#pragma unroll
+    for (int d = 0; d < D; ++d) bv[d] = 0;
+#pragma unroll
+    for (int q = Q - 6; q >= 0; --q) {
+      const uint32_t dq = c % D;
+      c /= D;
+      const T* r = V + (q * D + dq) * D;
+#pragma unroll
+      for (int d = 0; d < D; ++d) bv[d] = add_f(bv[d], r[d], one);
+    }
+  };
+
+  // the lowest leaf of the winning super-block and the outputs (as search_batch_kernel)
+  auto finish = [&](const Slot& S, uint64_t e, uint64_t key) {
+    const T* in = S.in;
+    const T* c4 = in + 7 * D;
+    const T target = (T)(key >> 32);
+    const uint32_t sb = (uint32_t)key;
+    T base[D];
+    {
+      T b2[D];
+      chunk_base(S.V, sb / D, b2);
+      const T* r = S.V + ((Q - 5) * D + sb % D) * D;
+#pragma unroll
+      for (int d = 0; d < D; ++d) base[d] = add_f(b2[d], r[d], one);
+    }
+    const uint32_t x = (uint32_t)lane / D, i = (uint32_t)lane % D;
+    T PB[D], PC[D];
+    T Mp = 0;
+#pragma unroll
+    for (int d = 0; d < D; ++d) {
+      T v = base[d];
+      if (x == (uint32_t)d) v += c4[d];
+      if (i == (uint32_t)d) v += in[0 * D + d];
+      Mp = max2(Mp, v);
+      PB[d] = v + in[1 * D + d];
+      PC[d] = v + in[2 * D + d];
+    }
+    uint32_t hit = 0xffffffffu;
+#pragma unroll
+    for (int j = D - 1; j >= 0; --j)
+#pragma unroll
+      for (int k = D - 1; k >= 0; --k) {
+        const T v = (j == k) ? max2(Mp, PB[j] + in[2 * D + j]) : max3(Mp, PB[j], PC[k]);
+        if (v == target) hit = (uint32_t)(j * D + k);
+      }
+    const uint32_t m = __ballot_sync(0xffffffffu, lane < D * D && hit != 0xffffffffu);
+    uint64_t idx = kNone;
+    if (m) {
+      const int src = __ffs(m) - 1;
+      const uint32_t t = __shfl_sync(0xffffffffu, hit, src);
+      idx = (uint64_t)sb * (uint64_t)(D * D * D * D) + (uint64_t)src * (D * D) + t;
+    }
+    if (lane == 0) {
+      a.index[e] = idx;
+      a.makespan[e] = (uint64_t)target;
+    }
+    if (a.mapping && lane < Q) {
+      uint64_t rest = idx;
+      for (int q = Q - 1; q > lane; --q) rest /= D;
+      a.mapping[e * Q + lane] = (uint8_t)(rest % D);
+    }
+  };
+
+  if (wib < kPoolAhead && (uint32_t)wib < n_ord) prepare((uint32_t)wib);
+  for (;;) {
+    uint32_t t = 0;
+    if (lane == 0) t = atomicAdd(&s_next, 1u);
+    t = __shfl_sync(0xffffffffu, t, 0);
+    if (t >= total) {
+#ifdef MCL_TRACE
+      if (lane == 0 && b < 1024) {
+        if (t == total) g_mcl_ptrace[b][2] = btrace_ns();
+        if (atomicAdd(&s_exit, 1u) == kPoolWarps - 1) g_mcl_ptrace[b][3] = btrace_ns();
+      }
+#endif
+      break;
+    }
+    // (ordinal, part, super-blocks per lane): the last kPoolTail ordinals in single-super-
+    // block parts, so the warps' last parts end closer together
+    uint32_t n, p, sbl, parts;
+    if (t < t_big) {
+      n = t / kParts;
+      p = t % kParts;
+      sbl = kSbLane;
+      parts = kParts;
+    } else {
+      n = n_big + (t - t_big) / kParts1;
+      p = (t - t_big) % kParts1;
+      sbl = 1;
+      parts = kParts1;
+    }
+    const int si = (int)(n % kPoolSlots);
+    if (p == 0 && n + kPoolAhead < n_ord) prepare(n + kPoolAhead);
+    if (lane == 0) {
+      while (*(volatile int*)&s_ready[si] != (int)n) __nanosleep(32);
+    }
+    __syncwarp();
+    fence_cta();
+#ifdef MCL_TRACE
+    if (lane == 0 && b < 1024 && atomicExch(&s_first, 1u) == 0) g_mcl_ptrace[b][1] = btrace_ns();
+#endif
+    const bool skip = *(volatile uint32_t*)&s_skip[si] != 0;
+    const Slot& S = s_slot[si];
+    if (!skip) {
+      const T* in = S.in;
+      const T* c4 = in + 7 * D;
+      T best = ~T(0);
+      uint32_t best_sb = 0xffffffffu;
+      const uint32_t sb0 = (p * 32u + (uint32_t)lane) * sbl;
+      // a lane's super-blocks sb0 .. sb0 + n - 1 (n divides D: one chunk), compile-time n
+      auto walk = [&](auto nsb) {
+        constexpr uint32_t n_sb = decltype(nsb)::value;
+        T base2[D];
+        chunk_base(S.V, sb0 / D, base2);
+#pragma unroll
+        for (uint32_t j = 0; j < n_sb; ++j) {
+          const uint32_t sb = sb0 + j;
+          const T* r = S.V + ((Q - 5) * D + sb % D) * D;
+          T base[D];
+#pragma unroll
+          for (int d = 0; d < D; ++d) base[d] = add_f(base2[d], r[d], one);
+          const T gs = superblock_eval<T, D>(base, in, c4, one);
+          if (gs < best) {
+            best = gs;
+            best_sb = sb;
+          }
+        }
+      };
+      if (sb0 < kSb) {
+        if (kSbLane > 1 && sbl == kSbLane) walk(std::integral_constant<uint32_t, kSbLane>{});
+        else walk(std::integral_constant<uint32_t, 1u>{});
+      }
+      const uint32_t g = __reduce_min_sync(0xffffffffu, (uint32_t)best);
+      const uint32_t bsb = __reduce_min_sync(0xffffffffu, (uint32_t)best == g ? best_sb : 0xffffffffu);
+      if (lane == 0) atomicMin(&s_key[si], ((unsigned long long)g << 32) | bsb);
+    }
+    uint32_t c = 0;
+    if (lane == 0) {
+      fence_cta();
+      c = atomicAdd(&s_cnt[si], 1u);
+    }
+    c = __shfl_sync(0xffffffffu, c, 0);
+    if (c == parts - 1) {  // this warp completed the epoch
+      fence_cta();
+      const uint64_t key = *(volatile unsigned long long*)&s_key[si];
+      if (!skip) finish(S, b + (uint64_t)n * G, key);
+      __syncwarp();
+      if (lane == 0) {
+        s_key[si] = ~0ull;
+        s_cnt[si] = 0;
+        fence_cta();
+        *(volatile int*)&s_done[si] = (int)n;
+      }
+    }
+  }
+}
+
 #ifdef MCL_TRACE
 }  // namespace mcl
 extern "C" int mcl_btrace_read(unsigned long long* out, unsigned int* sm, int nwarps) {
@@ -309,12 +622,23 @@ extern "C" int mcl_btrace_read(unsigned long long* out, unsigned int* sm, int nw
   if (e == cudaSuccess) e = cudaMemcpyFromSymbol(sm, mcl::g_mcl_bsm, (size_t)nwarps * 4);
   return (int)e;
 }
+extern "C" int mcl_ptrace_read(unsigned long long* out) {
+  return (int)cudaMemcpyFromSymbol(out, mcl::g_mcl_ptrace, sizeof(mcl::g_mcl_ptrace));
+}
 namespace mcl {
 #endif
 
 namespace {
 template <int Q, int D>
-cudaError_t launch_batch_t(const BatchArgs& a, int num_sms, cudaStream_t st, int* grid_out) {
+cudaError_t launch_batch_t(const BatchArgs& a, int num_sms, cudaStream_t st, int* grid_out, bool* pooled) {
+  *pooled = false;
+  if (MCL_BATCH_POOL && a.E >= (uint64_t)num_sms * kPoolMinPerSm) {
+    // one 16-warp CTA per SM, epochs blockIdx.x + n * gridDim.x
+    search_pool_kernel<Q, D><<<(unsigned)num_sms, 32 * kPoolWarps, 0, st>>>(a);
+    *grid_out = num_sms;
+    *pooled = true;
+    return cudaGetLastError();
+  }
   auto k = search_batch_kernel<Q, D>;
   static std::atomic<int> occ[64];
   int dev = 0;
@@ -357,18 +681,18 @@ bool batch_supported(uint32_t Q, uint32_t D) {
   }
 }
 
-cudaError_t launch_batch(const BatchArgs& a, int num_sms, cudaStream_t st, int* grid_out) {
+cudaError_t launch_batch(const BatchArgs& a, int num_sms, cudaStream_t st, int* grid_out, bool* pooled) {
   switch (a.Q * 100 + a.D) {
-    case 803: return launch_batch_t<8, 3>(a, num_sms, st, grid_out);
-    case 903: return launch_batch_t<9, 3>(a, num_sms, st, grid_out);
-    case 1003: return launch_batch_t<10, 3>(a, num_sms, st, grid_out);
-    case 1103: return launch_batch_t<11, 3>(a, num_sms, st, grid_out);
-    case 804: return launch_batch_t<8, 4>(a, num_sms, st, grid_out);
-    case 904: return launch_batch_t<9, 4>(a, num_sms, st, grid_out);
-    case 1004: return launch_batch_t<10, 4>(a, num_sms, st, grid_out);
-    case 1104: return launch_batch_t<11, 4>(a, num_sms, st, grid_out);
-    case 805: return launch_batch_t<8, 5>(a, num_sms, st, grid_out);
-    case 905: return launch_batch_t<9, 5>(a, num_sms, st, grid_out);
+    case 803: return launch_batch_t<8, 3>(a, num_sms, st, grid_out, pooled);
+    case 903: return launch_batch_t<9, 3>(a, num_sms, st, grid_out, pooled);
+    case 1003: return launch_batch_t<10, 3>(a, num_sms, st, grid_out, pooled);
+    case 1103: return launch_batch_t<11, 3>(a, num_sms, st, grid_out, pooled);
+    case 804: return launch_batch_t<8, 4>(a, num_sms, st, grid_out, pooled);
+    case 904: return launch_batch_t<9, 4>(a, num_sms, st, grid_out, pooled);
+    case 1004: return launch_batch_t<10, 4>(a, num_sms, st, grid_out, pooled);
+    case 1104: return launch_batch_t<11, 4>(a, num_sms, st, grid_out, pooled);
+    case 805: return launch_batch_t<8, 5>(a, num_sms, st, grid_out, pooled);
+    case 905: return launch_batch_t<9, 5>(a, num_sms, st, grid_out, pooled);
     default: return cudaErrorInvalidValue;
   }
 }

@@ -19,7 +19,7 @@ LIB_PATH = os.path.join(_HERE, "libmcl.so")
 MCL_OK, MCL_E_INVAL, MCL_E_RANGE, MCL_E_CUDA, MCL_E_NCCL, MCL_E_NOMEM = 0, -1, -2, -3, -4, -5
 PATH_NAMES = {1: "blocked_u32", 2: "blocked_u64", 3: "generic", 4: "small_batched", 5: "flat_u32",
               6: "pruned", 7: "batch_u32", 8: "blocked_u32_lean", 9: "mixed_u32", 10: "mixed_u64",
-              11: "mixed_warp_u32"}
+              11: "mixed_warp_u32", 12: "batch_pool_u32"}
 
 # Every symbol the headers declare (tests check the library exports all of them).
 EXPORTED = [

@@ -3,7 +3,7 @@
     python scripts/ab_lib.py build/ab/libmcl_old.so build/ab/libmcl_new.so [more.so ...] [rounds]
 
 Each round runs every library in a fresh subprocess (alternating order) and prints the
-median kernel time (CUDA events, 200 us spin hold, L2 flushed) of the single-epoch configs
+median (AB_STAT=mean: mean; AB_N launches, default 9) kernel time (CUDA events, 200 us spin hold, L2 flushed) of the single-epoch configs
 at G = 1 and of rank 0 at G = 8, and of cfg2.
 """
 import json
@@ -25,9 +25,12 @@ for name in os.environ.get("AB_WORKLOADS", "cfg5,cfg4,cfg2").split(","):
     for G in ((1, 8) if name in ("cfg4", "cfg5") else (1,)):
         with mcl.Mapper(0, stream=st.cuda_stream, rank=0, world=G) as m:
             m.set_timing(True, hold_us=200); ts = []
-            for i in range(9):
+            for i in range(int(os.environ.get("AB_N", "9"))):
                 flush.fill_(i); flush.view(torch.int64).sum(); m.map_queues(Kd, Xd); ts.append(m.last_kernel_time_ms()[0])
-        out[f"{name}/G{G}"] = round(statistics.median(ts[2:]), 5)
+        # AB_STAT=mean: the CUDA-event clock of some boxes ticks in ~1 us steps, so a mean
+        # over many launches resolves differences a median of a few cannot
+        stat = statistics.mean if os.environ.get("AB_STAT") == "mean" else statistics.median
+        out[f"{name}/G{G}"] = round(stat(ts[2:]), 5)
 print(json.dumps(out))
 '''
 

@@ -82,7 +82,7 @@ def test_batch_auto_selection_cfg2(torch_cuda, mapper):
     K, X = workloads.cfg2()
     want = oracle.oracle_map(K, X)
     got, info = run(torch_cuda, mapper, K, X, 0)
-    assert info["path"] == "batch_u32", info
+    assert info["path"] == "batch_pool_u32", info
     check(got, want, "cfg2 auto")
     got, info = run(torch_cuda, mapper, K, X, 1)
     assert info["path"] == "blocked_u32"
@@ -126,7 +126,7 @@ def test_batch_whole_and_split_epochs(torch_cuda, mapper, Q, D):
     want = oracle.oracle_map(K, X)
     for rep in range(2):
         got, info = run(torch_cuda, mapper, K, X, 7)
-        assert info["path"] == "batch_u32"
+        assert info["path"] == "batch_pool_u32"
         check(got, want, f"{Q}x{D} E={E} rep {rep}")
         sub = 3 + 40 * rep  # every epoch split, then whole + split again
         got, _ = run(torch_cuda, mapper, K[:sub], X[:sub], 7)
@@ -150,3 +150,57 @@ def test_batch_single_epoch_and_no_mapping_output(torch_cuda, mapper):
         mapper.force_path(0)
     wi, wms, _ = oracle.oracle_map(K, X)
     assert (idx.cpu().numpy() == wi).all() and (ms.cpu().numpy() == wms).all()
+
+
+# ---- the SM-pooled form (path 12): batches of >= 2 epochs per SM ----
+POOL_E = 148 * 2 + 37  # >= 2 epochs per SM, ragged over the 148 CTAs
+
+
+@pytest.mark.parametrize("Q,D", BATCH_SHAPES)
+def test_pool_kernel_shapes(torch_cuda, mapper, Q, D):
+    """Every instantiated shape, random and tie-heavy tables, bit-exact vs the oracle."""
+    E = POOL_E if D**Q <= 1_100_000 else 300
+    for seed, maker in ((60 * Q + D, workloads.random_tables), (700 + 60 * Q + D, workloads.small_int_tables)):
+        K, X = maker(seed, E, Q, D)
+        got, info = run(torch_cuda, mapper, K, X, 7)
+        assert info["path"] == "batch_pool_u32", info
+        assert info["threads"] == 512
+        check(got, oracle.oracle_map(K, X), f"pool Q={Q} D={D} {maker.__name__}")
+
+
+def test_pool_degenerate_ties_and_sizes(torch_cuda, mapper):
+    """All-zero / all-equal / one-hot epochs spread over a pooled batch, then the same
+    handle at other batch sizes (pool state lives in shared memory: nothing carries over)."""
+    Q, D = 8, 4
+    K, X = workloads.small_int_tables(4242, 1200, Q, D, hi=3)
+    K[::7] = 0
+    X[::7] = 0
+    K[3::11] = 9
+    X[3::11] = 0
+    K[5::13] = 1000
+    K[5::13, :, 2] = 1
+    X[5::13] = 0
+    want = oracle.oracle_map(K, X)
+    for E in (1200, 296, 297, 1199, 1200):
+        got, info = run(torch_cuda, mapper, K[:E], X[:E], 7)
+        assert info["path"] == "batch_pool_u32", (E, info)
+        check(got, tuple(w[:E] for w in want), f"pool ties E={E}")
+
+
+def test_pool_u64_rerun_and_range_error(torch_cuda, mapper):
+    """An epoch of a pooled batch whose bound needs 64 bits reruns the batch on the 64-bit
+    kernel; an entry >= 2^48 fails the call; the next pooled call is exact."""
+    K, X = workloads.random_tables(81, POOL_E, 8, 4)
+    K[200] = np.random.default_rng(2).integers(1 << 46, 1 << 47, size=(8, 4), dtype=np.uint64)
+    got, info = run(torch_cuda, mapper, K, X, 7)
+    assert info["path"] == "blocked_u64"
+    check(got, oracle.oracle_map(K, X), "pool u64 rerun")
+    K, X = workloads.random_tables(82, POOL_E, 8, 4)
+    X[300, 2, 1] = 1 << 48
+    with pytest.raises(MclError) as ei:
+        run(torch_cuda, mapper, K, X, 7)
+    assert ei.value.status == MCL_E_RANGE
+    X[300, 2, 1] = 5
+    got, info = run(torch_cuda, mapper, K, X, 7)
+    assert info["path"] == "batch_pool_u32"
+    check(got, oracle.oracle_map(K, X), "pool after range error")

@@ -130,7 +130,7 @@ def test_cfg2_full(torch_cuda, mapper):
     K, X = workloads.cfg2()
     want = oracle.oracle_map(K, X)
     assert_same(run_gpu(torch_cuda, mapper, K, X), want, "cfg2")
-    assert mapper.launch_info()["path"] == "batch_u32"
+    assert mapper.launch_info()["path"] == "batch_pool_u32"
     assert_same(run_gpu(torch_cuda, mapper, K, X, 5), want, "cfg2 flattened")
     assert_same(run_gpu(torch_cuda, mapper, K, X, 1), want, "cfg2 CTA per epoch")
     # repeated calls reuse the self-resetting per-epoch keys; a smaller batch after a larger one
