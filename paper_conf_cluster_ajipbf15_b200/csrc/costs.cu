@@ -86,13 +86,22 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
   constexpr int PS32 = D % 2 ? D : D + 1;
   uint32_t* s_prof32 = reinterpret_cast<uint32_t*>(s_prof);
   bool fits32 = false;
+  __shared__ uint32_t s_pmax;  // largest entry of a 32-bit table
+  if (tid == 0) s_pmax = 0;
   if (prof_in_smem) {
     bool big = false;
-    for (uint32_t t = tid; t < a.num_kernels * D; t += blockDim.x) big |= (a.profile[t] >> 32) != 0;
+    uint32_t pm = 0;
+    for (uint32_t t = tid; t < a.num_kernels * D; t += blockDim.x) {
+      big |= (a.profile[t] >> 32) != 0;
+      pm = max(pm, (uint32_t)a.profile[t]);
+    }
+    pm = __reduce_max_sync(0xffffffffu, pm);
+    if (lane == 0 && pm) atomicMax(&s_pmax, pm);
     fits32 = !__syncthreads_or(big);
-    if (fits32)
+    if (fits32) {
       for (uint32_t t = tid; t < a.num_kernels * D; t += blockDim.x)
         s_prof32[(t / D) * PS32 + t % D] = (uint32_t)a.profile[t];
+    }
     else
       for (uint32_t t = tid; t < a.num_kernels * D; t += blockDim.x) s_prof[(t / D) * PS + t % D] = a.profile[t];
   }
@@ -160,6 +169,28 @@ __global__ void __launch_bounds__(kCostTile) build_costs_kernel(CostArgs a) {
             break;
           }
         }
+      } else if (ok && fits32 && a.num_kernels != 0 && j1 - j0 < (1ull << 31) &&
+                 (uint64_t)(j1 - j0) * s_pmax < (1ull << 32)) {
+        // the list's sums fit 32 bits (n x largest entry < 2^32): 32-bit accumulators and
+        // 32-bit positions; ids are clamped into the table and checked once after the loop
+        // (an id >= num_kernels flags the pair, as the early exit below does)
+        const uint32_t n = (uint32_t)(j1 - j0), kcap = a.num_kernels - 1;
+        const uint32_t* ids = a.ids + j0;
+        uint32_t k32[D];
+#pragma unroll
+        for (int d = 0; d < D; ++d) k32[d] = 0;
+        uint32_t idmax = 0;
+        auto add_id = [&](uint32_t kid) {
+          idmax = max(idmax, kid);
+          const uint32_t* row = s_prof32 + (size_t)min(kid, kcap) * PS32;
+#pragma unroll
+          for (int d = 0; d < D; ++d) k32[d] += row[d];
+        };
+#pragma unroll 4
+        for (uint32_t t = 0; t < n; ++t) add_id(__ldg(ids + t));
+        ok = idmax <= kcap;
+#pragma unroll
+        for (int d = 0; d < D; ++d) k[d] = ok ? k32[d] : 0;
       } else if (ok && fits32) {
 #pragma unroll 4
         for (uint64_t j = j0; j < j1; ++j) {

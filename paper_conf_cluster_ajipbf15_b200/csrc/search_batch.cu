@@ -334,7 +334,7 @@ constexpr int kPoolAhead = 4;  // epochs prepared ahead of the claims (PCIe read
 // than __threadfence_block's sequentially consistent MEMBAR.SC.CTA)
 __device__ __forceinline__ void fence_cta() { asm volatile("fence.acq_rel.cta;" ::: "memory"); }
 #ifndef MCL_POOL_TAIL
-#define MCL_POOL_TAIL 2  // last ordinals of each CTA cut into single-super-block parts
+#define MCL_POOL_TAIL 1  // last ordinals of each CTA cut into single-super-block parts
 #endif
 #ifndef MCL_POOL_UNROLL
 #define MCL_POOL_UNROLL 1  // unroll of a lane's super-block loop within a part
