@@ -248,6 +248,8 @@ struct BatchArgs {
   volatile uint32_t* flags;
   uint32_t one;
   uint64_t e_full;    // set by launch_batch: epochs searched by one warp (whole waves)
+  bool host_inputs;   // K / X are pinned host memory read in place (zero-copy): the
+                      // warp-per-epoch form, whose per-warp prefetch hides PCIe latency
 };
 bool batch_supported(uint32_t Q, uint32_t D);
 // *pooled = true when the SM-pooled form ran (one 16-warp CTA per SM, sub-epoch parts)

@@ -199,7 +199,9 @@ mcl_status_t nccl_fail(mcl_mapper* h, ncclResult_t r, const char* what) {
 // few hundred bytes of inputs and writes its outputs over the bus instead of 2 H2D + 3 D2H
 // copies, each a separate runtime call (cfg1 host-buffer call 36 -> ~16 us). Larger pinned
 // batches and pageable memory are staged (pipelined copy engines beat PCIe zero-copy there).
-mcl_status_t classify(mcl_mapper* h, const void* p, bool* on_device, const void** dptr = nullptr) {
+mcl_status_t classify(mcl_mapper* h, const void* p, bool* on_device, const void** dptr = nullptr,
+                      bool* in_place_host = nullptr) {
+  if (in_place_host) *in_place_host = false;
   cudaPointerAttributes at;
   cudaError_t e = cudaPointerGetAttributes(&at, p);
   if (e != cudaSuccess) {  // CUDA >= 11 reports unregistered host memory as success
@@ -219,6 +221,7 @@ mcl_status_t classify(mcl_mapper* h, const void* p, bool* on_device, const void*
   } else if (at.type == cudaMemoryTypeHost && h->zero_copy && at.devicePointer) {
     *on_device = true;  // pinned host memory, small call: zero-copy
     if (dptr) *dptr = at.devicePointer;
+    if (in_place_host) *in_place_host = true;
   } else {
     *on_device = false;  // pageable or (large call) pinned host memory: staged
   }
@@ -446,12 +449,13 @@ mcl_status_t stage_in(mcl_mapper* h, DevBuf& buf, const void* src, size_t bytes,
 
 // Classify a caller buffer, then stage it in (`src` may be NULL: *out = NULL).
 mcl_status_t classify_stage_in(mcl_mapper* h, DevBuf& buf, const void* src, size_t bytes,
-                               const void** out) {
+                               const void** out, bool* in_place_host = nullptr) {
   *out = nullptr;
+  if (in_place_host) *in_place_host = false;
   if (!src) return MCL_OK;
   bool on = false;
   const void* d = nullptr;
-  mcl_status_t st = classify(h, src, &on, &d);
+  mcl_status_t st = classify(h, src, &on, &d, in_place_host);
   if (st != MCL_OK) return st;
   return stage_in(h, buf, src, bytes, on, out, d);
 }
@@ -769,8 +773,9 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
   if (h->timing >= 2) MCL_CUDA(h, cudaEventRecord(h->ev[2], s), "cudaEventRecord");
   const size_t in_bytes = (size_t)epochs * Q * D * sizeof(uint64_t);
   const void *Kp, *Xp, *Bp, *Ep;
-  if ((st = classify_stage_in(h, h->in_k, cost_kernel, in_bytes, &Kp)) != MCL_OK) return st;
-  if ((st = classify_stage_in(h, h->in_x, cost_xfer, in_bytes, &Xp)) != MCL_OK) return st;
+  bool k_host = false, x_host = false;  // pinned host inputs read in place (zero-copy)
+  if ((st = classify_stage_in(h, h->in_k, cost_kernel, in_bytes, &Kp, &k_host)) != MCL_OK) return st;
+  if ((st = classify_stage_in(h, h->in_x, cost_xfer, in_bytes, &Xp, &x_host)) != MCL_OK) return st;
   // constrained variant: base loads [E][D] and eligible masks [E][Q] (either may be NULL)
   if ((st = classify_stage_in(h, h->in_base, base_load, epochs * D * 8, &Bp)) != MCL_OK) return st;
   if ((st = classify_stage_in(h, h->in_elig, eligible, epochs * Q * 2, &Ep)) != MCL_OK) return st;
@@ -849,7 +854,7 @@ mcl_status_t map_impl(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64_t epochs,
     bool pool_ran = false;  // the SM-pooled batch kernel (reported as path 12)
     if (h->timing) MCL_CUDA(h, record_start(h, s), "cudaEventRecord(start)");
     if (path == 7) {
-      mcl::BatchArgs a{Q, D, epochs, K, X, o_idx, o_ms, o_map, h->flags_dev, 1u};
+      mcl::BatchArgs a{Q, D, epochs, K, X, o_idx, o_ms, o_map, h->flags_dev, 1u, 0, k_host || x_host};
       int gx = 0;
       MCL_CUDA(h, mcl::launch_batch(a, h->num_sms, s, &gx, &pool_ran), "search_batch launch");
       grid.x = gx;

@@ -632,7 +632,7 @@ namespace {
 template <int Q, int D>
 cudaError_t launch_batch_t(const BatchArgs& a, int num_sms, cudaStream_t st, int* grid_out, bool* pooled) {
   *pooled = false;
-  if (MCL_BATCH_POOL && a.E >= (uint64_t)num_sms * kPoolMinPerSm) {
+  if (MCL_BATCH_POOL && !a.host_inputs && a.E >= (uint64_t)num_sms * kPoolMinPerSm) {
     // one 16-warp CTA per SM, epochs blockIdx.x + n * gridDim.x
     search_pool_kernel<Q, D><<<(unsigned)num_sms, 32 * kPoolWarps, 0, st>>>(a);
     *grid_out = num_sms;

@@ -98,7 +98,7 @@ def test_pipelined_auto_matches_unpipelined(torch_cuda, mapper):
     finally:
         mapper.set_pipeline_chunks(0)
     got_zc = host_call(torch_cuda, mapper, K, X, pinned=True)
-    assert mapper.launch_info()["chunks"] == 0 and mapper.launch_info()["path"] == "batch_pool_u32"
+    assert mapper.launch_info()["chunks"] == 0 and mapper.launch_info()["path"] == "batch_u32"
     for a, b, c in zip(got_auto, got_off, got_zc):
         assert (a == b).all() and (a == c).all()
     check(got_auto, oracle.oracle_map(K, X), "cfg2 auto")
