@@ -632,7 +632,10 @@ namespace {
 template <int Q, int D>
 cudaError_t launch_batch_t(const BatchArgs& a, int num_sms, cudaStream_t st, int* grid_out, bool* pooled) {
   *pooled = false;
-  if (MCL_BATCH_POOL && !a.host_inputs && a.E >= (uint64_t)num_sms * kPoolMinPerSm) {
+  // MCL_POOL_MIN_PER_SM (environment, tests / sanitizer runs): the smallest batch, in
+  // epochs per SM, that takes the pooled form (a huge value keeps the warp-per-epoch form)
+  static const int min_per_sm = env_int("MCL_POOL_MIN_PER_SM", kPoolMinPerSm, 1, 1 << 30);
+  if (MCL_BATCH_POOL && !a.host_inputs && a.E >= (uint64_t)num_sms * min_per_sm) {
     // one 16-warp CTA per SM, epochs blockIdx.x + n * gridDim.x
     search_pool_kernel<Q, D><<<(unsigned)num_sms, 32 * kPoolWarps, 0, st>>>(a);
     *grid_out = num_sms;

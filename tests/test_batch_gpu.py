@@ -204,3 +204,22 @@ def test_pool_u64_rerun_and_range_error(torch_cuda, mapper):
     got, info = run(torch_cuda, mapper, K, X, 7)
     assert info["path"] == "batch_pool_u32"
     check(got, oracle.oracle_map(K, X), "pool after range error")
+
+
+def test_pool_repeatable_under_load(torch_cuda, mapper):
+    """The pooled kernel's shared-memory hand-offs (claims, table slots, key merges, slot
+    reuse) checked by repetition: 12 back-to-back launches of full cfg2 (10^4 epochs over
+    148 CTAs, 16 slots recycled ~4 times per CTA) must all equal the oracle bit for bit.
+    (compute-sanitizer is not available on this pool: repeated exact parity stands in.)"""
+    torch = torch_cuda
+    K, X = workloads.cfg2()
+    wi, wms, wmp = oracle.oracle_map(K, X)
+    Kd, Xd = torch.from_numpy(K).cuda(), torch.from_numpy(X).cuda()
+    outs = []
+    for _ in range(12):
+        idx, mp, ms = mapper.map_queues(Kd, Xd)
+        assert mapper.launch_info()["path"] == "batch_pool_u32"
+        outs.append((idx, mp, ms))
+    for idx, mp, ms in outs:
+        assert (idx.cpu().numpy() == wi).all() and (ms.cpu().numpy() == wms).all()
+        assert (mp.cpu().numpy() == wmp).all()
