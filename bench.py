@@ -644,6 +644,18 @@ def main():
     t_all = time.perf_counter()
     for n in names:
         entries[n] = measure(ctx, n)
+    # after every timed region: what CUDA events report around a kernel that does nothing,
+    # timed as the configs' kernel_ms are (the share of a short kernel's kernel_ms that no
+    # kernel can avoid on this platform; SS12)
+    floor = None
+    if ctx.rank == 0:
+        try:
+            k_us, e_us = mcl.mcl_probe_launch_floor(ctx.dev_index, 30)
+            floor = {"empty_kernel_us": k_us, "events_only_us": e_us,
+                     "note": "CUDA events around an empty 148 x 512 kernel after a 200 us hold "
+                             "(mcl_probe_launch_floor), as kernel_ms is timed; not subtracted anywhere"}
+        except Exception as exc:  # pragma: no cover
+            floor = {"error": str(exc)}
     if ctx.comm:
         mcl.mcl_comm_destroy(ctx.comm)
     if dist.is_initialized():
@@ -661,6 +673,8 @@ def main():
     }
     if "ranks_agree" in head:
         line["ranks_agree"] = head["ranks_agree"]
+    if floor is not None:
+        line["launch_floor"] = floor
     others = {n: e for n, e in entries.items() if n != args.workload}
     if ctx.world == 1 and not args.no_cpu_baseline:
         import oracle

@@ -42,6 +42,16 @@ mcl_status_t mcl_set_timing_hold(mcl_mapper_t* h, uint32_t hold_us);
 mcl_status_t mcl_probe_int_rate(int device, int op, double* lane_ops_per_s,
                                 double* lane_ops_per_clk_sm, double* eff_mhz);
 
+/*
+ * Launch floor on `device`: the mean over `reps` (>= 1) of what CUDA events report around
+ * a kernel that does nothing (one CTA of 512 threads per SM), each timed as the search
+ * kernels are timed by mcl_set_timing + mcl_set_timing_hold(200), and of the events alone.
+ * It is the part of every event-timed kernel duration that no kernel can avoid on this
+ * platform. Synchronous, on the legacy default stream. Any output pointer may be NULL.
+ * MCL_E_INVAL for a bad device or reps < 1.
+ */
+mcl_status_t mcl_probe_launch_floor(int device, int reps, double* empty_kernel_us, double* events_only_us);
+
 /* Testing aid: force the kernel of later mcl_map_queues calls on h. path: 0 = automatic
    (default), 1 = register-blocked (u32 loads, falls back to 64-bit when a bound needs it),
    2 = register-blocked with 64-bit loads, 3 = generic, 4 = small batched, 5 = register-

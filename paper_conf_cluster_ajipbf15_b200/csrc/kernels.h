@@ -125,6 +125,7 @@ size_t blocked_smem_bytes(uint32_t Q, uint32_t D, bool wide, int threads, size_t
                           size_t* off_dig);
 // one-thread kernel spinning for `ns` nanoseconds of %globaltimer (timing aid, probe.cu)
 cudaError_t launch_hold(uint64_t ns, cudaStream_t st);
+cudaError_t probe_launch_floor(int sms, cudaStream_t st, int reps, double* empty_us, double* events_us);
 cudaError_t launch_blocked(const BlockedArgs& a, bool wide, dim3 grid, int threads, size_t smem,
                            cudaStream_t st, bool lean = false);
 

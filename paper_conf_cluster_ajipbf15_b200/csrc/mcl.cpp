@@ -1465,6 +1465,22 @@ mcl_status_t mcl_probe_int_rate(int device, int op, double* lane_ops_per_s,
   return MCL_OK;
 }
 
+mcl_status_t mcl_probe_launch_floor(int device, int reps, double* empty_kernel_us, double* events_only_us) {
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev || reps < 1)
+    return MCL_E_INVAL;
+  DeviceGuard g(device);
+  int sms = 0;
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess)
+    return MCL_E_CUDA;
+  double k = 0, e = 0;
+  cudaError_t err = mcl::probe_launch_floor(sms, nullptr, reps, &k, &e);
+  if (err != cudaSuccess) return cuda_fail(nullptr, err, "launch floor probe");
+  if (empty_kernel_us) *empty_kernel_us = k;
+  if (events_only_us) *events_only_us = e;
+  return MCL_OK;
+}
+
 mcl_status_t mcl_device_sms(int device, int* sms) {
   if (!sms) return MCL_E_INVAL;
   cudaError_t e = cudaDeviceGetAttribute(sms, cudaDevAttrMultiProcessorCount, device);

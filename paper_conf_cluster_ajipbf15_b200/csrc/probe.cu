@@ -137,4 +137,38 @@ cudaError_t launch_hold(uint64_t ns, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+// Launch floor: what CUDA events around a kernel that does nothing report, timed as the
+// search kernels are timed (a 200 us hold first, so the events bracket device execution).
+// One CTA per SM of 512 threads (the pooled batch kernel's shape). Also the events alone.
+__global__ void empty_kernel(int* never) {
+  if (never && threadIdx.x == 1023) *never = 1;  // never true: 512 threads
+}
+
+cudaError_t probe_launch_floor(int sms, cudaStream_t st, int reps, double* empty_us,
+                               double* events_us) {
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  cudaError_t err = cudaEventCreate(&e0);
+  if (err == cudaSuccess) err = cudaEventCreate(&e1);
+  double sum_k = 0, sum_e = 0;
+  for (int kind = 0; kind < 2 && err == cudaSuccess; ++kind) {
+    for (int i = 0; i < reps + 3 && err == cudaSuccess; ++i) {
+      hold_kernel<<<1, 1, 0, st>>>(200000);
+      cudaEventRecord(e0, st);
+      if (kind == 0) empty_kernel<<<sms, 512, 0, st>>>(nullptr);
+      cudaEventRecord(e1, st);
+      err = cudaEventSynchronize(e1);
+      float ms = 0;
+      if (err == cudaSuccess) err = cudaEventElapsedTime(&ms, e0, e1);
+      if (i >= 3) (kind == 0 ? sum_k : sum_e) += ms * 1e3;
+    }
+  }
+  if (err == cudaSuccess) {
+    *empty_us = sum_k / reps;
+    *events_us = sum_e / reps;
+  }
+  if (e0) cudaEventDestroy(e0);
+  if (e1) cudaEventDestroy(e1);
+  return err;
+}
+
 }  // namespace mcl

@@ -26,6 +26,7 @@ EXPORTED = [
     "mcl_mapper_create", "mcl_map_queues", "mcl_mapper_destroy", "mcl_status_string",
     "mcl_last_error_string", "mcl_last_launch_info", "mcl_version",
     "mcl_set_timing", "mcl_set_timing_hold", "mcl_last_kernel_time", "mcl_force_path", "mcl_set_pipeline_chunks", "mcl_probe_int_rate",
+    "mcl_probe_launch_floor",
     "mcl_device_sms",
     "mcl_comm_unique_id", "mcl_comm_init", "mcl_comm_destroy",
     "mcl_map_queues_constrained", "mcl_score_mappings", "mcl_map_queues_pruned",
@@ -100,6 +101,7 @@ def load_library(path: str | None = None) -> ctypes.CDLL:
         "mcl_last_kernel_time": (i32, [vp, ctypes.POINTER(ctypes.c_float), ctypes.POINTER(ctypes.c_float)]),
         "mcl_probe_int_rate": (i32, [i32, i32, ctypes.POINTER(ctypes.c_double),
                                      ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]),
+        "mcl_probe_launch_floor": (i32, [i32, i32, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]),
         "mcl_device_sms": (i32, [i32, ctypes.POINTER(i32)]),
         "mcl_comm_unique_id": (i32, [ctypes.c_char_p]),
         "mcl_comm_init": (i32, [i32, i32, i32, ctypes.c_char_p, ctypes.POINTER(vp)]),
@@ -166,6 +168,15 @@ def mcl_last_launch_info(handle: int) -> list[int]:
     arr = (ctypes.c_int64 * 8)()
     load_library().mcl_last_launch_info(handle, arr)
     return list(arr)
+
+
+def mcl_probe_launch_floor(device: int, reps: int = 20) -> tuple[float, float]:
+    """(empty-kernel event time, events-alone time) in microseconds (mcl_ext.h)."""
+    k, e = ctypes.c_double(), ctypes.c_double()
+    st = load_library().mcl_probe_launch_floor(device, reps, ctypes.byref(k), ctypes.byref(e))
+    if st != MCL_OK:
+        raise MclError(st, "mcl_probe_launch_floor", mcl_last_error_string(None))
+    return k.value, e.value
 
 
 def mcl_probe_int_rate(device: int, op: int) -> tuple[float, float, float]:
