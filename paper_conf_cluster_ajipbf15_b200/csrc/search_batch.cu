@@ -325,8 +325,14 @@ __global__ void __launch_bounds__(32 * kBatchWarps, 4) search_batch_kernel(Batch
 #endif
 namespace {
 constexpr int kPoolWarps = 16;
-constexpr int kPoolSlots = 16;
-constexpr int kPoolAhead = 4;  // epochs prepared ahead of the claims (PCIe reads when zero-copy)
+#ifndef MCL_POOL_SLOTS
+#define MCL_POOL_SLOTS 32
+#endif
+constexpr int kPoolSlots = MCL_POOL_SLOTS;  // ring of per-epoch table slots
+#ifndef MCL_POOL_AHEAD
+#define MCL_POOL_AHEAD 12
+#endif
+constexpr int kPoolAhead = MCL_POOL_AHEAD;  // epochs prepared ahead of the claims
 #ifndef MCL_POOL_SBL
 #define MCL_POOL_SBL 2u  // super-blocks per lane in one part (when it divides D)
 #endif
@@ -572,7 +578,8 @@ __global__ void __launch_bounds__(32 * kPoolWarps, 1) search_pool_kernel(BatchAr
         constexpr uint32_t n_sb = decltype(nsb)::value;
         T base2[D];
         chunk_base(S.V, sb0 / D, base2);
-#pragma unroll
+        // at most two super-block bodies in the code (four thrash the instruction cache)
+#pragma unroll 2
         for (uint32_t j = 0; j < n_sb; ++j) {
           const uint32_t sb = sb0 + j;
           const T* r = S.V + ((Q - 5) * D + sb % D) * D;
