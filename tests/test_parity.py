@@ -555,3 +555,23 @@ def test_small_pinned_calls_zero_copy(torch_cuda, mapper):
     base, elig = workloads.constraints(77, 8, 7, 4)
     gi, gmp, gms = mapper.map_queues_constrained(pinned(K), pinned(X), pinned(base), pinned(elig))
     assert_same((gi.numpy(), gmp.numpy(), gms.numpy()), oracle.oracle_map_constrained(K, X, base, elig), "constrained")
+
+
+def test_u32_top_of_range_pooled_batch(torch_cuda, mapper):
+    """The SM-pooled batch kernel (path 12) at the top of the u32 range: a 400-epoch 8 x 4
+    batch mixing random epochs with epochs whose optimum equals the bound UB = 2^32 - 2
+    stays on the pooled u32 kernel and is exact; one more epoch at ms* = UB = 2^32 - 1 makes
+    the device flag the batch and the call rerun on 64-bit loads, still exact."""
+    Q, D, E = 8, 4, 400
+    K, X = workloads.random_tables(4040, E, Q, D)
+    for e in (0, 137, 399):
+        K[e], X[e] = (a[0] for a in _one_big_queue(1, Q, D, [U32_TOP - 1], big_q=e % Q))
+    want = oracle.oracle_map(K, X)
+    assert int(want[1][137]) == U32_TOP - 1
+    assert_same(run_gpu(torch_cuda, mapper, K, X, 7), want, "pooled, ms* = 2^32 - 2")
+    assert mapper.launch_info()["path"] == "batch_pool_u32"
+    K[250], X[250] = (a[0] for a in _one_big_queue(1, Q, D, [U32_TOP], big_q=3))
+    want = oracle.oracle_map(K, X)
+    assert int(want[1][250]) == U32_TOP
+    assert_same(run_gpu(torch_cuda, mapper, K, X, 7), want, "pooled batch with ms* = 2^32 - 1")
+    assert mapper.launch_info()["path"] == "blocked_u64"
