@@ -520,9 +520,11 @@ __global__ void __launch_bounds__(32 * kPoolWarps, 1) search_pool_kernel(BatchAr
       a.index[e] = idx;
       a.makespan[e] = (uint64_t)target;
     }
-    if (a.mapping && lane < Q) {
-      uint64_t rest = idx;
-      for (int q = Q - 1; q > lane; --q) rest /= D;
+    if (a.mapping && lane < Q) {  // D^Q < 2^32 for every pooled shape: 32-bit digits,
+      uint32_t rest = (uint32_t)idx;  // predicated constant divisions (no divergent loop)
+#pragma unroll
+      for (int q = Q - 1; q > 0; --q)
+        if (q > lane) rest /= D;
       a.mapping[e * Q + lane] = (uint8_t)(rest % D);
     }
   };
