@@ -333,6 +333,9 @@ constexpr int kPoolSlots = MCL_POOL_SLOTS;  // ring of per-epoch table slots
 #define MCL_POOL_AHEAD 12
 #endif
 constexpr int kPoolAhead = MCL_POOL_AHEAD;  // epochs prepared ahead of the claims
+#ifndef MCL_POOL_ZERO_COPY
+#define MCL_POOL_ZERO_COPY 0  // 1: the pooled form also for pinned host inputs read in place
+#endif
 #ifndef MCL_POOL_SBL
 #define MCL_POOL_SBL 2u  // super-blocks per lane in one part (when it divides D)
 #endif
@@ -644,7 +647,7 @@ cudaError_t launch_batch_t(const BatchArgs& a, int num_sms, cudaStream_t st, int
   // MCL_POOL_MIN_PER_SM (environment, tests / sanitizer runs): the smallest batch, in
   // epochs per SM, that takes the pooled form (a huge value keeps the warp-per-epoch form)
   static const int min_per_sm = env_int("MCL_POOL_MIN_PER_SM", kPoolMinPerSm, 1, 1 << 30);
-  if (MCL_BATCH_POOL && !a.host_inputs && a.E >= (uint64_t)num_sms * min_per_sm) {
+  if (MCL_BATCH_POOL && (MCL_POOL_ZERO_COPY || !a.host_inputs) && a.E >= (uint64_t)num_sms * min_per_sm) {
     // one 16-warp CTA per SM, epochs blockIdx.x + n * gridDim.x
     search_pool_kernel<Q, D><<<(unsigned)num_sms, 32 * kPoolWarps, 0, st>>>(a);
     *grid_out = num_sms;
