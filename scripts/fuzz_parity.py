@@ -24,7 +24,34 @@ paths = {}
 t0 = time.time()
 with Mapper(0) as m:
     while time.time() - t0 < budget:
-        kind = rng.integers(0, 4)
+        kind = rng.integers(0, 6)
+        if kind >= 4:  # constrained (mixed-radix kernels) and pruned calls vs the constrained oracle
+            Q, D = int(rng.integers(3, 11)), int(rng.integers(2, 9))
+            while D ** Q > 3e5:
+                Q -= 1
+            E = int(rng.choice([1, 4, 50, 700]))
+            hi = int(rng.choice([8, 1 << 12, 1 << 22]))
+            K = rng.integers(0, hi, size=(E, Q, D), dtype=np.uint64)
+            X = rng.integers(0, hi, size=(E, Q, D), dtype=np.uint64)
+            base = rng.integers(0, hi, size=(E, D), dtype=np.uint64)
+            elig = np.zeros((E, Q), np.uint16)
+            r = rng.random((E, Q))
+            elig[r < 0.25] = (1 << rng.integers(0, D, size=(E, Q))).astype(np.uint16)[r < 0.25]
+            sub = rng.integers(1, 1 << D, size=(E, Q)).astype(np.uint16)
+            elig[(r >= 0.25) & (r < 0.5)] = sub[(r >= 0.25) & (r < 0.5)]
+            args = [torch.from_numpy(a).cuda() for a in (K, X, base, elig)]
+            fn = m.map_queues_constrained if kind == 4 else m.map_queues_pruned
+            gi, gmp, gms = fn(*args)
+            path = ("constrained:" if kind == 4 else "pruned:") + m.launch_info()["path"]
+            wi, wms, wmp = oracle.oracle_map_constrained(K, X, base, elig)
+            ok = bool((gi.cpu().numpy() == wi).all() and (gms.cpu().numpy() == wms).all()
+                      and (gmp.cpu().numpy() == wmp).all())
+            cases += 1
+            paths[path] = paths.get(path, 0) + 1
+            if not ok:
+                fails += 1
+                print(json.dumps({"FAIL": True, "Q": Q, "D": D, "E": E, "hi": hi, "kind": int(kind), "path": path}), flush=True)
+            continue
         if kind == 0:  # batch shapes, pooled / warp / CTA kernels
             Q, D = BATCH[rng.integers(0, len(BATCH))]
             E = int(rng.choice([1, 5, 37, 150, 296, 333, 600, 1000]))
