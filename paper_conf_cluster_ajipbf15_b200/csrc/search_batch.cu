@@ -345,11 +345,7 @@ __device__ __forceinline__ void fence_cta() { asm volatile("fence.acq_rel.cta;" 
 #ifndef MCL_POOL_TAIL
 #define MCL_POOL_TAIL 1  // last ordinals of each CTA cut into single-super-block parts
 #endif
-#ifndef MCL_POOL_UNROLL
-#define MCL_POOL_UNROLL 1  // unroll of a lane's super-block loop within a part
-#endif
 constexpr int kPoolTail = MCL_POOL_TAIL;
-constexpr int kPoolUnroll = MCL_POOL_UNROLL;
 #ifndef MCL_POOL_MIN_PER_SM
 #define MCL_POOL_MIN_PER_SM 2
 #endif
