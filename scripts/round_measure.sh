@@ -8,6 +8,7 @@
 #   scaling.jsonl        projected strong scaling from per-rank shard kernels
 #   variants.jsonl       NEXT-1..4 variants (constrained, policies, pruned, cost tables)
 #   costs.jsonl          cost-table kernel, L2 flushed
+#   fuzz_parity.json     randomised GPU-vs-oracle sweep (120 s)
 cd "${GRAFT_REPO_ROOT:-$(dirname "$0")/..}"
 mkdir -p gpurun_out
 timeout 900 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err
@@ -24,4 +25,5 @@ timeout 300 python scripts/resident_latency.py > gpurun_out/resident_latency.jso
 timeout 600 python scripts/scaling_model.py > gpurun_out/scaling.jsonl 2>&1
 timeout 900 python scripts/bench_variants.py --reps 7 > gpurun_out/variants.jsonl 2>&1
 timeout 300 python scripts/bench_costs.py > gpurun_out/costs.jsonl 2>&1
+timeout 300 python scripts/fuzz_parity.py 120 $RANDOM > gpurun_out/fuzz_parity.json 2>&1
 echo done
