@@ -77,3 +77,8 @@ def test_default_bench_line_gpu():
         assert e["value"] > 0 and e["e2e"]["value"] > 0 and "roofline" in e and "clocks" in e, name
     assert d["roofline"]["bound"] == "alu" and 0 < d["roofline"]["frac"] < 1.05
     assert "frac_survey" in d["roofline"] and d["clocks"]["sm_mhz"]
+    # the live launch floor: an empty kernel costs more than the events alone, and far less
+    # than any search kernel the line reports
+    lf = d["launch_floor"]
+    assert 0 < lf["events_only_us"] < lf["empty_kernel_us"] < 50, lf
+    assert lf["empty_kernel_us"] * 1e-3 < d["configs"]["cfg1"]["roofline"]["kernel_ms"] * 1.5
