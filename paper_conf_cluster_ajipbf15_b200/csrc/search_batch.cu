@@ -342,6 +342,23 @@ constexpr int kPoolAhead = MCL_POOL_AHEAD;  // epochs prepared ahead of the clai
 // CTA-scope acquire/release fence for the shared-memory hand-offs between warps (lighter
 // than __threadfence_block's sequentially consistent MEMBAR.SC.CTA)
 __device__ __forceinline__ void fence_cta() { asm volatile("fence.acq_rel.cta;" ::: "memory"); }
+#ifndef MCL_POOL_ACQREL
+#define MCL_POOL_ACQREL 1  // release stores / acquire loads / acq_rel atomics instead of fences
+#endif
+__device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void st_release_cta(int* p, int v) {
+  asm volatile("st.release.cta.shared.b32 [%0], %1;" ::"r"(smem_addr(p)), "r"(v) : "memory");
+}
+__device__ __forceinline__ int ld_acquire_cta(const int* p) {
+  int v;
+  asm volatile("ld.acquire.cta.shared.b32 %0, [%1];" : "=r"(v) : "r"(smem_addr(p)) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t atom_add_acq_rel_cta(uint32_t* p, uint32_t v) {
+  uint32_t old;
+  asm volatile("atom.acq_rel.cta.shared.add.u32 %0, [%1], %2;" : "=r"(old) : "r"(smem_addr(p)), "r"(v) : "memory");
+  return old;
+}
 #ifndef MCL_POOL_TAIL
 #define MCL_POOL_TAIL 1  // last ordinals of each CTA cut into single-super-block parts
 #endif
@@ -414,7 +431,11 @@ __global__ void __launch_bounds__(32 * kPoolWarps, 1) search_pool_kernel(BatchAr
     if (lane < QD) { k0 = Ke[lane]; x0 = Xe[lane]; }
     if (lane + 32 < QD) { k1 = Ke[lane + 32]; x1 = Xe[lane + 32]; }
     if (lane == 0) {  // the slot's previous occupant (ordinal n - kPoolSlots) is finished
+#if MCL_POOL_ACQREL
+      while (ld_acquire_cta(&s_done[si]) != (int)n - kPoolSlots) __nanosleep(64);
+#else
       while (*(volatile int*)&s_done[si] != (int)n - kPoolSlots) __nanosleep(64);
+#endif
     }
     __syncwarp();
     bool bad = false;
@@ -457,8 +478,12 @@ __global__ void __launch_bounds__(32 * kPoolWarps, 1) search_pool_kernel(BatchAr
     }
     if (lane == 0) s_skip[si] = skip ? 1u : 0u;
     __syncwarp();
+#if MCL_POOL_ACQREL
+    if (lane == 0) st_release_cta(&s_ready[si], (int)n);
+#else
     fence_cta();
     if (lane == 0) *(volatile int*)&s_ready[si] = (int)n;
+#endif
   };
 
   auto chunk_base = [&](const T* V, uint32_t c, T (&bv)[D]) {
@@ -558,11 +583,18 @@ __global__ void __launch_bounds__(32 * kPoolWarps, 1) search_pool_kernel(BatchAr
     }
     const int si = (int)(n % kPoolSlots);
     if (p == 0 && n + kPoolAhead < n_ord) prepare(n + kPoolAhead);
+#if MCL_POOL_ACQREL
+    if (lane == 0) {
+      while (ld_acquire_cta(&s_ready[si]) != (int)n) __nanosleep(32);
+    }
+    __syncwarp();
+#else
     if (lane == 0) {
       while (*(volatile int*)&s_ready[si] != (int)n) __nanosleep(32);
     }
     __syncwarp();
     fence_cta();
+#endif
 #ifdef MCL_TRACE
     if (lane == 0 && b < 1024 && atomicExch(&s_first, 1u) == 0) g_mcl_ptrace[b][1] = btrace_ns();
 #endif
@@ -603,6 +635,12 @@ __global__ void __launch_bounds__(32 * kPoolWarps, 1) search_pool_kernel(BatchAr
       if (lane == 0) atomicMin(&s_key[si], ((unsigned long long)g << 32) | bsb);
     }
     uint32_t c = 0;
+#if MCL_POOL_ACQREL
+    if (lane == 0) c = atom_add_acq_rel_cta(&s_cnt[si], 1u);  // releases this part's key
+    c = __shfl_sync(0xffffffffu, c, 0);
+    if (c == parts - 1) {  // this warp completed the epoch (lane 0 acquired every part's key)
+      __syncwarp();
+#else
     if (lane == 0) {
       fence_cta();
       c = atomicAdd(&s_cnt[si], 1u);
@@ -610,14 +648,19 @@ __global__ void __launch_bounds__(32 * kPoolWarps, 1) search_pool_kernel(BatchAr
     c = __shfl_sync(0xffffffffu, c, 0);
     if (c == parts - 1) {  // this warp completed the epoch
       fence_cta();
+#endif
       const uint64_t key = *(volatile unsigned long long*)&s_key[si];
       if (!skip) finish(S, b + (uint64_t)n * G, key);
       __syncwarp();
       if (lane == 0) {
         s_key[si] = ~0ull;
         s_cnt[si] = 0;
+#if MCL_POOL_ACQREL
+        st_release_cta(&s_done[si], (int)n);
+#else
         fence_cta();
         *(volatile int*)&s_done[si] = (int)n;
+#endif
       }
     }
   }
