@@ -223,3 +223,36 @@ def test_pool_repeatable_under_load(torch_cuda, mapper):
     for idx, mp, ms in outs:
         assert (idx.cpu().numpy() == wi).all() and (ms.cpu().numpy() == wms).all()
         assert (mp.cpu().numpy() == wmp).all()
+
+
+def test_pool_concurrent_handles_on_two_streams(torch_cuda):
+    """Two handles on two CUDA streams, driven from two host threads, each repeating its
+    own batch: the pooled kernel keeps all its state in shared memory and the handles'
+    scratch is separate, so concurrent searches stay exact."""
+    torch = torch_cuda
+    K1, X1 = workloads.cfg2(E=3000, seed=31)
+    K2, X2 = workloads.small_int_tables(32, 2000, 9, 4, hi=50)
+    w1, w2 = oracle.oracle_map(K1, X1), oracle.oracle_map(K2, X2)
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    d1 = [torch.from_numpy(a).cuda() for a in (K1, X1)]
+    d2 = [torch.from_numpy(a).cuda() for a in (K2, X2)]
+    torch.cuda.synchronize()
+    import threading
+
+    results = {}
+
+    def worker(name, stream, dK, dX, reps):
+        with Mapper(0, stream=stream.cuda_stream) as m:
+            outs = []
+            for _ in range(reps):
+                outs.append(m.map_queues(dK, dX))
+                assert m.launch_info()["path"] == "batch_pool_u32"
+            results[name] = [tuple(t.cpu().numpy() for t in o) for o in outs]
+
+    t1 = threading.Thread(target=worker, args=("a", s1, *d1, 6))
+    t2 = threading.Thread(target=worker, args=("b", s2, *d2, 6))
+    t1.start(); t2.start(); t1.join(); t2.join()
+    for gi, gmp, gms in results["a"]:
+        check((gi, gmp, gms), w1, "handle a")
+    for gi, gmp, gms in results["b"]:
+        check((gi, gmp, gms), w2, "handle b")
