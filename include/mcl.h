@@ -295,7 +295,8 @@ mcl_status_t mcl_static_mappings(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint64
  * in pinned, device-mapped host memory; mcl_resident_map writes the inputs and a request
  * number into it and spins until the warp publishes the answer (no launch, no copy engine,
  * no stream synchronisation per call). Same definition and outputs as mcl_map_queues.
- *   Q, D        : fixed per start; D^Q <= 4096, Q <= 16, D <= 16.
+ *   Q, D        : fixed per start; D^Q <= 8192 (the paper's largest decision: FT, 8 queues on
+ *                 3 devices = 6561 mappings), Q <= 16, D <= 16.
  *   max_epochs  : epochs per mcl_resident_map call, 1..64.
  *   idle_ms     : the warp exits after this long without a request (0 = 100 ms); the next
  *                 mcl_resident_map relaunches it (one launch, then resident again).

@@ -300,7 +300,8 @@ struct ResidentBox {
   uint32_t pad2[16];
 };
 static_assert(sizeof(ResidentBox) == 192, "three 64-byte lines");
-constexpr uint32_t kResidentMaxMappings = 4096;  // D^Q per epoch (12 index bits)
+constexpr uint32_t kResidentMaxMappings = 8192;  // D^Q per epoch (13 index bits: the paper's
+                                                 // largest decision, FT's 8 queues x 3 devices = 6561)
 constexpr uint32_t kResidentMaxQ = 16, kResidentMaxD = 16;
 // Result record of one epoch, three u64 words each written whole by one store (single-copy
 // atomic at system scope), each tagged with the request number so the host accepts a
@@ -318,7 +319,6 @@ struct ResidentArgs {
   uint32_t seq0;              // request number already served when the warp starts
   uint64_t idle_ns;
 };
-size_t resident_smem_bytes(uint32_t Q, uint32_t D, uint32_t cap);
 cudaError_t launch_resident(const ResidentArgs& a, cudaStream_t st);
 
 // ALU throughput probe (probe.cu), SURVEY N7.

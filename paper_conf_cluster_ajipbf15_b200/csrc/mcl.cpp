@@ -1558,7 +1558,7 @@ mcl_status_t mcl_resident_start(mcl_mapper_t* h, uint32_t Q, uint32_t D, uint32_
   uint64_t N = 0;
   if (Q < 1 || D < 1 || Q > mcl::kResidentMaxQ || D > mcl::kResidentMaxD || max_epochs < 1 ||
       max_epochs > 64 || mul_overflow_pow(D, Q, mcl::kResidentMaxMappings, &N)) {
-    h->last_err = "resident mapper: needs D^Q <= 4096, Q <= 16, D <= 16, 1 <= max_epochs <= 64";
+    h->last_err = "resident mapper: needs D^Q <= 8192, Q <= 16, D <= 16, 1 <= max_epochs <= 64";
     return MCL_E_INVAL;
   }
   DeviceGuard g(h->device);

@@ -14,10 +14,12 @@
 // so the host accepts the answer without a fence or a separate done flag (kernels.h,
 // ResidentArgs). No launch, no copy engine, no stream synchronisation per decision.
 //
-// Shape: any Q <= 16, D <= 16 with D^Q <= 4096 (one warp; lane l scores mappings l, l + 32,
-// ... in increasing order keeping its first strict minimum, then five shuffle rounds of the
-// lexicographic (makespan, index) minimum). The warp exits when the host sets `stop`, or
-// after `idle_ns` without a request (the host relaunches it on demand).
+// Shape: any Q <= 16, D <= 16 with D^Q <= 8192: one warp up to 4096 mappings (lane l scores
+// mappings l, l + 32, ... in increasing order keeping its first strict minimum, then five
+// shuffle rounds of the lexicographic (makespan, index) minimum), 8 warps above (the same per
+// warp, then the warps' minima in shared memory; thread 0 alone polls the mailbox). The
+// kernel exits when the host sets `stop`, or after `idle_ns` without a request (the host
+// relaunches it on demand).
 #include "common.cuh"
 #include "kernels.h"
 
@@ -48,13 +50,18 @@ __device__ __forceinline__ uint64_t now_ns() {
 }
 
 // Lowest-index minimum makespan of one epoch (C = [Q][D] composed costs in shared memory),
-// by the 32 lanes: lane l scores m = l, l + 32, ... in increasing order (strict <), then
-// five shuffle rounds of the lexicographic (makespan, index) minimum. QT, DT > 0: shape
-// fixed at compile time (digits by constant division, loads in registers by static
-// selects); 0: runtime shape (loads in this lane's shared-memory row).
-template <int QT, int DT>
+// by the NT = 32 * W threads: thread t scores m = t, t + NT, ... in increasing order
+// (strict <), then five shuffle rounds of the lexicographic (makespan, index) minimum per
+// warp and, for W > 1, one more over the warps' results in shared memory (every thread
+// returns the epoch's result). QT, DT > 0: shape fixed at compile time (digits by constant
+// division, loads in registers by static selects); 0: runtime shape (loads in this
+// thread's shared-memory row).
+template <int QT, int DT, int W>
 __device__ __forceinline__ void score_epoch(const uint64_t* C, uint32_t Qr, uint32_t Dr, uint32_t N,
-                                            uint64_t* sL, uint64_t& best_ms, uint32_t& best_m) {
+                                            uint64_t* sL, uint64_t* s_wms, uint32_t* s_wm,
+                                            uint64_t& best_ms, uint32_t& best_m) {
+  constexpr uint32_t NT = 32u * W;
+  const uint32_t tid = threadIdx.x;
   const int lane = threadIdx.x & 31;
   uint64_t bms = ~0ull;
   uint32_t bm = 0xffffffffu;
@@ -64,7 +71,7 @@ __device__ __forceinline__ void score_epoch(const uint64_t* C, uint32_t Qr, uint
     for (int q = 0; q < QT; ++q)
 #pragma unroll
       for (int d = 0; d < DT; ++d) c[q][d] = C[q * DT + d];
-    for (uint32_t m = lane; m < N; m += 32) {
+    for (uint32_t m = tid; m < N; m += NT) {
       uint64_t L[DT];
 #pragma unroll
       for (int d = 0; d < DT; ++d) L[d] = 0;
@@ -79,13 +86,13 @@ __device__ __forceinline__ void score_epoch(const uint64_t* C, uint32_t Qr, uint
       uint64_t ms = L[0];
 #pragma unroll
       for (int d = 1; d < DT; ++d) ms = max(ms, L[d]);  // a4
-      if (ms < bms) {  // a5: strict, so the lane keeps its lowest index of a tie
+      if (ms < bms) {  // a5: strict, so the thread keeps its lowest index of a tie
         bms = ms;
         bm = m;
       }
     }
   } else {
-    for (uint32_t m = lane; m < N; m += 32) {
+    for (uint32_t m = tid; m < N; m += NT) {
       for (uint32_t d = 0; d < Dr; ++d) sL[d] = 0;
       uint32_t rest = m;
       for (int q = (int)Qr - 1; q >= 0; --q) {
@@ -110,27 +117,52 @@ __device__ __forceinline__ void score_epoch(const uint64_t* C, uint32_t Qr, uint
       bm = om;
     }
   }
+  if constexpr (W > 1) {  // across the warps (every warp's lane 0 holds its minimum)
+    const int w = (int)(tid >> 5);
+    if (lane == 0) {
+      s_wms[w] = bms;
+      s_wm[w] = bm;
+    }
+    __syncthreads();
+    bms = s_wms[0];
+    bm = s_wm[0];
+#pragma unroll
+    for (int v = 1; v < W; ++v) {
+      const uint64_t oms = s_wms[v];
+      const uint32_t om = s_wm[v];
+      if (oms < bms || (oms == bms && om < bm)) {
+        bms = oms;
+        bm = om;
+      }
+    }
+    __syncthreads();  // s_wms / s_wm are rewritten by the next epoch
+  }
   best_ms = bms;
   best_m = bm;
 }
 
 }  // namespace
 
-template <int QT, int DT>
-__global__ void __launch_bounds__(32) resident_kernel(ResidentArgs a) {
+template <int QT, int DT, int W>
+__global__ void __launch_bounds__(32 * W) resident_kernel(ResidentArgs a) {
   extern __shared__ __align__(16) uint64_t s_res[];
-  const int lane = threadIdx.x;
+  constexpr uint32_t NT = 32u * W;
+  const uint32_t tid = threadIdx.x;
   const uint32_t Q = QT > 0 ? QT : a.Q, D = DT > 0 ? DT : a.D, N = a.N, QD = Q * D;
-  uint64_t* sC = s_res;                                   // [cap][Q][D] composed costs
-  uint64_t* sL = s_res + (size_t)a.cap * QD + lane * 16;  // generic shapes: this lane's loads
+  uint64_t* sC = s_res;                                  // [cap][Q][D] composed costs
+  uint64_t* sL = s_res + (size_t)a.cap * QD + tid * 16;  // generic shapes: this thread's loads
+  __shared__ uint64_t s_req;                             // W > 1: the request, broadcast
+  __shared__ uint32_t s_quit;
+  __shared__ uint64_t s_wms[W];                          // W > 1: per-warp minima
+  __shared__ uint32_t s_wm[W];
   ResidentBox* box = a.box;
   uint32_t last = a.seq0;
   uint64_t t_idle = now_ns();
   for (;;) {
-    // ---- wait for a request: lane 0 polls one word (number, epochs, stop) over PCIe ----
+    // ---- wait for a request: thread 0 polls one word (number, epochs, stop) over PCIe ----
     uint64_t req = 0;
     uint32_t quit = 0;
-    if (lane == 0) {
+    if (tid == 0) {
       // one acquire load of the request word at a time: measured, several relaxed loads
       // in flight (4 or 8, staggered), a pause between polls, or polling tagged inputs
       // together with the request word only add latency (SS7, resident mapper)
@@ -147,10 +179,20 @@ __global__ void __launch_bounds__(32) resident_kernel(ResidentArgs a) {
         }
       }
     }
-    quit = __shfl_sync(0xffffffffu, quit, 0);
-    req = __shfl_sync(0xffffffffu, req, 0);
+    if constexpr (W == 1) {
+      quit = __shfl_sync(0xffffffffu, quit, 0);
+      req = __shfl_sync(0xffffffffu, req, 0);
+    } else {  // the other warps wait at the barrier (no polling of their own)
+      if (tid == 0) {
+        s_req = req;
+        s_quit = quit;
+      }
+      __syncthreads();
+      req = s_req;
+      quit = s_quit;
+    }
     if (quit) {
-      if (lane == 0) {
+      if (tid == 0) {
         box->exit_reason = quit;
         st_release_sys(&box->alive, 0u);
       }
@@ -166,38 +208,42 @@ __global__ void __launch_bounds__(32) resident_kernel(ResidentArgs a) {
     if (E > a.cap || E == 0) status |= kFlagBadModel;
     const uint32_t n = (E <= a.cap ? E : 0u) * QD;
     bool bad = false;
-    for (uint32_t i0 = lane; i0 < n; i0 += 4 * 32) {  // 8 loads in flight per lane (PCIe)
+    for (uint32_t i0 = tid; i0 < n; i0 += 4 * NT) {  // 8 loads in flight per thread (PCIe)
       uint64_t k[4], x[4];
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
-        const uint32_t i = i0 + 32 * u;
+        const uint32_t i = i0 + NT * u;
         k[u] = i < n ? ld_relaxed_sys64(a.K + i) : 0;
         x[u] = i < n ? ld_relaxed_sys64(a.X + i) : 0;
       }
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
-        const uint32_t i = i0 + 32 * u;
+        const uint32_t i = i0 + NT * u;
         bad |= (k[u] >= kEntryLimit) | (x[u] >= kEntryLimit);
         if (i < n) sC[i] = k[u] + x[u];
       }
     }
-    if (__any_sync(0xffffffffu, bad)) status |= kFlagRange;
-    __syncwarp();
+    if constexpr (W == 1) {
+      if (__any_sync(0xffffffffu, bad)) status |= kFlagRange;
+      __syncwarp();
+    } else {
+      if (__syncthreads_or(bad)) status |= kFlagRange;
+    }
 #ifdef MCL_RESIDENT_TRACE
     const uint64_t tr1 = now_ns();
 #endif
-    // digit width b: the smallest b with D <= 2^b (0 for D = 1); Q * b <= 16 here
+    // digit width b: the smallest b with D <= 2^b (0 for D = 1); Q * b <= 16 for D^Q <= 8192
     const uint32_t b = D <= 1 ? 0u : 32u - __clz(D - 1);
     for (uint32_t e = 0; e < (status == 0 ? E : 1u); ++e) {
       uint64_t ms = 0;
       uint32_t idx = 0;
-      if (status == 0) score_epoch<QT, DT>(sC + (size_t)e * QD, Q, D, N, sL, ms, idx);
+      if (status == 0) score_epoch<QT, DT, W>(sC + (size_t)e * QD, Q, D, N, sL, s_wms, s_wm, ms, idx);
       uint64_t* rec = a.rec + (size_t)e * kResidentRecWords;
-      if (lane == 0) {
+      if (tid == 0) {
         st_relaxed_sys64(rec + 0, ((uint64_t)seq << 32) | ((uint64_t)status << 16) | idx);
-      } else if (lane == 1) {
+      } else if (tid == 1) {
         st_relaxed_sys64(rec + 1, ((uint64_t)(seq & 0x7ffu) << 53) | ms);
-      } else if (lane == 2) {  // a7: digits of the index, queue 0 most significant
+      } else if (tid == 2) {  // a7: digits of the index, queue 0 most significant
         uint32_t rest = idx, packed = 0;
         for (int q = (int)Q - 1; q >= 0; --q) {
           packed |= (rest % D) << (q * b);
@@ -207,7 +253,7 @@ __global__ void __launch_bounds__(32) resident_kernel(ResidentArgs a) {
       }
     }
 #ifdef MCL_RESIDENT_TRACE
-    if (lane == 0) {
+    if (tid == 0) {
       box->trace[0] = tr0;
       box->trace[1] = tr1;
       box->trace[2] = now_ns();
@@ -218,30 +264,40 @@ __global__ void __launch_bounds__(32) resident_kernel(ResidentArgs a) {
   }
 }
 
-size_t resident_smem_bytes(uint32_t Q, uint32_t D, uint32_t cap) {
-  return ((size_t)cap * Q * D + 32 * 16) * sizeof(uint64_t);
-}
+// Decisions above kResidentWarpMappings (e.g. the paper's FT: 8 queues x 3 devices = 6561
+// mappings) are scored by 8 warps: one warp alone took 44 us per 8 x 3 decision, more than
+// a launch per call (19 us device-resident).
+constexpr uint32_t kResidentWarpMappings = 4096;
+constexpr int kResidentWide = 8;
 
 cudaError_t launch_resident(const ResidentArgs& a, cudaStream_t st) {
-  const size_t smem = resident_smem_bytes(a.Q, a.D, a.cap);
-  void (*k)(ResidentArgs) = resident_kernel<0, 0>;
-  switch (a.Q * 100 + a.D) {  // compile-time shapes of small decisions (cfg1: 4 x 3)
-#define MCL_RES_CASE(QQ, DD) \
-  case QQ * 100 + DD: k = resident_kernel<QQ, DD>; break;
+  const bool wide = a.N > kResidentWarpMappings;
+  void (*k)(ResidentArgs) = wide ? resident_kernel<0, 0, kResidentWide> : resident_kernel<0, 0, 1>;
+  bool generic = true;
+  switch (a.Q * 100 + a.D) {  // compile-time shapes of small decisions (cfg1: 4 x 3; FT: 8 x 3)
+#define MCL_RES_CASE(QQ, DD)                                                              \
+  case QQ * 100 + DD:                                                                     \
+    k = wide ? resident_kernel<QQ, DD, kResidentWide> : resident_kernel<QQ, DD, 1>;       \
+    generic = false;                                                                      \
+    break;
     MCL_RES_CASE(2, 2) MCL_RES_CASE(2, 3) MCL_RES_CASE(2, 4) MCL_RES_CASE(3, 2) MCL_RES_CASE(3, 3)
     MCL_RES_CASE(3, 4) MCL_RES_CASE(4, 2) MCL_RES_CASE(4, 3) MCL_RES_CASE(4, 4) MCL_RES_CASE(5, 3)
     MCL_RES_CASE(5, 4) MCL_RES_CASE(6, 3) MCL_RES_CASE(6, 4) MCL_RES_CASE(8, 2) MCL_RES_CASE(8, 3)
 #undef MCL_RES_CASE
     default: break;
   }
-  // the compile-time shapes need at most 64 x 8 x 4 entries + the lane rows (20 KB, under
-  // the default 48 KB); only the generic kernel may need the larger opt-in
-  if (k == resident_kernel<0, 0>) {
-    static SmemAttrCache cache;
-    cudaError_t err = ensure_smem(k, smem, cache);
+  const uint32_t threads = 32u * (wide ? kResidentWide : 1);
+  // composed costs of up to cap epochs, plus one 16-entry load row per thread for the
+  // generic (runtime-shape) kernel
+  const size_t smem = ((size_t)a.cap * a.Q * a.D + (generic ? threads * 16 : 0)) * sizeof(uint64_t);
+  // the compile-time shapes need at most 64 x 8 x 4 entries (16 KB, under the default
+  // 48 KB); only the generic kernels (one cache each) may need the larger opt-in
+  if (generic) {
+    static SmemAttrCache cache[2];
+    cudaError_t err = ensure_smem(k, smem, cache[wide ? 1 : 0]);
     if (err != cudaSuccess) return err;
   }
-  k<<<1, 32, smem, st>>>(a);
+  k<<<1, threads, smem, st>>>(a);
   return cudaGetLastError();
 }
 

@@ -533,7 +533,7 @@ class Mapper:
 
     def resident_start(self, Q: int, D: int, max_epochs: int = 1, idle_ms: int = 0) -> None:
         """Leave one warp resident for low-latency decisions (include/mcl.h
-        mcl_resident_start): D^Q <= 4096, max_epochs <= 64 per resident_map call. While it is
+        mcl_resident_start): D^Q <= 8192, max_epochs <= 64 per resident_map call. While it is
         resident, device-wide synchronisation waits for it (up to idle_ms): stop it first."""
         st = load_library().mcl_resident_start(self.handle, Q, D, max_epochs, idle_ms)
         if st != MCL_OK:

@@ -25,8 +25,14 @@ if "--lib" in argv:
     i = argv.index("--lib")
     mcl.load_library(os.path.abspath(argv[i + 1]))
     del argv[i:i + 2]
+shape = None
+if "--shape" in argv:  # e.g. --shape 8x3: the paper's FT-sized decision (8 queues, 3 devices)
+    i = argv.index("--shape")
+    shape = tuple(int(v) for v in argv[i + 1].split("x"))
+    del argv[i:i + 2]
 calls = int(argv[0]) if argv else 500
-K, X = workloads.make("cfg1")
+K, X = workloads.make("cfg1") if shape is None else workloads.cfg1_random(11, Q=shape[0], D=shape[1])
+label = "cfg1 decision latency" if shape is None else f"{shape[0]}x{shape[1]} decision latency"
 Kp, Xp = torch.from_numpy(K).pin_memory(), torch.from_numpy(X).pin_memory()
 Kd, Xd = Kp.cuda(), Xp.cuda()
 out = []
@@ -54,16 +60,16 @@ with Mapper(0) as m:
         m.resident_map(Kn, Xn, out=r_out)
         assert r_out[0][0] == ref[0][0] and r_out[2][0] == ref[2][0] and (r_out[1] == ref[1]).all()
         med, best = per_call(lambda: m.resident_map(Kn, Xn, out=r_out))
-        out.append({"measure": "cfg1 decision latency", "path": "resident", "lib": os.path.basename(mcl.LIB_PATH if not "--lib" in sys.argv else sys.argv[sys.argv.index("--lib") + 1]), "us_per_call_median": med,
+        out.append({"measure": label, "path": "resident", "lib": os.path.basename(mcl.LIB_PATH if not "--lib" in sys.argv else sys.argv[sys.argv.index("--lib") + 1]), "us_per_call_median": med,
                     "us_per_call_best_round": best})
     finally:
         m.resident_stop()
     med, best = per_call(lambda: m.map_queues_into(Kp, Xp, idx, mp, ms))
     assert idx[0] == ref[0][0] and ms[0] == ref[2][0]
-    out.append({"measure": "cfg1 decision latency", "path": "launch_host_pinned", "us_per_call_median": med,
+    out.append({"measure": label, "path": "launch_host_pinned", "us_per_call_median": med,
                 "us_per_call_best_round": best})
     med, best = per_call(lambda: m.map_queues_into(Kd, Xd, idx_d, mp_d, ms_d))
-    out.append({"measure": "cfg1 decision latency", "path": "launch_device_resident", "us_per_call_median": med,
+    out.append({"measure": label, "path": "launch_device_resident", "us_per_call_median": med,
                 "us_per_call_best_round": best})
 for o in out:
     print(json.dumps(o), flush=True)

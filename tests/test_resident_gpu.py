@@ -1,7 +1,7 @@
 """GPU parity of the resident mapper (include/mcl.h mcl_resident_*): one warp resident on
 the device serving decisions from a pinned host mailbox, against the CPU oracle, bit-exact
 (index, makespan, mapping) -- cfg1's shape and every other shape the mode accepts
-(D^Q <= 4096), tie-heavy tables, back-to-back calls, the idle exit and relaunch, and the
+(D^Q <= 8192, incl. the paper's FT-sized 8 x 3 decision), tie-heavy tables, back-to-back calls, the idle exit and relaunch, and the
 error cases."""
 from __future__ import annotations
 
@@ -35,7 +35,7 @@ def check(got, K, X, ctx=""):
     assert (gmp == wmp).all(), ctx
 
 
-SHAPES = [(1, 1), (1, 5), (2, 2), (3, 4), (4, 3), (5, 5), (6, 4), (12, 2), (3, 16), (7, 3), (16, 1)]
+SHAPES = [(1, 1), (1, 5), (2, 2), (3, 4), (4, 3), (5, 5), (6, 4), (12, 2), (3, 16), (7, 3), (16, 1), (8, 3), (13, 2)]
 
 
 @pytest.mark.parametrize("Q,D", SHAPES)
@@ -104,7 +104,7 @@ def test_resident_errors(torch_cuda):
     torch = torch_cuda
     with Mapper(0) as m:
         with pytest.raises(MclError) as ei:
-            m.resident_start(13, 2)  # 2^13 > 4096
+            m.resident_start(14, 2)  # 2^14 > 8192
         assert ei.value.status == MCL_E_INVAL
         with pytest.raises(MclError):
             m.resident_start(4, 17)
