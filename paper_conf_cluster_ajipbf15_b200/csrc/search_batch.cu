@@ -1,5 +1,9 @@
-// search_batch.cu -- batched exhaustive search, one WARP per epoch with compile-time
-// (Q, D) (cfg2: 8 queues x 4 devices x 10^4 epochs).
+// search_batch.cu -- batched exhaustive search with compile-time (Q, D) (
+// cfg2: 8 queues x 4 devices x 10^4 epochs), in two forms:
+//   * search_pool_kernel (below; the default for device-resident batches of >= 2 epochs per
+//     SM): one 16-warp CTA per SM whose warps claim sub-epoch parts of the SM's epochs;
+//   * search_batch_kernel (first): one WARP per epoch -- pinned host inputs read in place
+//     (its per-warp next-epoch prefetch hides PCIe latency) and smaller batches.
 //
 // Same scoring core as search_blocked.cu (blocked_core.cuh: the D^4 leaves of a
 // super-block folded into one running minimum, one integer max per mapping; PAPER.md
