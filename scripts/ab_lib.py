@@ -21,12 +21,19 @@ flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 st = torch.cuda.Stream(); torch.cuda.set_stream(st)
 out = {}
 for name in os.environ.get("AB_WORKLOADS", "cfg5,cfg4,cfg2").split(","):
-    K, X = workloads.make(name); Kd, Xd = torch.from_numpy(K).cuda(), torch.from_numpy(X).cuda()
+    cons = name.endswith("c")  # e.g. cfg2c: 25 % pinned + 25 % masked queues (NEXT-3)
+    K, X = workloads.make(name.rstrip("c")); Kd, Xd = torch.from_numpy(K).cuda(), torch.from_numpy(X).cuda()
+    if cons:
+        base, elig = workloads.constraints(77, *K.shape)
+        Bd, Ed = torch.from_numpy(base).cuda(), torch.from_numpy(elig).cuda()
     for G in ((1, 8) if name in ("cfg4", "cfg5") else (1,)):
         with mcl.Mapper(0, stream=st.cuda_stream, rank=0, world=G) as m:
             m.set_timing(True, hold_us=200); ts = []
             for i in range(int(os.environ.get("AB_N", "9"))):
-                flush.fill_(i); flush.view(torch.int64).sum(); m.map_queues(Kd, Xd); ts.append(m.last_kernel_time_ms()[0])
+                flush.fill_(i); flush.view(torch.int64).sum()
+                if cons: m.map_queues_constrained(Kd, Xd, Bd, Ed)
+                else: m.map_queues(Kd, Xd)
+                ts.append(m.last_kernel_time_ms()[0])
         # AB_STAT=mean: the CUDA-event clock of some boxes ticks in ~1 us steps, so a mean
         # over many launches resolves differences a median of a few cannot
         stat = statistics.mean if os.environ.get("AB_STAT") == "mean" else statistics.median
